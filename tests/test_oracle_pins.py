@@ -1,0 +1,377 @@
+"""Pins for the CPU oracle (SURVEY.md §8(c) table "What pins each part"), CPU only.
+
+Each test ties the oracle to something other than itself: published known-answer vectors, exact
+counting identities, closed-form Markov / PPR distributions (matrix powers and a linear solve),
+the geometric length law, brute force on tiny inputs. A plausible slip anywhere in oracle.c (a
+swapped Philox lane, a wrong key bump, an off-by-one in t, a biased range reduction, a wrong
+termination order) fails at least one of these.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+from scipy import stats
+
+import lt_inputs
+import oracle as O
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+P_MIN = 1e-4  # chi-square acceptance; seeds are fixed, so every run is deterministic
+
+
+def _h(s):
+    return int(s, 16)
+
+
+# ---------------------------------------------------------------- P1: Philox known answers
+def test_p1_philox_kat():
+    kat = json.load(open(os.path.join(GOLDEN, "philox_kat.json")))
+    for v in kat["vectors"]:
+        out = O.philox4x32_10([_h(x) for x in v["ctr"]], [_h(x) for x in v["key"]])
+        assert out == [_h(x) for x in v["out"]]
+
+
+# ---------------------------------------------------------------- P3: worked example
+def test_p3_worked_example_first_hop():
+    g = json.load(open(os.path.join(GOLDEN, "worked_example_p3.json")))
+    assert O.philox4x32_10([0, 0, 0, 0], [0, 0]) == g["block0"]
+    T = O.ppr_threshold(0.15)
+    assert T == g["ppr_threshold_alpha_0_15"]
+    assert (g["block0"][0] >= T) == g["ppr_moves_at_t0"]
+    for d_s, idx in g["lemire_first_index"].items():
+        d = int(d_s)
+        got, used = O.lemire(0, 0, 0, d)
+        assert (got, used) == (idx, 1)
+        # On a star whose centre 0 has neighbours 1..d, walk 0 (seed 0) must hop to idx+1, for
+        # DeepWalk and for PPR (which moves at t=0 per the golden coin).
+        star = lt_inputs.small_graph([(0, k) for k in range(1, d + 1)])
+        for app in (O.DEEPWALK, O.PPR):
+            paths, lengths, _, _ = O.walks(star.row_ptr, star.col, np.array([0], np.uint32), app=app,
+                                           length=1, alpha=0.15, seed=0)
+            assert paths[0, 0] == 0 and paths[0, 1] == idx + 1
+
+
+def test_ppr_threshold_values():
+    assert O.ppr_threshold(0.15) == 644245094          # floor(0.15 * 2^32) (reading R5)
+    assert O.ppr_threshold(0.5) == 2 ** 31
+    assert O.ppr_threshold(0.0) == 0
+    assert O.ppr_threshold(2.0 ** -32) == 1
+
+
+# ---------------------------------------------------------------- P4: Lemire exactness
+@pytest.mark.parametrize("d", [1, 3, 7, 1000, 65536, 1_000_003])
+def test_p4_lemire_exhaustive(d):
+    hist, rej = O.lemire_exhaustive(d)
+    # every residue is hit exactly floor(2^32/d) times; exactly 2^32 mod d words are rejected
+    assert np.all(hist == (2 ** 32) // d)
+    assert rej == (2 ** 32) % d
+
+
+def test_p4_lemire_power_of_two_is_top_bits():
+    rng = np.random.default_rng(5)
+    for k in (1, 4, 13, 31):
+        d = 2 ** k
+        for x in rng.integers(0, 2 ** 32, size=200, dtype=np.uint64):
+            ok, idx = O.lemire_accept(int(x), d)
+            assert ok and idx == int(x) >> (32 - k)
+
+
+def test_lemire_rejection_consumes_next_words_in_stream_order():
+    # d = 2^31 + 1 rejects about half of all words, so the word stream order matters.
+    d = 2 ** 31 + 1
+    seen_multi = 0
+    for w in range(200):
+        idx, used = O.lemire(7, w, 3, d)
+        blk0 = O.philox4x32_10([3, 0, w, 0], [7, 0])
+        blk1 = O.philox4x32_10([3, 1, w, 0], [7, 0])
+        stream = blk0[1:] + blk1            # x1,x2,x3 of block 0 then x0..x3 of block 1
+        for i, x in enumerate(stream):
+            ok, j = O.lemire_accept(x, d)
+            if ok:
+                assert (idx, used) == (j, i + 1)
+                break
+        seen_multi += used > 1
+    assert seen_multi > 50
+
+
+# ---------------------------------------------------------------- P5 / P9: path invariants
+def _is_edge(g, u, v):
+    a = g.col[int(g.row_ptr[u]):int(g.row_ptr[u + 1])]
+    i = np.searchsorted(a, v)
+    return i < len(a) and a[i] == v
+
+
+@pytest.fixture(scope="module")
+def rmat12():
+    return lt_inputs.rmat_cpu(12, 65536, seed=1)
+
+
+def test_p5_p9_deepwalk_edges_and_lengths(rmat12):
+    g = rmat12
+    W, l = 4096, 10
+    starts = lt_inputs.deepwalk_starts(W, g.n)
+    paths, lengths, steps, trunc = O.walks(g.row_ptr, g.col, starts, app=O.DEEPWALK, length=l, seed=1)
+    assert np.all(lengths == l + 1) and steps == W * l and trunc == 0
+    assert np.all(paths[:, 0] == starts)
+    for w in range(0, W, 7):
+        for t in range(l):
+            assert _is_edge(g, paths[w, t], paths[w, t + 1])
+
+
+def test_p5_ppr_edges_and_padding(rmat12):
+    g = rmat12
+    W = 4096
+    starts = lt_inputs.ppr_starts(W, g.argmax_deg)
+    paths, lengths, steps, trunc = O.walks(g.row_ptr, g.col, starts, app=O.PPR, alpha=0.15, seed=3)
+    assert steps == int((lengths.astype(np.int64) - 1).sum())
+    for w in range(W):
+        L = lengths[w]
+        assert np.all(paths[w, L:] == O.EMPTY) and np.all(paths[w, :L] != O.EMPTY)
+        for t in range(L - 1):
+            assert _is_edge(g, paths[w, t], paths[w, t + 1])
+
+
+def test_dead_end_and_zero_length():
+    g = lt_inputs.small_graph([(0, 1)], n=3)          # vertex 2 isolated (d == 0, reading R9)
+    paths, lengths, _, _ = O.walks(g.row_ptr, g.col, np.array([2, 0], np.uint32), app=O.DEEPWALK, length=5)
+    assert list(lengths) == [1, 6]
+    assert list(paths[1]) == [0, 1, 0, 1, 0, 1]
+    paths, lengths, _, _ = O.walks(g.row_ptr, g.col, np.array([0], np.uint32), app=O.DEEPWALK, length=0)
+    assert list(lengths) == [1] and paths.shape == (1, 1)
+
+
+def test_ppr_truncation_at_lmax():
+    g = lt_inputs.small_graph([(0, 1), (1, 2), (2, 0)])
+    W = 500
+    # alpha = 2^-32 -> T = 1: the coin x0 < 1 essentially never fires, so every walk is capped.
+    paths, lengths, steps, trunc = O.walks(g.row_ptr, g.col, np.zeros(W, np.uint32), app=O.PPR,
+                                           alpha=2.0 ** -32, lmax=5)
+    assert np.all(lengths == 6) and trunc == W and steps == 5 * W
+
+
+# ---------------------------------------------------------------- P6: uniform neighbour
+def test_p6_neighbour_uniformity_chi2(rmat12):
+    g = rmat12
+    hub = g.argmax_deg
+    d = int(g.row_ptr[hub + 1] - g.row_ptr[hub])
+    W = 200 * d
+    paths, _, _, _ = O.walks(g.row_ptr, g.col, np.full(W, hub, np.uint32), app=O.DEEPWALK, length=1, seed=11)
+    nb = g.col[int(g.row_ptr[hub]):int(g.row_ptr[hub + 1])]
+    idx = np.searchsorted(nb, paths[:, 1])
+    counts = np.bincount(idx, minlength=d)
+    assert counts.sum() == W
+    p = stats.chisquare(counts).pvalue
+    assert p > P_MIN, p
+
+
+# ---------------------------------------------------------------- P7: closed forms
+TINY = {
+    "star": [(0, k) for k in range(1, 6)],
+    "cycle5": [(k, (k + 1) % 5) for k in range(5)],
+    "k4": [(a, b) for a in range(4) for b in range(a + 1, 4)],
+    "irregular6": [(0, 1), (0, 2), (1, 2), (2, 3), (3, 4), (3, 5), (4, 5), (1, 4)],
+}
+
+
+def _transition(g):
+    n = g.n
+    A = np.zeros((n, n))
+    for u in range(n):
+        for v in g.col[int(g.row_ptr[u]):int(g.row_ptr[u + 1])]:
+            A[u, v] = 1.0
+    return A / A.sum(axis=1, keepdims=True)
+
+
+def _chi2_against(counts, probs):
+    probs = np.asarray(probs, dtype=float)
+    zero = probs < 1e-15
+    assert np.all(counts[zero] == 0), "walk reached an unreachable vertex"
+    counts, probs = counts[~zero], probs[~zero] / probs[~zero].sum()
+    if len(counts) == 1:
+        return 1.0
+    return stats.chisquare(counts, probs * counts.sum()).pvalue
+
+
+@pytest.mark.parametrize("name", sorted(TINY))
+@pytest.mark.parametrize("t", [1, 3, 8])
+def test_p7_deepwalk_endpoint_is_matrix_power(name, t):
+    g = lt_inputs.small_graph(TINY[name])
+    P = _transition(g)
+    s = 0 if name != "irregular6" else 2
+    W = 200_000
+    paths, lengths, _, _ = O.walks(g.row_ptr, g.col, np.full(W, s, np.uint32), app=O.DEEPWALK, length=t,
+                                   seed=100 + t)
+    expect = np.linalg.matrix_power(P, t)[s]
+    counts = np.bincount(paths[:, t], minlength=g.n)
+    assert _chi2_against(counts, expect) > P_MIN
+
+
+@pytest.mark.parametrize("name", sorted(TINY))
+def test_p7_ppr_endpoint_is_textbook_ppr_vector(name):
+    g = lt_inputs.small_graph(TINY[name])
+    P = _transition(g)
+    alpha = 0.15
+    s = 1
+    # PPR vector (Fogaras et al., cited at PAPER.md:287): pi = alpha e_s (I - (1-alpha) P)^-1
+    e = np.zeros(g.n)
+    e[s] = 1.0
+    pi = alpha * np.linalg.solve((np.eye(g.n) - (1 - alpha) * P).T, e)
+    W = 200_000
+    paths, lengths, _, trunc = O.walks(g.row_ptr, g.col, np.full(W, s, np.uint32), app=O.PPR, alpha=alpha,
+                                       seed=7)
+    assert trunc == 0
+    ends = paths[np.arange(W), lengths - 1]
+    assert abs(pi.sum() - 1) < 1e-12
+    assert _chi2_against(np.bincount(ends, minlength=g.n), pi) > P_MIN
+
+
+# ---------------------------------------------------------------- P8: PPR length law
+def test_p8_ppr_length_is_geometric():
+    g = lt_inputs.small_graph(TINY["k4"])
+    alpha = 0.15
+    W = 300_000
+    _, lengths, _, trunc = O.walks(g.row_ptr, g.col, np.zeros(W, np.uint32), app=O.PPR, alpha=alpha, seed=9)
+    assert trunc == 0
+    N = lengths.astype(np.int64)               # path vertices, N ~ Geometric(alpha) on {1,2,...}
+    K = 40
+    obs = np.bincount(np.minimum(N, K), minlength=K + 1)[1:]
+    pmf = (1 - alpha) ** (np.arange(1, K) - 1) * alpha
+    probs = np.append(pmf, 1 - pmf.sum())
+    assert stats.chisquare(obs, probs * W).pvalue > P_MIN
+    mean, sd = N.mean(), np.sqrt((1 - alpha) / alpha ** 2 / W)
+    assert abs(mean - 1 / alpha) < 4 * sd
+
+
+# ---------------------------------------------------------------- P10: brute force, synchronous
+_M0, _M1, _W0, _W1 = 0xD2511F53, 0xCD9E8D57, 0x9E3779B9, 0xBB67AE85
+_MASK = np.uint64(0xFFFFFFFF)
+
+
+def _np_philox(c0, c1, c2, c3, k0, k1):
+    """Vectorised Philox4x32-10 over uint64 arrays holding u32 lanes (independent re-implementation
+    for the synchronous brute force; itself checked against the KATs below)."""
+    c0, c1, c2, c3 = (np.asarray(x, dtype=np.uint64) for x in (c0, c1, c2, c3))
+    k0, k1 = np.uint64(k0), np.uint64(k1)
+    for r in range(10):
+        if r:
+            k0 = (k0 + np.uint64(_W0)) & _MASK
+            k1 = (k1 + np.uint64(_W1)) & _MASK
+        p0 = np.uint64(_M0) * c0
+        p1 = np.uint64(_M1) * c2
+        c0, c1, c2, c3 = (p1 >> np.uint64(32)) ^ c1 ^ k0, p1 & _MASK, (p0 >> np.uint64(32)) ^ c3 ^ k1, p0 & _MASK
+    return c0, c1, c2, c3
+
+
+def test_np_philox_matches_kat():
+    kat = json.load(open(os.path.join(GOLDEN, "philox_kat.json")))
+    for v in kat["vectors"]:
+        c = [np.array([_h(x)], dtype=np.uint64) for x in v["ctr"]]
+        k = [_h(x) for x in v["key"]]
+        out = _np_philox(*c, *k)
+        assert [int(o[0]) for o in out] == [_h(x) for x in v["out"]]
+
+
+def _sync_simulator(g, starts, app, length, alpha, lmax, seed):
+    """All walks advance together, one global step at a time (different loop structure from the
+    per-walk oracle; same definition)."""
+    W = len(starts)
+    stride = length + 1 if app == O.DEEPWALK else lmax + 1
+    paths = np.full((W, stride), O.EMPTY, dtype=np.uint64)
+    v = starts.astype(np.uint64)
+    paths[:, 0] = v
+    alive = np.ones(W, dtype=bool)
+    t_len = np.ones(W, dtype=np.int64)
+    T = np.uint64(int(np.floor(alpha * 2.0 ** 32))) if app == O.PPR else None
+    rp = g.row_ptr.astype(np.uint64)
+    wid = np.arange(W, dtype=np.uint64)
+    for t in range(stride - 1 + 1):
+        if app == O.DEEPWALK and t == length:
+            break
+        if app == O.PPR and t == lmax:
+            break
+        idx = np.nonzero(alive)[0]
+        if len(idx) == 0:
+            break
+        ww = wid[idx]
+        b = _np_philox(np.full(len(idx), t), np.zeros(len(idx)), ww & _MASK, ww >> np.uint64(32),
+                       seed & 0xFFFFFFFF, seed >> 32)
+        if app == O.PPR:
+            stop = b[0] < T
+            alive[idx[stop]] = False
+            idx, b = idx[~stop], tuple(x[~stop] for x in b)
+        d = rp[v[idx] + np.uint64(1)] - rp[v[idx]]
+        dead = d == 0
+        alive[idx[dead]] = False
+        idx, d, b = idx[~dead], d[~dead], tuple(x[~dead] for x in b)
+        choice = np.zeros(len(idx), dtype=np.uint64)
+        done = np.zeros(len(idx), dtype=bool)
+        thr = (np.uint64(2 ** 32) % d)
+        words = [b[1], b[2], b[3]]
+        j = 0
+        while not done.all():
+            if not words:
+                j += 1
+                nb = _np_philox(np.full(len(idx), t), np.full(len(idx), j), wid[idx] & _MASK,
+                                wid[idx] >> np.uint64(32), seed & 0xFFFFFFFF, seed >> 32)
+                words = list(nb)
+            x = words.pop(0)
+            m = x * d
+            acc = (~done) & ((m & _MASK) >= thr)
+            choice[acc] = m[acc] >> np.uint64(32)
+            done |= acc
+        v[idx] = g.col[(rp[v[idx]] + choice).astype(np.int64)].astype(np.uint64)
+        paths[idx, t + 1] = v[idx]
+        t_len[idx] = t + 2
+    return paths.astype(np.uint32), t_len.astype(np.uint32)
+
+
+@pytest.mark.parametrize("app", [O.DEEPWALK, O.PPR])
+def test_p10_brute_force_synchronous_equals_oracle(app):
+    g = lt_inputs.rmat_cpu(10, 16 * 1024, seed=4)
+    W = 3000
+    starts = lt_inputs.deepwalk_starts(W, g.n) if app == O.DEEPWALK else lt_inputs.ppr_starts(W, g.argmax_deg)
+    kw = dict(app=app, length=12, alpha=0.3, lmax=20, seed=0x1234_5678_9ABC)
+    po, lo, _, _ = O.walks(g.row_ptr, g.col, starts, **kw)
+    ps, ls = _sync_simulator(g, starts, kw["app"], kw["length"], kw["alpha"], kw["lmax"], kw["seed"])
+    np.testing.assert_array_equal(lo, ls)
+    np.testing.assert_array_equal(po, ps)
+
+
+def test_p10_brute_force_with_rejections():
+    # a vertex of degree 2^31+1 cannot be built; instead force many rejections with a multigraph-free
+    # trick: compare Lemire on huge d directly against the synchronous word loop for one step.
+    d = np.uint64(2 ** 31 + 1)
+    for w in range(64):
+        idx, used = O.lemire(99, w, 5, int(d))
+        b = _np_philox([5], [0], [w], [0], 99, 0)
+        words, j = [b[1], b[2], b[3]], 0
+        thr = np.uint64(2 ** 32) % d
+        while True:
+            if not words:
+                j += 1
+                words = list(_np_philox([5], [j], [w], [0], 99, 0))
+            x = words.pop(0)
+            m = x * d
+            if (m & _MASK)[0] >= thr:
+                assert int(m[0] >> np.uint64(32)) == idx
+                break
+
+
+# ---------------------------------------------------------------- determinism
+def test_oracle_thread_count_independent(rmat12):
+    g = rmat12
+    starts = lt_inputs.deepwalk_starts(5000, g.n)
+    a = O.walks(g.row_ptr, g.col, starts, length=15, threads=1)
+    b = O.walks(g.row_ptr, g.col, starts, length=15, threads=4)
+    np.testing.assert_array_equal(a[0], b[0])
+
+
+def test_oracle_ids_subset_equals_full(rmat12):
+    g = rmat12
+    W = 4096
+    starts = lt_inputs.deepwalk_starts(W, g.n)
+    full, fl, _, _ = O.walks(g.row_ptr, g.col, starts, length=10, seed=5)
+    ids = np.array([0, 17, 4095, 2048], dtype=np.uint64)
+    sub, sl, _, _ = O.walks(g.row_ptr, g.col, starts[ids.astype(np.int64)], length=10, seed=5, ids=ids)
+    np.testing.assert_array_equal(sub, full[ids.astype(np.int64)])
