@@ -1,0 +1,426 @@
+#!/usr/bin/env python3
+"""Benchmark of the B200-native LightTraffic walk-update path (one JSON line on rank 0).
+
+A "step" is one pass of the whole hot path over one batch of synthetic input: lt_walks_init (walk
+records + path[w][0] + insertion into the start partitions' buckets, §8(a) a2/a5) followed by
+lt_run (partition scheduler + walk-update/insertion kernels until every walk has terminated,
+a3-a7). Workload (default): BASELINE.json configs[3], the Friendster-shaped R-MAT graph at scale 26
+(1.8B tuples) with |V| DeepWalk walks of length 80 on one B200, HBM-resident.
+
+  value     walk steps/s with inputs (graph, starts) resident in HBM, device-timed with CUDA events
+            on the stream the library launches on, max over ranks.
+  e2e       the same metric through the C ABI with HOST buffers: pinned starts copied H2D inside
+            lt_walks_init, and every path and length copied D2H by lt_get_paths, per step.
+  roofline  the update kernel (the dominant kernel): algorithmic bytes per launch (DESIGN.md
+            "Roofline": 32 B row_ptr sector + 32 B col sector + 4 B path entry per step, 16 B record
+            read per visit, 16 B record write per partition change, 4 B length per finished walk)
+            / its CUDA-event-timed average launch duration, against MEASURED_PEAKS.json hbm_gbs.
+  cpu_baseline  the CPU oracle (oracle/, as it stands) on this box's host cores over a bounded
+            sample of the same workload's walks (rank 0, N=1 only).
+
+Multi-GPU (torchrun, N>1): "replicas" mode — every rank holds the whole graph and runs its own |V|
+walks (walk IDs offset by rank*|V|): no data-path collective, weak scaling.
+`--impl reference` times the oracle (the reference arm of this tier) on the host cores instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import lt_inputs  # noqa: E402
+
+METRIC = "walk steps/sec (device-timed, max over ranks) at 1/2/4/8 B200; HBM GB/s vs peak"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="lt", choices=["lt", "reference"])
+    ap.add_argument("--config", type=int, default=4, help="BASELINE.json configs[i-1]")
+    ap.add_argument("--scale", type=int, default=None, help="override the config's R-MAT scale")
+    ap.add_argument("--tuples", type=int, default=None)
+    ap.add_argument("--partitions", type=int, default=None, help="P; default per DESIGN.md")
+    ap.add_argument("--chunk-walks", type=int, default=8192)
+    ap.add_argument("--policy", type=int, default=0)
+    ap.add_argument("--insert-mode", type=int, default=0)
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--sweep", default="", help="comma list of P values to time (extra key)")
+    return ap.parse_args()
+
+
+DEFAULT_P = {1: 4, 2: 1, 3: 1, 4: 1, 5: 1}
+
+
+def workload(args):
+    c = dict(lt_inputs.CONFIGS[args.config])
+    if args.scale is not None:
+        c["scale"] = args.scale
+    if args.tuples is not None:
+        c["tuples"] = args.tuples
+    c["partitions"] = args.partitions if args.partitions is not None else (c.get("partitions") or DEFAULT_P[args.config])
+    return c
+
+
+def app_param(c):
+    import paper_conf_icde_xing0wxl23_b200 as LT
+    if c["app"] == "deepwalk":
+        return LT.DEEPWALK, float(c["length"])
+    return LT.PPR, float(c["alpha"])
+
+
+def starts_for(c, g, W, first):
+    if c["app"] == "deepwalk":
+        return lt_inputs.deepwalk_starts(W, g.n, first_walk_id=first)
+    return lt_inputs.ppr_starts(W, g.argmax_deg)
+
+
+def num_walks(c, g):
+    return 4096 if c["walks"] == "4096" else g.n
+
+
+# ------------------------------------------------------------------------------ clocks sampling
+class Clocks:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(device), f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm = [float(r[1]) for r in rows if len(r) >= 9 and r[1].strip().replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in rows if len(r) >= 9 and r[2].strip().replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            if len(r) < 9:
+                continue
+            for nm, val in zip(names, r[5:9]):
+                if "Active" in val and "Not" not in val:
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------ CPU oracle legs
+def oracle_sample(c, g_host, W, first, seconds, threads=0):
+    """Time the oracle (as it stands) on a bounded prefix sample of the workload's walks."""
+    import oracle as O
+    app = O.DEEPWALK if c["app"] == "deepwalk" else O.PPR
+    kw = dict(app=app, length=int(c.get("length", 0)), alpha=float(c.get("alpha", 0.15)), seed=c["seed"],
+              threads=threads)
+    # calibrate on a small prefix, then size the sample for ~`seconds` of work
+    n0 = min(W, 20_000)
+    st = starts_for(c, g_host, n0, first)
+    t0 = time.perf_counter()
+    O.walks(g_host.row_ptr, g_host.col, st, ids=np.arange(first, first + n0, dtype=np.uint64), **kw)
+    dt = max(time.perf_counter() - t0, 1e-4)
+    ns = int(min(W, max(n0, n0 * seconds / dt)))
+    ids = np.arange(first, first + ns, dtype=np.uint64)
+    st = starts_for(c, g_host, ns, first)
+    t0 = time.perf_counter()
+    paths, lengths, steps, _ = O.walks(g_host.row_ptr, g_host.col, st, ids=ids, **kw)
+    dt = time.perf_counter() - t0
+    return dict(value=steps / dt, steps=steps, seconds=dt, walks=ns, paths=paths, lengths=lengths)
+
+
+def host_graph(g):
+    if isinstance(g.row_ptr, np.ndarray):
+        return g
+    return lt_inputs.Graph(g.n, g.m, g.row_ptr.cpu().numpy().view(np.uint64), g.col.cpu().numpy().view(np.uint32),
+                           g.max_deg, g.argmax_deg)
+
+
+def make_graph(c, device):
+    import torch
+    if c["scale"] <= 16:
+        g = lt_inputs.rmat_cpu(c["scale"], c["tuples"], seed=c.get("graph_seed", 1), permute=c["permute"])
+        return lt_inputs.Graph(g.n, g.m, torch.from_numpy(g.row_ptr.view(np.int64)).cuda(device),
+                               torch.from_numpy(g.col.view(np.int32)).cuda(device), g.max_deg, g.argmax_deg)
+    return lt_inputs.rmat_gpu(c["scale"], c["tuples"], seed=c.get("graph_seed", 1), permute=c["permute"],
+                              device=device)
+
+
+def cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
+def cfg_json(c, g, W, extra):
+    d = {"workload": f"{c['name']} (BASELINE.json configs[{c['idx'] - 1}])", "scale": c["scale"],
+         "rmat_tuples": c["tuples"], "kronecker": bool(c["permute"]), "vertices": g.n, "csr_entries": g.m,
+         "walks_per_gpu": W, "app": c["app"]}
+    if c["app"] == "deepwalk":
+        d["length"] = c["length"]
+    else:
+        d["alpha"] = c["alpha"]
+    d.update(extra)
+    return d
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    c = workload(args)
+    c["idx"] = args.config
+    c["seed"] = args.seed
+    g = lt_inputs.rmat_cpu(c["scale"], c["tuples"], seed=1, permute=c["permute"]) if c["scale"] <= 22 else None
+    if g is None:
+        import torch
+        torch.cuda.set_device(0)
+        g = host_graph(make_graph(c, 0))
+    W = num_walks(c, g)
+    per = max(1.0, 120.0 / max(1, args.steps + args.warmup))  # whole run within a few minutes
+    for _ in range(args.warmup):
+        oracle_sample(c, g, W, 0, min(per, 3.0))
+    vals, steps_all, secs = [], 0, 0.0
+    ns = None
+    for _ in range(args.steps):
+        r = oracle_sample(c, g, W, 0, per)
+        vals.append(r["value"])
+        steps_all += r["steps"]
+        secs += r["seconds"]
+        ns = r["walks"]
+    value = steps_all / secs
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "steps/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * secs / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic", "config": cfg_json(c, g, W, {"partitions": None}),
+            "cpu_baseline": {"value": value, "unit": "steps/s", "cores": cores(), "kind": "oracle",
+                             "sample": f"walks 0..{ns - 1} of the workload per step (oracle/ C + OpenMP)"},
+            "e2e": {"value": value, "unit": "steps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------ CUDA arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icde_xing0wxl23_b200 as LT
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    c = workload(args)
+    c["idx"] = args.config
+    c["seed"] = args.seed
+    P = c["partitions"]
+    t0 = time.time()
+    g = make_graph(c, local)
+    gen_s = time.time() - t0
+    W = num_walks(c, g)
+    first = rank * W
+    app, param = app_param(c)
+    starts_h = starts_for(c, g, W, first)
+    starts_d = torch.from_numpy(starts_h.view(np.int32)).cuda(local)
+
+    eng = LT.Engine(device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
+                    timing=True)
+    eng.graph_load(g.row_ptr, g.col, P)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+            torch.cuda.synchronize()
+
+    def one_step():
+        eng.walks_init(starts_d, app, param, args.seed, first)
+        eng.run()
+        return eng.stats()
+
+    for _ in range(args.warmup):
+        one_step()
+    # ---- timed region: K steps, device-timed on the library's stream (the legacy default stream)
+    clocks = Clocks(local)
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    stats = []
+    for _ in range(args.steps):
+        stats.append(one_step())
+    ev1.record()
+    barrier()
+    ck = clocks.stop()
+    ms = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    steps_local = sum(s["steps"] for s in stats)
+    tot = torch.tensor([steps_local], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(tot)
+    value = float(tot.item()) / (ms_max / 1000.0)
+
+    # ---- roofline of the update kernel (algorithmic bytes / CUDA-event launch time)
+    upd_ms = sum(s["update_ms"] for s in stats)
+    upd_launches = sum(s["update_launches"] for s in stats)
+    visits = sum(s["visits"] for s in stats)
+    steps_k = steps_local
+    moves = visits - len(stats) * W  # each walk's final visit ends in termination, every other visit in a move
+    alg_bytes = steps_k * (32 + 32 + 4) + visits * 16 + moves * 16 + len(stats) * W * 4
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
+    if os.path.exists(peaks_path):
+        peak, peak_src = float(json.load(open(peaks_path))["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
+    achieved = (alg_bytes / upd_launches) / (upd_ms / upd_launches / 1000.0) / 1e9 if upd_ms > 0 else None
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", "update_kernel_traffic.json")
+    if os.path.exists(prof):
+        pj = json.load(open(prof))
+        if pj.get("config_key") == f"cfg{args.config}-P{P}-C{args.chunk_walks}":
+            traffic = pj.get("dram_bytes_per_launch")
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+            "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+            "kernel": "k_update", "launches": upd_launches, "avg_launch_ms": upd_ms / max(1, upd_launches),
+            "alg_bytes_per_step": alg_bytes / max(1, steps_k), "peak_source": peak_src,
+            "update_share_of_step": upd_ms / ms}
+
+    # ---- extra partition-count sweep (context; the headline uses P above)
+    sweep = {}
+    for ps in [int(x) for x in args.sweep.split(",") if x.strip()]:
+        with LT.Engine(device=local, chunk_walks=args.chunk_walks, timing=True) as e2:
+            e2.graph_load(g.row_ptr, g.col, ps)
+            for _ in range(2):
+                e2.walks_init(starts_d, app, param, args.seed, first)
+                e2.run()
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            sts = []
+            for _ in range(3):
+                e2.walks_init(starts_d, app, param, args.seed, first)
+                e2.run()
+                sts.append(e2.stats())
+            b.record()
+            torch.cuda.synchronize()
+            sweep[str(ps)] = {"steps_per_s": sum(s["steps"] for s in sts) / (a.elapsed_time(b) / 1000),
+                              "visits_per_step": sum(s["visits"] for s in sts) / max(1, sum(s["steps"] for s in sts)),
+                              "sweeps": sts[-1]["sweeps"], "update_launches": sts[-1]["update_launches"]}
+
+    # ---- e2e through the C ABI with host buffers (pinned), H2D + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e and args.e2e_steps > 0:
+        S = int(c["length"]) + 1 if c["app"] == "deepwalk" else 128
+        try:
+            h_paths = torch.empty((W, S), dtype=torch.int32, pin_memory=True)
+            h_len = torch.empty(W, dtype=torch.int32, pin_memory=True)
+            h_starts = torch.from_numpy(starts_h.view(np.int32)).pin_memory()
+            pinned = True
+        except Exception:
+            h_paths = np.empty((W, S), dtype=np.uint32)
+            h_len = np.empty(W, dtype=np.uint32)
+            h_starts = starts_h
+            pinned = False
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        e_steps = 0
+        for _ in range(args.e2e_steps):
+            eng.walks_init(h_starts, app, param, args.seed, first)
+            eng.run()
+            eng.get_paths(h_paths, h_len)
+            e_steps += eng.stats()["steps"]
+        b.record()
+        barrier()
+        ems = a.elapsed_time(b)
+        et = torch.tensor([ems], dtype=torch.float64, device="cuda")
+        es = torch.tensor([e_steps], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+            dist.all_reduce(es)
+        e2e = {"value": float(es.item()) / (float(et.item()) / 1000), "unit": "steps/s",
+               "h2d_bytes_per_step": W * 4, "d2h_bytes_per_step": W * S * 4 + W * 4, "pinned": pinned,
+               "steps": args.e2e_steps}
+        del h_paths, h_len
+
+    # ---- CPU oracle baseline on a bounded sample (rank 0, N=1) + sampled parity of that sample
+    cpu = None
+    parity = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        eng.walks_init(starts_d, app, param, args.seed, first)
+        eng.run()
+        gh = host_graph(g)
+        r = oracle_sample(c, gh, W, first, args.cpu_seconds)
+        cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "kind": "oracle",
+               "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
+                         f"{r['seconds']:.1f} s; oracle/ C + OpenMP, nproc threads)"}
+        idx = np.linspace(0, r["walks"] - 1, num=min(r["walks"], 20000)).astype(np.uint64)
+        gp, gl = eng.get_paths_rows(idx)
+        ii = idx.astype(np.int64)
+        mism = int(np.sum(np.any(gp != r["paths"][ii], axis=1) | (gl != r["lengths"][ii])))
+        parity = {"sampled_walks": int(len(idx)), "mismatched_walks": mism, "vs": "oracle (bit-exact)"}
+
+    last = stats[-1]
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "steps/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": cfg_json(c, g, W, {"partitions": P, "chunk_walks": args.chunk_walks,
+                                             "policy": "selective" if args.policy == 0 else "round_robin",
+                                             "insert_mode": "warp_aggregated" if args.insert_mode == 0 else "direct",
+                                             "parallelism": f"replicas{world}" if world > 1 else "single",
+                                             "l2": "inputs larger than L2 (CSR >> 126 MB); no flush",
+                                             "graph_gen_s": round(gen_s, 2)}),
+                "clocks": ck, "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "parity_sample": parity,
+                "per_step": {"steps": last["steps"], "visits": last["visits"], "sweeps": last["sweeps"],
+                             "update_launches": last["update_launches"], "run_ms": last["run_ms"],
+                             "init_ms": last["init_ms"], "update_ms": last["update_ms"],
+                             "chunks_total": last["chunks_total"], "chunks_free_min": last["chunks_free_min"]}}
+        if sweep:
+            line["partition_sweep"] = sweep
+        print(json.dumps(line), flush=True)
+    eng.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,169 @@
+/* lt.h — C ABI of the B200-native LightTraffic walk-update path (liblt.so).
+ *
+ * The path (BASELINE.json north_star): vertices of a CSR graph are split into
+ * range partitions (§III-B "Graph data and partition"); walk states live in
+ * per-partition buckets made of fixed-size chunks of a pool reserved up front (PAPER.md:118,
+ * :124, :132-134, §III-B "Memory pool reservation" / "Walk index"); for each scheduled partition
+ * a kernel advances every walk in that partition's bucket until it terminates or leaves the
+ * partition (Alg. 1), and the updated walk is appended to the bucket
+ * of its new partition (walk reshuffling, §III-C). The host scheduler picks
+ * partitions by pending-walk count (selective scheduling) until no active walk
+ * remains (Alg. 2 line 1).
+ *
+ * The walk itself (PAPER.md:45 §II-A; :287 §IV-A): uniform neighbour per step; DeepWalk stops after
+ * l steps; PPR terminates with probability alpha before each move, capped at L_max steps. Sampling
+ * is Philox4x32-10 keyed by (walk_id, step) plus Lemire's unbiased range reduction, so every path is
+ * a pure function of (CSR, starts, app, parameter, seed, L_max) — independent of the partition
+ * count, chunk size, scheduling policy and launch shape (readings R1-R6).
+ *
+ * Conventions for every function:
+ *   - Returns lt_status; never aborts, never throws across the ABI. On error, lt_last_error()
+ *     returns a thread-local message describing the first failure.
+ *   - Host pointers are caller-owned and only read during the call (copied before return).
+ *     "Device" pointers are CUDA device memory (e.g. torch tensors) that the caller keeps alive
+ *     for as long as the context uses them; the library never frees them.
+ *   - Call order: lt_create -> lt_graph_load* -> lt_walks_init* -> lt_run -> lt_get_* ;
+ *     lt_walks_init* may be repeated after lt_run (a new epoch on the same graph). Out-of-order
+ *     calls return LT_ERR_STATE. Device memory is reserved in lt_graph_load(_device) and lt_walks_init(_ex) only
+ *     ("reserve the memory ... in advance"); lt_run never allocates.
+ *   - Layout: row_ptr is u64[n+1] (row_ptr[0]=0, non-decreasing, row_ptr[n]=m); col is u32[m] with
+ *     col[i] < n (Table II sizes imply 8-byte offsets and 4-byte IDs). Paths
+ *     are row-major u32[W][stride]; row w holds path vertices 0..length[w]-1, then 0xFFFFFFFF.
+ */
+#ifndef LT_H
+#define LT_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct lt_ctx lt_ctx;
+
+typedef enum {
+  LT_OK = 0,
+  LT_ERR_INVALID = 1, /* bad argument: malformed CSR, start >= n, P == 0 or P > n, bad l/alpha */
+  LT_ERR_STATE = 2,   /* call out of order */
+  LT_ERR_OOM = 3,     /* device memory reservation failed (create / graph_load / walks_init) */
+  LT_ERR_CUDA = 4,    /* a CUDA runtime error, or a device-side invariant violation */
+  LT_ERR_NCCL = 5     /* reserved for the multi-GPU exchange */
+} lt_status;
+
+typedef enum {
+  LT_APP_DEEPWALK = 0, /* uniform sampling, fixed length l */
+  LT_APP_PPR = 1       /* personalized PageRank: stop with probability alpha per step */
+} lt_app;
+
+typedef enum {
+  LT_POLICY_SELECTIVE = 0,  /* partitions in descending pending-walk order */
+  LT_POLICY_ROUND_ROBIN = 1 /* partitions in ID order (the ablation baseline) */
+} lt_policy;
+
+typedef enum {
+  LT_INSERT_WARP_AGGREGATED = 0, /* __match_any_sync groups: one atomic per (warp, dest) */
+  LT_INSERT_DIRECT = 1           /* one global atomic per walk ("direct write") */
+} lt_insert_mode;
+
+typedef struct lt_config {
+  int device;                 /* CUDA ordinal */
+  void* stream;               /* cudaStream_t to run on; NULL -> the legacy default stream */
+  uint32_t chunk_walks;       /* C, walks per pool chunk, power of two >= 64; 0 -> 8192 */
+  uint32_t ppr_max_len;       /* L_max, PPR step cap (reading R6); 0 -> 127 */
+  uint32_t policy;            /* lt_policy */
+  uint32_t insert_mode;       /* lt_insert_mode */
+  uint32_t timing;            /* 1 -> CUDA events around every update launch (lt_stats.update_ms) */
+  uint32_t block_threads;     /* update kernel block size (multiple of 32); 0 -> 256 */
+  uint32_t blocks_per_sm;     /* update kernel resident blocks per SM for the grid; 0 -> occupancy */
+  uint32_t reserved[8];
+} lt_config;
+
+typedef struct lt_stats {
+  uint64_t num_walks;          /* W of the last lt_walks_init */
+  uint64_t steps;              /* sum over walks of (path vertices - 1) ("steps") */
+  uint64_t visits;             /* walk records consumed by update launches (residences) */
+  uint64_t truncated;          /* PPR walks stopped by L_max */
+  uint64_t sweeps;             /* scheduler passes over the partitions */
+  uint64_t update_launches;    /* walk-update kernel launches in the last lt_run */
+  uint64_t kernel_launches;    /* all kernels the library launched in the last lt_walks_init + lt_run */
+  uint64_t chunks_total;       /* pool size in chunks */
+  uint64_t chunks_free_min;    /* low-water mark of free chunks seen at sweep boundaries */
+  uint64_t h2d_bytes;          /* host->device bytes moved by the last init/run/get calls */
+  uint64_t d2h_bytes;
+  double update_ms;            /* sum of CUDA-event durations of update launches (if timing) */
+  double run_ms;               /* CUDA-event duration of the last lt_run (first launch..last) */
+  double init_ms;              /* CUDA-event duration of the last lt_walks_init* */
+} lt_stats;
+
+/* Fill *cfg with defaults (device 0, library stream, C=8192, L_max=127, selective, aggregated). */
+lt_status lt_config_default(lt_config* cfg);
+
+/* Create a context on cfg->device. No graph or walk memory is reserved yet. */
+lt_status lt_create(const lt_config* cfg, lt_ctx** out);
+void lt_destroy(lt_ctx* ctx);
+const char* lt_last_error(void);
+
+/* Range partitioning. Host-only utility, no GPU needed:
+ * bounds[0]=0 < bounds[1] < ... < bounds[P]=n; partition k = [bounds[k], bounds[k+1]); edges go
+ * with their source. Bounds balance the CSR bytes cost(v) = 8 v + 4 row_ptr[v]:
+ * bounds[k] = min{v : P cost(v) >= k cost(n)} (exact), then forced strictly increasing.
+ * Requires 1 <= P <= n. */
+lt_status lt_partition_bounds(uint32_t n, const uint64_t* row_ptr, uint32_t P, uint32_t* bounds);
+
+/* Load the graph and partition it into P ranges (a1). lt_graph_load copies host arrays into
+ * device memory the library owns; lt_graph_load_device BORROWS device arrays (no copy; the caller
+ * keeps them alive and unchanged until lt_destroy or the next load). Validates the CSR (host
+ * variant: full check; device variant: row_ptr checked on a host copy, col range checked on the
+ * device). */
+lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row_ptr,
+                        const uint32_t* col, uint32_t num_partitions);
+lt_status lt_graph_load_device(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* d_row_ptr,
+                               const uint32_t* d_col, uint32_t num_partitions);
+/* Partition bounds in use: bounds must hold P+1 entries (query P with bounds == NULL). */
+lt_status lt_get_bounds(lt_ctx* ctx, uint32_t* bounds, uint32_t* P);
+
+/* Create W walks (a2): walk i has ID first_walk_id + i (the Philox key counter), starts at
+ * starts[i] < n, and is appended to the bucket of its start's partition. length_or_alpha is the
+ * DeepWalk length l (a non-negative integer) or the PPR alpha in (0, 1). starts is host memory
+ * (lt_walks_init) or device memory (lt_walks_init_device). W < 2^32 - 1. */
+lt_status lt_walks_init(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, lt_app app,
+                        double length_or_alpha, uint64_t seed);
+lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, int starts_on_device,
+                           uint64_t first_walk_id, lt_app app, double length_or_alpha, uint64_t seed);
+
+/* Run the partition scheduler until every walk has terminated (a3-a7). Blocks the host. */
+lt_status lt_run(lt_ctx* ctx);
+
+/* Row stride of the path matrix: l+1 (DeepWalk) or L_max+1 (PPR). */
+lt_status lt_path_stride(lt_ctx* ctx, uint32_t* stride);
+
+/* Copy all paths (W x stride u32, row-major) and lengths (W u32, path vertices) to HOST buffers.
+ * Either pointer may be NULL to skip it. */
+lt_status lt_get_paths(lt_ctx* ctx, uint32_t* paths, uint32_t* lengths);
+/* Copy the rows listed in host array rows[count] (local walk indices) to host paths[count x stride]
+ * and lengths[count]. */
+lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, uint32_t* paths,
+                            uint32_t* lengths);
+/* Copy all paths / lengths into caller-owned DEVICE buffers (same layout as lt_get_paths). */
+lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_lengths);
+
+lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out);
+
+/* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:
+ * pending + finished == num_walks; free_chunks + ring_chunks == total_chunks. */
+typedef struct lt_pool_state {
+  int64_t free_chunks;     /* free-stack depth */
+  uint64_t ring_chunks;    /* installed (non-empty) ring slots over all partitions */
+  uint64_t reserved0;
+  uint64_t total_chunks;
+  uint64_t pending;        /* sum over partitions of cursor - head (walks waiting in buckets) */
+  uint64_t finished;       /* walks with a recorded length */
+  uint32_t device_err;     /* device error bits (1: pool exhausted, 2: ring slot reinstalled) */
+  uint32_t reserved;
+} lt_pool_state;
+lt_status lt_get_pool_state(lt_ctx* ctx, lt_pool_state* out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -129,9 +129,9 @@ def tuple_at(scale: int, seed: int, permute: bool, e: int) -> tuple[int, int]:
     return int(u.value), int(v.value)
 
 
-def deepwalk_starts(num_walks: int, n: int, first_walk: int = 0) -> np.ndarray:
+def deepwalk_starts(num_walks: int, n: int, first_walk_id: int = 0) -> np.ndarray:
     """Walk w starts at vertex w mod n (SURVEY.md §8(c) reading #7 of PAPER.md:287)."""
-    w = np.arange(first_walk, first_walk + num_walks, dtype=np.uint64)
+    w = np.arange(first_walk_id, first_walk_id + num_walks, dtype=np.uint64)
     return (w % np.uint64(n)).astype(np.uint32)
 
 

@@ -1,0 +1,586 @@
+// lt_abi.cpp — the C ABI (include/lt.h): context, validation, range partitioner (a1), pool
+// reservation (a6 sizing), and the host partition scheduler (a7; Alg. 2).
+#include "lt.h"
+#include "lt_internal.h"
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+namespace {
+
+thread_local std::string g_err;
+
+lt_status fail(lt_status s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+#define CK(call)                                                                        \
+  do {                                                                                  \
+    cudaError_t _e = (call);                                                            \
+    if (_e != cudaSuccess)                                                              \
+      return fail(_e == cudaErrorMemoryAllocation ? LT_ERR_OOM : LT_ERR_CUDA,           \
+                  std::string(#call) + ": " + cudaGetErrorString(_e));                  \
+  } while (0)
+
+template <class T>
+cudaError_t ensure(T*& p, size_t& cap, size_t count) {
+  if (count <= cap && p) return cudaSuccess;
+  if (p) cudaFree(p);
+  p = nullptr;
+  cap = 0;
+  cudaError_t e = cudaMalloc((void**)&p, std::max<size_t>(count, 1) * sizeof(T));
+  if (e == cudaSuccess) cap = count;
+  return e;
+}
+
+}  // namespace
+
+struct lt_ctx {
+  lt_config cfg{};
+  cudaStream_t stream = nullptr;
+  int num_sms = 148;
+  int occ = 1;
+  uint32_t block = 256;
+  // graph
+  bool graph_loaded = false;
+  uint32_t n = 0;
+  uint64_t m = 0;
+  uint32_t P = 0;
+  unsigned long long* d_row_ptr = nullptr;
+  uint32_t* d_col = nullptr;
+  bool own_graph = false;
+  std::vector<uint32_t> h_bounds;
+  uint32_t* d_bounds = nullptr;
+  size_t bounds_cap = 0;
+  // walks
+  bool walks_ready = false;
+  bool ran = false;
+  uint64_t W = 0, first = 0, seed = 0;
+  lt_app app = LT_APP_DEEPWALK;
+  uint32_t length = 0, T = 0, lmax = 127, stride = 1;
+  uint32_t* d_paths = nullptr;
+  size_t paths_cap = 0;
+  uint32_t* d_lengths = nullptr;
+  size_t lengths_cap = 0;
+  uint32_t* d_starts = nullptr;
+  size_t starts_cap = 0;
+  // pool
+  uint4* d_slots = nullptr;
+  size_t slots_cap = 0;
+  uint32_t* d_ring = nullptr;
+  size_t ring_cap = 0;
+  unsigned long long* d_hc = nullptr;  // head[P] then cursor[P]
+  size_t hc_cap = 0;
+  uint32_t* d_free = nullptr;
+  size_t free_cap = 0;
+  uint32_t* d_small = nullptr;  // [0]=free_top [1]=unused [2..3]=scratch flags
+  lt::Counters* d_ctr = nullptr;
+  // pinned staging
+  unsigned long long* h_hc = nullptr;
+  size_t h_hc_cap = 0;
+  lt::Counters* h_ctr = nullptr;
+  lt::Params params{};
+  lt_stats stats{};
+  std::vector<cudaEvent_t> events;
+  cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+};
+
+extern "C" {
+
+const char* lt_last_error(void) { return g_err.c_str(); }
+
+lt_status lt_config_default(lt_config* cfg) {
+  if (!cfg) return fail(LT_ERR_INVALID, "cfg is NULL");
+  std::memset(cfg, 0, sizeof(*cfg));
+  cfg->chunk_walks = 8192;
+  cfg->ppr_max_len = 127;
+  return LT_OK;
+}
+
+lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
+  if (!out) return fail(LT_ERR_INVALID, "out is NULL");
+  *out = nullptr;
+  lt_config c;
+  if (cfg) c = *cfg; else lt_config_default(&c);
+  if (c.chunk_walks == 0) c.chunk_walks = 8192;
+  if (c.chunk_walks < 64 || (c.chunk_walks & (c.chunk_walks - 1)))
+    return fail(LT_ERR_INVALID, "chunk_walks must be a power of two >= 64");
+  if (c.ppr_max_len == 0) c.ppr_max_len = 127;
+  if (c.block_threads == 0) c.block_threads = 256;
+  if (c.block_threads != 256) return fail(LT_ERR_INVALID, "block_threads must be 256 in this build");
+  if (c.policy > 1 || c.insert_mode > 1) return fail(LT_ERR_INVALID, "bad policy / insert_mode");
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  if (c.device < 0 || c.device >= ndev) return fail(LT_ERR_INVALID, "bad device ordinal");
+  CK(cudaSetDevice(c.device));
+  lt_ctx* ctx = new lt_ctx();
+  ctx->cfg = c;
+  ctx->stream = (cudaStream_t)c.stream;
+  ctx->block = c.block_threads;
+  cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, c.device);
+  ctx->occ = c.blocks_per_sm ? (int)c.blocks_per_sm : lt::update_kernel_occupancy(ctx->block);
+  cudaError_t e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_ctr, sizeof(lt::Counters));
+  if (e == cudaSuccess) e = cudaMallocHost((void**)&ctx->h_ctr, sizeof(lt::Counters));
+  if (e == cudaSuccess) e = cudaEventCreate(&ctx->ev_a);
+  if (e == cudaSuccess) e = cudaEventCreate(&ctx->ev_b);
+  if (e != cudaSuccess) {
+    lt_destroy(ctx);
+    return fail(LT_ERR_CUDA, std::string("lt_create: ") + cudaGetErrorString(e));
+  }
+  *out = ctx;
+  return LT_OK;
+}
+
+void lt_destroy(lt_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->cfg.device);
+  if (ctx->stream) cudaStreamSynchronize(ctx->stream); else cudaDeviceSynchronize();
+  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  cudaFree(ctx->d_bounds);
+  cudaFree(ctx->d_paths);
+  cudaFree(ctx->d_lengths);
+  cudaFree(ctx->d_starts);
+  cudaFree(ctx->d_slots);
+  cudaFree(ctx->d_ring);
+  cudaFree(ctx->d_hc);
+  cudaFree(ctx->d_free);
+  cudaFree(ctx->d_small);
+  cudaFree(ctx->d_ctr);
+  if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
+  if (ctx->h_ctr) cudaFreeHost(ctx->h_ctr);
+  for (auto ev : ctx->events) cudaEventDestroy(ev);
+  if (ctx->ev_a) cudaEventDestroy(ctx->ev_a);
+  if (ctx->ev_b) cudaEventDestroy(ctx->ev_b);
+  delete ctx;
+}
+
+// a1: byte-balanced range partitioning, cost(v) = 8 v + 4 row_ptr[v] (the CSR prefix
+// of vertices < v), bounds[k] = min{v : P cost(v) >= k cost(n)}, then made strictly increasing.
+lt_status lt_partition_bounds(uint32_t n, const uint64_t* row_ptr, uint32_t P, uint32_t* bounds) {
+  if (!row_ptr || !bounds) return fail(LT_ERR_INVALID, "NULL argument");
+  if (P == 0 || P > n) return fail(LT_ERR_INVALID, "need 1 <= num_partitions <= n");
+  auto cost = [&](uint64_t v) -> unsigned __int128 { return (unsigned __int128)8 * v + (unsigned __int128)4 * row_ptr[v]; };
+  const unsigned __int128 total = cost(n);
+  bounds[0] = 0;
+  bounds[P] = n;
+  for (uint32_t k = 1; k < P; ++k) {
+    const unsigned __int128 target = total * k;
+    uint64_t lo = 0, hi = n;  // first v with P cost(v) >= k cost(n)
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) / 2;
+      if (cost(mid) * P < target) lo = mid + 1; else hi = mid;
+    }
+    bounds[k] = (uint32_t)lo;
+  }
+  for (uint32_t k = 1; k < P; ++k) bounds[k] = std::max(bounds[k], bounds[k - 1] + 1);
+  for (uint32_t k = P - 1; k >= 1; --k) bounds[k] = std::min(bounds[k], bounds[k + 1] - 1);
+  return LT_OK;
+}
+
+static lt_status validate_row_ptr(uint32_t n, uint64_t m, const uint64_t* row_ptr) {
+  if (n == 0) return fail(LT_ERR_INVALID, "n must be >= 1");
+  if (row_ptr[0] != 0) return fail(LT_ERR_INVALID, "row_ptr[0] != 0");
+  if (row_ptr[n] != m) return fail(LT_ERR_INVALID, "row_ptr[n] != m");
+  for (uint32_t v = 0; v < n; ++v) {
+    if (row_ptr[v + 1] < row_ptr[v]) return fail(LT_ERR_INVALID, "row_ptr not monotone at " + std::to_string(v));
+    if (row_ptr[v + 1] - row_ptr[v] > 0xFFFFFFFFull) return fail(LT_ERR_INVALID, "degree >= 2^32");
+  }
+  return LT_OK;
+}
+
+static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* h_row_ptr, uint32_t P) {
+  std::vector<uint32_t> b(P + 1);
+  lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
+  if (s != LT_OK) return s;
+  CK(ensure(ctx->d_bounds, ctx->bounds_cap, P + 1));
+  CK(cudaMemcpy(ctx->d_bounds, b.data(), (P + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice));
+  CK(ensure(ctx->d_hc, ctx->hc_cap, 2 * (size_t)P));
+  if (ctx->h_hc_cap < 2 * (size_t)P) {
+    if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
+    ctx->h_hc = nullptr;
+    ctx->h_hc_cap = 0;
+    CK(cudaMallocHost((void**)&ctx->h_hc, 2 * (size_t)P * sizeof(unsigned long long)));
+    ctx->h_hc_cap = 2 * (size_t)P;
+  }
+  ctx->h_bounds = std::move(b);
+  ctx->n = n;
+  ctx->m = m;
+  ctx->P = P;
+  ctx->graph_loaded = true;
+  ctx->walks_ready = false;
+  ctx->ran = false;
+  return LT_OK;
+}
+
+lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row_ptr, const uint32_t* col,
+                        uint32_t P) {
+  if (!ctx || !row_ptr || (m && !col)) return fail(LT_ERR_INVALID, "NULL argument");
+  CK(cudaSetDevice(ctx->cfg.device));
+  lt_status s = validate_row_ptr(n, m, row_ptr);
+  if (s != LT_OK) return s;
+  for (uint64_t i = 0; i < m; ++i)
+    if (col[i] >= n) return fail(LT_ERR_INVALID, "col[" + std::to_string(i) + "] >= n");
+  if (P == 0 || P > n) return fail(LT_ERR_INVALID, "need 1 <= num_partitions <= n");
+  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  ctx->d_row_ptr = nullptr;
+  ctx->d_col = nullptr;
+  ctx->own_graph = true;
+  ctx->graph_loaded = false;
+  CK(cudaMalloc((void**)&ctx->d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t)));
+  CK(cudaMalloc((void**)&ctx->d_col, std::max<uint64_t>(m, 1) * sizeof(uint32_t)));
+  CK(cudaMemcpy(ctx->d_row_ptr, row_ptr, ((size_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  if (m) CK(cudaMemcpy(ctx->d_col, col, m * sizeof(uint32_t), cudaMemcpyHostToDevice));
+  ctx->stats.h2d_bytes += ((uint64_t)n + 1) * 8 + m * 4;
+  return finish_graph_load(ctx, n, m, row_ptr, P);
+}
+
+lt_status lt_graph_load_device(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* d_row_ptr, const uint32_t* d_col,
+                               uint32_t P) {
+  if (!ctx || !d_row_ptr || (m && !d_col)) return fail(LT_ERR_INVALID, "NULL argument");
+  CK(cudaSetDevice(ctx->cfg.device));
+  std::vector<uint64_t> h((size_t)n + 1);
+  CK(cudaMemcpy(h.data(), d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost));
+  lt_status s = validate_row_ptr(n, m, h.data());
+  if (s != LT_OK) return s;
+  if (P == 0 || P > n) return fail(LT_ERR_INVALID, "need 1 <= num_partitions <= n");
+  CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), ctx->stream));
+  CK(lt::launch_check_col(d_col, m, n, ctx->d_small + 2, ctx->stream));
+  uint32_t bad = 0;
+  CK(cudaMemcpyAsync(&bad, ctx->d_small + 2, sizeof(uint32_t), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  if (bad) return fail(LT_ERR_INVALID, "col entry >= n");
+  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  ctx->own_graph = false;
+  ctx->d_row_ptr = (unsigned long long*)d_row_ptr;
+  ctx->d_col = (uint32_t*)d_col;
+  return finish_graph_load(ctx, n, m, h.data(), P);
+}
+
+lt_status lt_get_bounds(lt_ctx* ctx, uint32_t* bounds, uint32_t* P) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "no graph loaded");
+  if (P) *P = ctx->P;
+  if (bounds) std::memcpy(bounds, ctx->h_bounds.data(), (ctx->P + 1) * sizeof(uint32_t));
+  return LT_OK;
+}
+
+lt_status lt_walks_init(lt_ctx* ctx, uint64_t W, const uint32_t* starts, lt_app app, double param, uint64_t seed) {
+  return lt_walks_init_ex(ctx, W, starts, 0, 0, app, param, seed);
+}
+
+lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device, uint64_t first_walk_id,
+                           lt_app app, double param, uint64_t seed) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_walks_init before lt_graph_load");
+  if (W && !starts) return fail(LT_ERR_INVALID, "starts is NULL");
+  if (W >= 0xFFFFFFFFull) return fail(LT_ERR_INVALID, "num_walks must be < 2^32 - 1");
+  CK(cudaSetDevice(ctx->cfg.device));
+  uint32_t length = 0, T = 0, stride = 0;
+  const uint32_t lmax = ctx->cfg.ppr_max_len;
+  if (app == LT_APP_DEEPWALK) {
+    if (!(param >= 0) || param != std::floor(param) || param > 1e6)
+      return fail(LT_ERR_INVALID, "DeepWalk length must be an integer in [0, 1e6]");
+    length = (uint32_t)param;
+    stride = length + 1;
+  } else if (app == LT_APP_PPR) {
+    if (!(param > 0 && param < 1)) return fail(LT_ERR_INVALID, "PPR alpha must be in (0, 1)");
+    const double t = param * 4294967296.0;  // T = floor(alpha 2^32) (reading R5)
+    T = (uint32_t)t;
+    stride = lmax + 1;
+  } else {
+    return fail(LT_ERR_INVALID, "unknown app");
+  }
+  ctx->walks_ready = false;
+  ctx->ran = false;
+  ctx->stats.h2d_bytes = 0;
+  ctx->stats.d2h_bytes = 0;
+  cudaStream_t s = ctx->stream;
+  // starts
+  const uint32_t* d_starts = starts;
+  if (!on_device) {
+    for (uint64_t i = 0; i < W; ++i)
+      if (starts[i] >= ctx->n) return fail(LT_ERR_INVALID, "starts[" + std::to_string(i) + "] >= n");
+    CK(ensure(ctx->d_starts, ctx->starts_cap, W));
+    if (W) CK(cudaMemcpyAsync(ctx->d_starts, starts, W * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+    ctx->stats.h2d_bytes += W * 4;
+    d_starts = ctx->d_starts;
+  }
+  // reserve: paths, lengths, pool
+  const uint64_t C = ctx->cfg.chunk_walks;
+  uint32_t c_shift = 0;
+  while ((1ull << c_shift) < C) ++c_shift;
+  const uint64_t wc = (W + C - 1) / C;
+  const uint64_t ring_len = wc + 2;
+  const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->P + 64;
+  if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
+  CK(ensure(ctx->d_paths, ctx->paths_cap, std::max<uint64_t>(W, 1) * stride));
+  CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
+  CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
+  CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->P * ring_len));
+  CK(ensure(ctx->d_free, ctx->free_cap, num_chunks));
+  if (on_device && W) {
+    CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
+    CK(lt::launch_check_starts(d_starts, W, ctx->n, ctx->d_small + 2, s));
+    uint32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, ctx->d_small + 2, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (bad) return fail(LT_ERR_INVALID, "a start vertex >= n");
+  }
+  lt::Params& p = ctx->params;
+  p.wk.row_ptr = ctx->d_row_ptr;
+  p.wk.col = ctx->d_col;
+  p.wk.bounds = ctx->d_bounds;
+  p.wk.P = ctx->P;
+  p.wk.paths = ctx->d_paths;
+  p.wk.stride = stride;
+  p.wk.lengths = ctx->d_lengths;
+  p.wk.first_walk_id = first_walk_id;
+  p.wk.seed_lo = (uint32_t)seed;
+  p.wk.seed_hi = (uint32_t)(seed >> 32);
+  p.wk.app = (uint32_t)app;
+  p.wk.length = length;
+  p.wk.T = T;
+  p.wk.lmax = lmax;
+  p.pool.slots = ctx->d_slots;
+  p.pool.C = (uint32_t)C;
+  p.pool.c_shift = c_shift;
+  p.pool.num_chunks = (uint32_t)num_chunks;
+  p.pool.ring = ctx->d_ring;
+  p.pool.ring_len = (uint32_t)ring_len;
+  p.pool.head = ctx->d_hc;
+  p.pool.cursor = ctx->d_hc + ctx->P;
+  p.pool.free_list = ctx->d_free;
+  p.pool.free_top = (int*)ctx->d_small;
+  p.ctr = ctx->d_ctr;
+  p.insert_mode = ctx->cfg.insert_mode;
+
+  ctx->W = W;
+  ctx->first = first_walk_id;
+  ctx->seed = seed;
+  ctx->app = app;
+  ctx->length = length;
+  ctx->T = T;
+  ctx->lmax = lmax;
+  ctx->stride = stride;
+  ctx->stats.num_walks = W;
+  ctx->stats.chunks_total = num_chunks;
+  ctx->stats.kernel_launches = 0;
+  CK(cudaEventRecord(ctx->ev_a, s));
+  CK(lt::launch_pool_reset(p, s));
+  ctx->stats.kernel_launches++;
+  if (W) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
+  if (W) {
+    CK(lt::launch_init(p, d_starts, W, s));
+    ctx->stats.kernel_launches++;
+  }
+  CK(cudaEventRecord(ctx->ev_b, s));
+  ctx->walks_ready = true;
+  return LT_OK;
+}
+
+lt_status lt_run(lt_ctx* ctx) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "lt_run before lt_walks_init");
+  if (ctx->ran) return fail(LT_ERR_STATE, "lt_run already done for these walks; call lt_walks_init again");
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaStream_t s = ctx->stream;
+  lt::Params& p = ctx->params;
+  const uint32_t P = ctx->P;
+  const uint64_t max_grid = (uint64_t)ctx->num_sms * ctx->occ;
+  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
+  {
+    float ms = 0;
+    CK(cudaEventSynchronize(ctx->ev_b));
+    CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
+    ctx->stats.init_ms = ms;
+  }
+  ctx->stats.sweeps = 0;
+  ctx->stats.update_launches = 0;
+  ctx->stats.update_ms = 0;
+  ctx->stats.chunks_free_min = ctx->stats.chunks_total;
+  size_t nev = 0;
+  std::vector<uint32_t> order;
+  order.reserve(P);
+  CK(cudaEventRecord(ctx->ev_a, s));
+  for (;;) {
+    // pending-walk counts at the sweep boundary (one small D2H + sync per sweep)
+    CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)P * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
+    uint32_t free_top = 0;
+    CK(cudaMemcpyAsync(&free_top, ctx->d_small, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (ctx->h_ctr->err) break;
+    ctx->stats.chunks_free_min = std::min<uint64_t>(ctx->stats.chunks_free_min, (uint64_t)(int)free_top);
+    const unsigned long long* head = ctx->h_hc;
+    const unsigned long long* cur = ctx->h_hc + P;
+    order.clear();
+    uint64_t total = 0;
+    for (uint32_t k = 0; k < P; ++k)
+      if (cur[k] > head[k]) { order.push_back(k); total += cur[k] - head[k]; }
+    if (total == 0) break;
+    if (ctx->stats.sweeps > max_len + 2)
+      return fail(LT_ERR_CUDA, "scheduler did not converge (walk count not decreasing)");
+    if (ctx->cfg.policy == LT_POLICY_SELECTIVE)  // most pending walks first
+      std::stable_sort(order.begin(), order.end(),
+                       [&](uint32_t a, uint32_t b) { return cur[a] - head[a] > cur[b] - head[b]; });
+    uint64_t earlier = 0;
+    for (uint32_t k : order) {
+      const uint64_t pend = cur[k] - head[k];
+      // walks present at launch time <= pending now + everything launched before in this sweep
+      const uint64_t bound = pend + earlier;
+      earlier += pend;
+      const uint64_t grid = std::min<uint64_t>(std::max<uint64_t>((bound + ctx->block - 1) / ctx->block, 1), max_grid);
+      if (ctx->cfg.timing) {
+        while (ctx->events.size() < nev + 2) {
+          cudaEvent_t ev;
+          CK(cudaEventCreate(&ev));
+          ctx->events.push_back(ev);
+        }
+        CK(cudaEventRecord(ctx->events[nev], s));
+      }
+      CK(lt::launch_update(p, k, (uint32_t)grid, ctx->block, s));
+      if (ctx->cfg.timing) {
+        CK(cudaEventRecord(ctx->events[nev + 1], s));
+        nev += 2;
+      }
+      ctx->stats.update_launches++;
+      ctx->stats.kernel_launches++;
+    }
+    ctx->stats.sweeps++;
+  }
+  CK(lt::launch_finalize_paths(p, ctx->W, s));
+  ctx->stats.kernel_launches++;
+  CK(cudaEventRecord(ctx->ev_b, s));
+  CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  {
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
+    ctx->stats.run_ms = ms;
+    double tot = 0;
+    for (size_t i = 0; i + 1 < nev; i += 2) {
+      CK(cudaEventElapsedTime(&ms, ctx->events[i], ctx->events[i + 1]));
+      tot += ms;
+    }
+    ctx->stats.update_ms = tot;
+  }
+  ctx->stats.steps = ctx->h_ctr->steps;
+  ctx->stats.visits = ctx->h_ctr->visits;
+  ctx->stats.truncated = ctx->h_ctr->truncated;
+  ctx->ran = true;
+  if (ctx->h_ctr->err & lt::kErrOOM) return fail(LT_ERR_CUDA, "walk pool exhausted on the device (invariant violated)");
+  if (ctx->h_ctr->err) return fail(LT_ERR_CUDA, "device invariant violated (ring slot reinstalled)");
+  return LT_OK;
+}
+
+lt_status lt_path_stride(lt_ctx* ctx, uint32_t* stride) {
+  if (!ctx || !stride) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  *stride = ctx->stride;
+  return LT_OK;
+}
+
+static lt_status need_ran(lt_ctx* ctx) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
+  return LT_OK;
+}
+
+lt_status lt_get_paths(lt_ctx* ctx, uint32_t* paths, uint32_t* lengths) {
+  lt_status st = need_ran(ctx);
+  if (st != LT_OK) return st;
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaStream_t s = ctx->stream;
+  if (paths && ctx->W) {
+    CK(cudaMemcpyAsync(paths, ctx->d_paths, ctx->W * ctx->stride * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    ctx->stats.d2h_bytes += ctx->W * ctx->stride * 4;
+  }
+  if (lengths && ctx->W) {
+    CK(cudaMemcpyAsync(lengths, ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    ctx->stats.d2h_bytes += ctx->W * 4;
+  }
+  CK(cudaStreamSynchronize(s));
+  return LT_OK;
+}
+
+lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, uint32_t* paths, uint32_t* lengths) {
+  lt_status st = need_ran(ctx);
+  if (st != LT_OK) return st;
+  if (count && (!rows || !paths || !lengths)) return fail(LT_ERR_INVALID, "NULL argument");
+  for (uint64_t i = 0; i < count; ++i)
+    if (rows[i] >= ctx->W) return fail(LT_ERR_INVALID, "row index >= W");
+  if (!count) return LT_OK;
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaStream_t s = ctx->stream;
+  unsigned long long* d_rows = nullptr;
+  uint32_t* d_out = nullptr;
+  uint32_t* d_len = nullptr;
+  CK(cudaMalloc((void**)&d_rows, count * sizeof(uint64_t)));
+  cudaError_t e = cudaMalloc((void**)&d_out, count * ctx->stride * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMalloc((void**)&d_len, count * sizeof(uint32_t));
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d_rows, rows, count * sizeof(uint64_t), cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess) e = lt::launch_gather_rows(ctx->params, d_rows, count, d_out, d_len, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(paths, d_out, count * ctx->stride * sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(lengths, d_len, count * sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaFree(d_rows);
+  cudaFree(d_out);
+  cudaFree(d_len);
+  if (e != cudaSuccess) return fail(LT_ERR_CUDA, std::string("lt_get_paths_rows: ") + cudaGetErrorString(e));
+  return LT_OK;
+}
+
+lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_lengths) {
+  lt_status st = need_ran(ctx);
+  if (st != LT_OK) return st;
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaStream_t s = ctx->stream;
+  if (d_paths && ctx->W)
+    CK(cudaMemcpyAsync(d_paths, ctx->d_paths, ctx->W * ctx->stride * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+  if (d_lengths && ctx->W)
+    CK(cudaMemcpyAsync(d_lengths, ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+  CK(cudaStreamSynchronize(s));
+  return LT_OK;
+}
+
+lt_status lt_get_pool_state(lt_ctx* ctx, lt_pool_state* out) {
+  if (!ctx || !out) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  CK(cudaSetDevice(ctx->cfg.device));
+  CK(cudaStreamSynchronize(ctx->stream));
+  const lt::Params& p = ctx->params;
+  std::memset(out, 0, sizeof(*out));
+  int32_t small[2] = {0, 0};
+  CK(cudaMemcpy(small, ctx->d_small, sizeof(small), cudaMemcpyDeviceToHost));
+  lt::Counters c;
+  CK(cudaMemcpy(&c, ctx->d_ctr, sizeof(c), cudaMemcpyDeviceToHost));
+  std::vector<uint32_t> ring((size_t)ctx->P * p.pool.ring_len);
+  CK(cudaMemcpy(ring.data(), ctx->d_ring, ring.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  std::vector<unsigned long long> hc(2 * (size_t)ctx->P);
+  CK(cudaMemcpy(hc.data(), ctx->d_hc, hc.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+  std::vector<uint32_t> len(ctx->W);
+  if (ctx->W) CK(cudaMemcpy(len.data(), ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  out->free_chunks = small[0];
+  out->total_chunks = p.pool.num_chunks;
+  for (uint32_t r : ring) out->ring_chunks += (r != lt::kEmpty);
+  for (uint32_t k = 0; k < ctx->P; ++k) out->pending += hc[ctx->P + k] - hc[k];
+  if (ctx->ran) out->finished = ctx->W;  // every walk terminated
+  else for (uint32_t l : len) out->finished += (l != 0 && l != lt::kEmpty);
+  out->device_err = c.err;
+  return LT_OK;
+}
+
+lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out) {
+  if (!ctx || !out) return fail(LT_ERR_INVALID, "NULL argument");
+  *out = ctx->stats;
+  return LT_OK;
+}
+
+}  // extern "C"

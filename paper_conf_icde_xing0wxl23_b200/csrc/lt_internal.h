@@ -1,0 +1,71 @@
+// lt_internal.h — device-side state shared by the host scheduler (lt_abi.cpp) and the kernels
+// (lt_kernels.cu). Not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace lt {
+
+constexpr uint32_t kEmpty = 0xFFFFFFFFu;   // empty ring slot / unused path slot
+constexpr uint32_t kErrOOM = 1u;           // device error bits
+constexpr uint32_t kErrRing = 2u;
+
+// A walk record (D5): 16 bytes, one 128-bit load/store.
+//   x = local walk index (row of the path matrix; walk_id = first_walk_id + x)
+//   y = current_vertex, z = walked_steps, w = reserved (0)
+
+// Walk pool (a6): `slots` is an arena of num_chunks chunks of C records.
+// Bucket k is the position range [head[k], cursor[k]) (monotone u64 counters); position pos lives
+// in chunk ring[k*ring_len + (pos/C) % ring_len] at offset pos % C. Ring slots are installed on
+// demand: exactly once per chunk, by the writer whose claim holds the chunk's first slot.
+struct Pool {
+  uint4* slots;
+  uint32_t C, c_shift;
+  uint32_t num_chunks;            // + 1 trash chunk at index num_chunks (writes after OOM)
+  uint32_t* ring;
+  uint32_t ring_len;
+  unsigned long long* head;       // [P]
+  unsigned long long* cursor;     // [P]
+  uint32_t* free_list;            // [num_chunks]
+  int* free_top;
+};
+
+struct Walk {
+  const unsigned long long* row_ptr;
+  const uint32_t* col;
+  const uint32_t* bounds;         // [P+1]
+  uint32_t P;
+  uint32_t* paths;
+  uint64_t stride;
+  uint32_t* lengths;
+  uint64_t first_walk_id;
+  uint32_t seed_lo, seed_hi;
+  uint32_t app, length, T, lmax;
+};
+
+struct Counters {
+  unsigned long long steps, visits, truncated;
+  uint32_t err;
+  uint32_t done_ctas;
+};
+
+struct Params {
+  Walk wk;
+  Pool pool;
+  Counters* ctr;
+  uint32_t insert_mode;
+};
+
+// launchers (lt_kernels.cu); all asynchronous on `s`
+cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cudaStream_t s);
+cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s);
+cudaError_t launch_finalize_paths(const Params& p, uint64_t W, cudaStream_t s);
+cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, uint64_t count,
+                               uint32_t* out_paths, uint32_t* out_lengths, cudaStream_t s);
+cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
+cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
+cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
+int update_kernel_occupancy(uint32_t block);   // resident blocks per SM for the update kernel
+uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
+
+}  // namespace lt

@@ -1,0 +1,246 @@
+"""Thin ctypes binding of liblt.so (include/lt.h). Argument marshalling only: every step of the
+walk-update path runs in the CUDA kernels behind the C ABI. There is no CPU fallback: if liblt.so
+is missing or fails to load, importing this module raises.
+
+Arrays may be numpy arrays / CPU torch tensors (host pointers; pinned tensors give fast copies)
+or CUDA torch tensors (device pointers, borrowed). uint64/uint32 data may be passed as int64/int32
+torch tensors (same bits).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liblt.so")
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build the CUDA extension first (`make lt` or "
+                      f"__graft_entry__.build()); there is no CPU fallback")
+_lib = ctypes.CDLL(LIB_PATH)
+
+LT_OK, LT_ERR_INVALID, LT_ERR_STATE, LT_ERR_OOM, LT_ERR_CUDA, LT_ERR_NCCL = range(6)
+DEEPWALK, PPR = 0, 1
+POLICY_SELECTIVE, POLICY_ROUND_ROBIN = 0, 1
+INSERT_WARP_AGGREGATED, INSERT_DIRECT = 0, 1
+EMPTY = 0xFFFFFFFF
+
+EXPORTED = [
+    "lt_config_default", "lt_create", "lt_destroy", "lt_last_error", "lt_partition_bounds", "lt_graph_load",
+    "lt_graph_load_device", "lt_get_bounds", "lt_walks_init", "lt_walks_init_ex", "lt_run", "lt_path_stride",
+    "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
+]
+
+
+class Config(ctypes.Structure):
+    _fields_ = [
+        ("device", ctypes.c_int),
+        ("stream", ctypes.c_void_p),
+        ("chunk_walks", ctypes.c_uint32),
+        ("ppr_max_len", ctypes.c_uint32),
+        ("policy", ctypes.c_uint32),
+        ("insert_mode", ctypes.c_uint32),
+        ("timing", ctypes.c_uint32),
+        ("block_threads", ctypes.c_uint32),
+        ("blocks_per_sm", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 8),
+    ]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [(name, ctypes.c_uint64) for name in (
+        "num_walks", "steps", "visits", "truncated", "sweeps", "update_launches", "kernel_launches",
+        "chunks_total", "chunks_free_min", "h2d_bytes", "d2h_bytes")] + [
+        ("update_ms", ctypes.c_double), ("run_ms", ctypes.c_double), ("init_ms", ctypes.c_double)]
+
+
+class PoolState(ctypes.Structure):
+    _fields_ = [("free_chunks", ctypes.c_int64), ("ring_chunks", ctypes.c_uint64), ("reserved0", ctypes.c_uint64),
+                ("total_chunks", ctypes.c_uint64), ("pending", ctypes.c_uint64), ("finished", ctypes.c_uint64),
+                ("device_err", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+
+
+_vp = ctypes.c_void_p
+_u32, _u64 = ctypes.c_uint32, ctypes.c_uint64
+_lib.lt_config_default.argtypes = [ctypes.POINTER(Config)]
+_lib.lt_create.argtypes = [ctypes.POINTER(Config), ctypes.POINTER(_vp)]
+_lib.lt_destroy.argtypes = [_vp]
+_lib.lt_destroy.restype = None
+_lib.lt_last_error.restype = ctypes.c_char_p
+_lib.lt_partition_bounds.argtypes = [_u32, _vp, _u32, _vp]
+_lib.lt_graph_load.argtypes = [_vp, _u32, _u64, _vp, _vp, _u32]
+_lib.lt_graph_load_device.argtypes = [_vp, _u32, _u64, _vp, _vp, _u32]
+_lib.lt_get_bounds.argtypes = [_vp, _vp, ctypes.POINTER(_u32)]
+_lib.lt_walks_init.argtypes = [_vp, _u64, _vp, ctypes.c_int, ctypes.c_double, _u64]
+_lib.lt_walks_init_ex.argtypes = [_vp, _u64, _vp, ctypes.c_int, _u64, ctypes.c_int, ctypes.c_double, _u64]
+_lib.lt_run.argtypes = [_vp]
+_lib.lt_path_stride.argtypes = [_vp, ctypes.POINTER(_u32)]
+_lib.lt_get_paths.argtypes = [_vp, _vp, _vp]
+_lib.lt_get_paths_rows.argtypes = [_vp, _vp, _u64, _vp, _vp]
+_lib.lt_get_paths_device.argtypes = [_vp, _vp, _vp]
+_lib.lt_get_stats.argtypes = [_vp, ctypes.POINTER(Stats)]
+_lib.lt_get_pool_state.argtypes = [_vp, ctypes.POINTER(PoolState)]
+
+
+class LTError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"lt status {status}: {msg}")
+        self.status = status
+
+
+def _check(status):
+    if status != LT_OK:
+        raise LTError(status, _lib.lt_last_error().decode(errors="replace"))
+
+
+def _is_torch(x):
+    return type(x).__module__.startswith("torch")
+
+
+def _ptr(x, np_dtype):
+    """(pointer, on_device, keepalive) for a numpy array or torch tensor of the given bit width."""
+    if x is None:
+        return None, False, None
+    if _is_torch(x):
+        if not x.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        if x.element_size() != np.dtype(np_dtype).itemsize:
+            raise ValueError(f"tensor element size must be {np.dtype(np_dtype).itemsize}")
+        return x.data_ptr(), bool(x.is_cuda), x
+    a = np.ascontiguousarray(x)
+    if a.dtype != np_dtype:
+        if a.dtype.itemsize == np.dtype(np_dtype).itemsize and a.dtype.kind in "iu":
+            a = a.view(np_dtype)
+        else:
+            a = a.astype(np_dtype)
+    return a.ctypes.data, False, a
+
+
+def partition_bounds(row_ptr, num_partitions: int) -> np.ndarray:
+    """Host-only range partitioner (lt_partition_bounds)."""
+    p, dev, keep = _ptr(row_ptr, np.uint64)
+    assert not dev, "partition_bounds takes host row_ptr"
+    n = len(keep) - 1
+    out = np.zeros(num_partitions + 1, dtype=np.uint32)
+    _check(_lib.lt_partition_bounds(n, p, num_partitions, out.ctypes.data))
+    return out
+
+
+class Engine:
+    """One lt_ctx on one GPU."""
+
+    def __init__(self, device: int = 0, chunk_walks: int = 8192, ppr_max_len: int = 127,
+                 policy: int = POLICY_SELECTIVE, insert_mode: int = INSERT_WARP_AGGREGATED,
+                 timing: bool = False, stream=None, blocks_per_sm: int = 0):
+        cfg = Config()
+        _check(_lib.lt_config_default(ctypes.byref(cfg)))
+        cfg.device = device
+        cfg.stream = stream
+        cfg.chunk_walks = chunk_walks
+        cfg.ppr_max_len = ppr_max_len
+        cfg.policy = policy
+        cfg.insert_mode = insert_mode
+        cfg.timing = int(bool(timing))
+        cfg.blocks_per_sm = blocks_per_sm
+        h = _vp()
+        _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))
+        self._h = h
+        self._graph_keep = None
+        self.num_walks = 0
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.lt_destroy(self._h)
+            self._h = None
+        self._graph_keep = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    def graph_load(self, row_ptr, col, num_partitions: int):
+        prp, dev_r, krp = _ptr(row_ptr, np.uint64)
+        pcol, dev_c, kcol = _ptr(col, np.uint32)
+        if dev_r != dev_c:
+            raise ValueError("row_ptr and col must both be host or both be device")
+        n = (len(krp) if not _is_torch(krp) else krp.numel()) - 1
+        m = len(kcol) if not _is_torch(kcol) else kcol.numel()
+        if dev_r:
+            _check(_lib.lt_graph_load_device(self._h, n, m, prp, pcol, num_partitions))
+            self._graph_keep = (krp, kcol)  # borrowed device memory stays alive
+        else:
+            _check(_lib.lt_graph_load(self._h, n, m, prp, pcol, num_partitions))
+            self._graph_keep = None
+        self.n, self.m = n, m
+
+    def bounds(self) -> np.ndarray:
+        P = _u32()
+        _check(_lib.lt_get_bounds(self._h, None, ctypes.byref(P)))
+        out = np.zeros(P.value + 1, dtype=np.uint32)
+        _check(_lib.lt_get_bounds(self._h, out.ctypes.data, ctypes.byref(P)))
+        return out
+
+    def walks_init(self, starts, app: int = DEEPWALK, param: float = 80, seed: int = 1, first_walk_id: int = 0):
+        p, dev, keep = _ptr(starts, np.uint32)
+        W = keep.numel() if _is_torch(keep) else len(keep)
+        _check(_lib.lt_walks_init_ex(self._h, W, p, int(dev), first_walk_id, app, float(param), seed))
+        self._starts_keep = keep
+        self.num_walks = W
+
+    def run(self):
+        _check(_lib.lt_run(self._h))
+
+    def stride(self) -> int:
+        s = _u32()
+        _check(_lib.lt_path_stride(self._h, ctypes.byref(s)))
+        return s.value
+
+    def get_paths(self, paths=None, lengths=None):
+        """Copy paths/lengths to host. Pass preallocated (e.g. pinned torch) buffers to reuse them;
+        pass paths=False to skip the path matrix."""
+        W, S = self.num_walks, self.stride()
+        if paths is None:
+            paths = np.empty((W, S), dtype=np.uint32)
+        if lengths is None:
+            lengths = np.empty(W, dtype=np.uint32)
+        pp, dp, kp = _ptr(paths, np.uint32) if paths is not False else (None, False, None)
+        pl, dl, kl = _ptr(lengths, np.uint32)
+        if dp or dl:
+            raise ValueError("get_paths copies to host; use get_paths_device for device buffers")
+        _check(_lib.lt_get_paths(self._h, pp, pl))
+        return (paths if paths is not False else None), lengths
+
+    def get_paths_rows(self, rows):
+        rows = np.ascontiguousarray(rows, dtype=np.uint64)
+        S = self.stride()
+        out = np.empty((len(rows), S), dtype=np.uint32)
+        ln = np.empty(len(rows), dtype=np.uint32)
+        _check(_lib.lt_get_paths_rows(self._h, rows.ctypes.data, len(rows), out.ctypes.data, ln.ctypes.data))
+        return out, ln
+
+    def get_paths_device(self, d_paths, d_lengths):
+        pp, dp, _ = _ptr(d_paths, np.uint32)
+        pl, dl, _ = _ptr(d_lengths, np.uint32)
+        if (d_paths is not None and not dp) or (d_lengths is not None and not dl):
+            raise ValueError("get_paths_device needs CUDA tensors")
+        _check(_lib.lt_get_paths_device(self._h, pp, pl))
+
+    def pool_state(self) -> dict:
+        s = PoolState()
+        _check(_lib.lt_get_pool_state(self._h, ctypes.byref(s)))
+        return {name: getattr(s, name) for name, _ in PoolState._fields_}
+
+    def stats(self) -> dict:
+        s = Stats()
+        _check(_lib.lt_get_stats(self._h, ctypes.byref(s)))
+        return {name: getattr(s, name) for name, _ in Stats._fields_}

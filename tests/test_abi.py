@@ -1,0 +1,101 @@
+"""CPU checks of the C-ABI library: it loads, exports every symbol include/lt.h declares, its host
+partitioner is right, and it fails cleanly (status codes, no crash) without a GPU."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import lt_inputs
+import paper_conf_icde_xing0wxl23_b200 as LT
+from paper_conf_icde_xing0wxl23_b200 import lt as ltmod
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "lt.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(lt_[a-z_]+)\s*\(", src)))
+
+
+def test_exports_every_declared_symbol():
+    names = _declared()
+    assert len(names) >= 15
+    lib = ctypes.CDLL(ltmod.LIB_PATH)
+    for n in names:
+        assert hasattr(lib, n), n
+    assert sorted(ltmod.EXPORTED) == names
+
+
+def test_product_never_touches_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_icde_xing0wxl23_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cpp", ".h", ".cuh")):
+                s = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in s and "from oracle" not in s and "oracle.h" not in s, f
+
+
+def _brute_bounds(row_ptr, P):
+    n = len(row_ptr) - 1
+    cost = 8 * np.arange(n + 1, dtype=object) + 4 * np.asarray(row_ptr, dtype=object)
+    b = [0]
+    for k in range(1, P):
+        target = (cost[n] * k) // P if (cost[n] * k) % P == 0 else None
+        # lower_bound of the exact rational k*cost(n)/P
+        v = next(v for v in range(n + 1) if cost[v] * P >= cost[n] * k)
+        b.append(v)
+    b.append(n)
+    for k in range(1, P):
+        b[k] = max(b[k], b[k - 1] + 1)
+    for k in range(P - 1, 0, -1):
+        b[k] = min(b[k], b[k + 1] - 1)
+    return np.array(b, dtype=np.uint32)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 7, 16, 100])
+def test_partition_bounds_brute_force(P):
+    g = lt_inputs.rmat_cpu(9, 4000, seed=2)
+    b = LT.partition_bounds(g.row_ptr, P)
+    np.testing.assert_array_equal(b, _brute_bounds(g.row_ptr, P))
+    assert b[0] == 0 and b[-1] == g.n and np.all(np.diff(b.astype(np.int64)) >= 1)
+
+
+def test_partition_bounds_degenerate():
+    g = lt_inputs.small_graph([(0, 1), (1, 2), (2, 3)])
+    np.testing.assert_array_equal(LT.partition_bounds(g.row_ptr, 4), [0, 1, 2, 3, 4])   # P == n
+    # one huge vertex: bounds still strictly increasing
+    g = lt_inputs.small_graph([(0, k) for k in range(1, 50)])
+    b = LT.partition_bounds(g.row_ptr, 8)
+    assert np.all(np.diff(b.astype(np.int64)) >= 1) and b[-1] == 50
+    with pytest.raises(LT.LTError):
+        LT.partition_bounds(g.row_ptr, 0)
+    with pytest.raises(LT.LTError):
+        LT.partition_bounds(g.row_ptr, 51)
+
+
+def test_partition_bounds_balance_bytes():
+    g = lt_inputs.rmat_cpu(14, 16 * 2 ** 14, seed=1)
+    P = 16
+    b = LT.partition_bounds(g.row_ptr, P).astype(np.int64)
+    rp = g.row_ptr.astype(np.int64)
+    cost = 8 * b + 4 * rp[b]
+    part = np.diff(cost)
+    maxdeg_bytes = 8 + 4 * g.max_deg
+    assert part.max() - part.min() <= 2 * maxdeg_bytes + 16
+
+
+@pytest.mark.skipif(os.environ.get("CUDA_VISIBLE_DEVICES", None) is None and __import__("torch").cuda.is_available(),
+                    reason="GPU present: covered by gpu tests")
+def test_create_without_gpu_fails_cleanly():
+    with pytest.raises(LT.LTError) as ei:
+        LT.Engine()
+    assert ei.value.status in (ltmod.LT_ERR_CUDA, ltmod.LT_ERR_INVALID)
+
+
+def test_struct_layout_matches_header():
+    # lt_config: int + pad + void* + 7 u32 + 8 u32 -> 8 + 8 + 60 = 76 -> 80 with alignment
+    assert ctypes.sizeof(ltmod.Config) == 80
+    assert ctypes.sizeof(ltmod.Stats) == 11 * 8 + 3 * 8

@@ -1,0 +1,225 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, walk by walk, bit-exact.
+
+Paths are integer data, so the bar is exact equality of every path entry and every length
+(paths are a pure function of CSR, starts, app, parameter, seed and L_max, and must
+not depend on P, chunk size, scheduling policy, insertion mode or launch shape).
+"""
+import numpy as np
+import pytest
+
+import lt_inputs
+import oracle as O
+import paper_conf_icde_xing0wxl23_b200 as LT
+
+pytestmark = pytest.mark.gpu
+
+
+def run_gpu(g, starts, app, param, seed, P, first=0, device_inputs=False, **cfg):
+    import torch
+    with LT.Engine(**cfg) as e:
+        if device_inputs:
+            rp = torch.from_numpy(g.row_ptr.view(np.int64)).cuda()
+            col = torch.from_numpy(g.col.view(np.int32)).cuda()
+            st = torch.from_numpy(np.ascontiguousarray(starts).view(np.int32)).cuda()
+            e.graph_load(rp, col, P)
+            e.walks_init(st, app, param, seed, first)
+        else:
+            e.graph_load(g.row_ptr, g.col, P)
+            e.walks_init(starts, app, param, seed, first)
+        e.run()
+        paths, lengths = e.get_paths()
+        return paths, lengths, e.stats(), e.bounds()
+
+
+def run_oracle(g, starts, app, param, seed, first=0, lmax=O.DEFAULT_LMAX):
+    ids = np.arange(first, first + len(starts), dtype=np.uint64)
+    kw = dict(app=app, seed=seed, ids=ids, lmax=lmax)
+    if app == O.DEEPWALK:
+        kw["length"] = int(param)
+    else:
+        kw["alpha"] = param
+    return O.walks(g.row_ptr, g.col, starts, **kw)
+
+
+def assert_parity(g, starts, app, param, seed, P, first=0, **cfg):
+    paths, lengths, st, bounds = run_gpu(g, starts, app, param, seed, P, first=first, **cfg)
+    op, ol, osteps, otrunc = run_oracle(g, starts, app, param, seed, first=first,
+                                        lmax=cfg.get("ppr_max_len", O.DEFAULT_LMAX))
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)
+    assert st["steps"] == osteps
+    assert st["truncated"] == otrunc
+    assert st["num_walks"] == len(starts)
+    if len(starts):
+        assert st["visits"] >= len(starts)
+        if P == 1:
+            assert st["visits"] == len(starts) and st["update_launches"] == 1
+    assert len(bounds) == P + 1
+    return st
+
+
+@pytest.fixture(scope="module")
+def cfg1():
+    """BASELINE.json configs[0]: R-MAT scale 12, 65,536 tuples, 4096 DeepWalk walks, l=10, P=4."""
+    return lt_inputs.rmat_cpu(12, 65_536, seed=1)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_cfg1_deepwalk_exact(gpu, cfg1, seed):
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    st = assert_parity(cfg1, starts, LT.DEEPWALK, 10, seed, P=4)
+    assert st["steps"] == 4096 * 10
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 7, 64, 1000, 3336])
+def test_deepwalk_invariant_to_partition_count(gpu, cfg1, P):
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    assert_parity(cfg1, starts, LT.DEEPWALK, 10, 1, P=min(P, cfg1.n))
+
+
+@pytest.mark.parametrize("chunk", [64, 128, 1024, 8192])
+@pytest.mark.parametrize("insert_mode", [LT.INSERT_WARP_AGGREGATED, LT.INSERT_DIRECT])
+@pytest.mark.parametrize("policy", [LT.POLICY_SELECTIVE, LT.POLICY_ROUND_ROBIN])
+def test_invariant_to_pool_and_policy(gpu, cfg1, chunk, insert_mode, policy):
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    assert_parity(cfg1, starts, LT.DEEPWALK, 10, 2, P=16, chunk_walks=chunk, insert_mode=insert_mode,
+                  policy=policy)
+
+
+@pytest.mark.parametrize("alpha", [0.15, 0.5])
+@pytest.mark.parametrize("P", [1, 4, 64])
+def test_ppr_exact(gpu, cfg1, alpha, P):
+    starts = lt_inputs.ppr_starts(4096, cfg1.argmax_deg)
+    assert_parity(cfg1, starts, LT.PPR, alpha, 5, P=P, chunk_walks=256)
+
+
+def test_ppr_truncation(gpu, cfg1):
+    starts = lt_inputs.ppr_starts(3000, cfg1.argmax_deg)
+    st = assert_parity(cfg1, starts, LT.PPR, 0.01, 9, P=8, ppr_max_len=10)
+    assert st["truncated"] > 2000
+
+
+@pytest.mark.parametrize("W", [0, 1, 31, 33, 4097])
+def test_ragged_walk_counts(gpu, cfg1, W):
+    starts = lt_inputs.deepwalk_starts(W, cfg1.n)
+    assert_parity(cfg1, starts, LT.DEEPWALK, 7, 4, P=5)
+
+
+def test_zero_length_and_dead_ends(gpu):
+    g = lt_inputs.small_graph([(0, 1), (1, 3), (3, 4)], n=6)   # vertices 2 and 5 isolated (d == 0)
+    starts = np.array([0, 2, 5, 4, 1, 2], dtype=np.uint32)
+    assert_parity(g, starts, LT.DEEPWALK, 9, 1, P=3)
+    assert_parity(g, starts, LT.DEEPWALK, 0, 1, P=2)
+    assert_parity(g, starts, LT.PPR, 0.2, 1, P=6)
+
+
+def test_first_walk_id_offsets_philox_counter(gpu, cfg1):
+    starts = lt_inputs.deepwalk_starts(1000, cfg1.n, first_walk_id=123_456_789)
+    assert_parity(cfg1, starts, LT.DEEPWALK, 10, 1, P=4, first=123_456_789)
+    assert_parity(cfg1, starts, LT.DEEPWALK, 10, 1, P=4, first=(1 << 32) + 5)
+
+
+def test_device_inputs(gpu, cfg1):
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    a = run_gpu(cfg1, starts, LT.DEEPWALK, 10, 3, P=4, device_inputs=True)
+    b = run_gpu(cfg1, starts, LT.DEEPWALK, 10, 3, P=4)
+    np.testing.assert_array_equal(a[0], b[0])
+    op, ol, _, _ = run_oracle(cfg1, starts, LT.DEEPWALK, 10, 3)
+    np.testing.assert_array_equal(a[0], op)
+
+
+def test_repeated_epochs_and_sampled_rows(gpu, cfg1):
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 8)
+        for seed in (1, 2, 1):
+            e.walks_init(starts, LT.DEEPWALK, 10, seed)
+            e.run()
+            p, l = e.get_paths()
+            op, ol, _, _ = run_oracle(cfg1, starts, LT.DEEPWALK, 10, seed)
+            np.testing.assert_array_equal(p, op)
+        rows = np.array([0, 5, 4095, 77], dtype=np.uint64)
+        rp, rl = e.get_paths_rows(rows)
+        np.testing.assert_array_equal(rp, op[rows.astype(np.int64)])
+        np.testing.assert_array_equal(rl, ol[rows.astype(np.int64)])
+
+
+def test_errors_are_status_codes(gpu, cfg1):
+    with LT.Engine() as e:
+        with pytest.raises(LT.LTError) as ei:
+            e.walks_init(np.zeros(4, np.uint32), LT.DEEPWALK, 5, 1)
+        assert ei.value.status == 2                     # STATE: no graph
+        e.graph_load(cfg1.row_ptr, cfg1.col, 4)
+        with pytest.raises(LT.LTError) as ei:
+            e.run()
+        assert ei.value.status == 2                     # STATE: no walks
+        with pytest.raises(LT.LTError) as ei:
+            e.walks_init(np.array([cfg1.n], np.uint32), LT.DEEPWALK, 5, 1)
+        assert ei.value.status == 1                     # INVALID start
+        for bad in (-1.0, 2.5):
+            with pytest.raises(LT.LTError):
+                e.walks_init(np.zeros(4, np.uint32), LT.DEEPWALK, bad, 1)
+        for bad in (0.0, 1.0):
+            with pytest.raises(LT.LTError):
+                e.walks_init(np.zeros(4, np.uint32), LT.PPR, bad, 1)
+        e.walks_init(np.zeros(4, np.uint32), LT.DEEPWALK, 5, 1)
+        e.run()
+        with pytest.raises(LT.LTError):
+            e.run()
+    with LT.Engine() as e:
+        bad_rp = cfg1.row_ptr.copy()
+        bad_rp[5] = bad_rp[6] + 1
+        with pytest.raises(LT.LTError):
+            e.graph_load(bad_rp, cfg1.col, 4)
+        bad_col = cfg1.col.copy()
+        bad_col[10] = cfg1.n
+        with pytest.raises(LT.LTError):
+            e.graph_load(cfg1.row_ptr, bad_col, 4)
+        with pytest.raises(LT.LTError):
+            e.graph_load(cfg1.row_ptr, cfg1.col, cfg1.n + 1)
+
+
+def test_scale16_two_walks_per_vertex(gpu):
+    g = lt_inputs.rmat_cpu(16, 16 * 65_536, seed=1)
+    starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+    assert_parity(g, starts, LT.DEEPWALK, 30, 1, P=32)
+    assert_parity(g, lt_inputs.ppr_starts(50_000, g.argmax_deg), LT.PPR, 0.15, 2, P=32)
+
+
+@pytest.mark.parametrize("P", [1, 16])
+def test_cfg2_lj_shaped_full_parity(gpu, P):
+    """BASELINE.json configs[1]: LJ-shaped R-MAT scale 22, 69M tuples, |V| DeepWalk walks, l=80,
+    HBM-resident; every walk compared."""
+    g = _cfg2()
+    starts = lt_inputs.deepwalk_starts(g.n, g.n)
+    st = assert_parity(g, starts, LT.DEEPWALK, 80, 1, P=P)
+    assert st["steps"] == g.n * 80
+
+
+_CFG2 = {}
+
+
+def _cfg2():
+    if "g" not in _CFG2:
+        _CFG2["g"] = lt_inputs.rmat_cpu(22, 69_000_000, seed=1)
+    return _CFG2["g"]
+
+
+@pytest.mark.parametrize("P,chunk", [(1, 8192), (4, 64), (16, 256), (64, 64)])
+def test_pool_invariants(gpu, cfg1, P, chunk):
+    """Conservation of walks and chunks (a6): after init every walk is pending in some bucket and
+    every chunk is either free or installed; after the run nothing is pending and nothing leaked."""
+    starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
+    with LT.Engine(chunk_walks=chunk) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, LT.DEEPWALK, 10, 1)
+        s0 = e.pool_state()
+        assert s0["device_err"] == 0, s0
+        assert s0["pending"] == 4096, s0
+        assert s0["free_chunks"] + s0["ring_chunks"] == s0["total_chunks"], s0
+        e.run()
+        s1 = e.pool_state()
+        assert s1["device_err"] == 0 and s1["pending"] == 0, s1
+        # only partially consumed chunks (at most one per partition) may stay installed
+        assert s1["ring_chunks"] <= P, s1
+        assert s1["free_chunks"] + s1["ring_chunks"] == s1["total_chunks"], s1

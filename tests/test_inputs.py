@@ -71,7 +71,7 @@ def test_small_graph_helper():
 
 def test_starts():
     assert list(lt_inputs.deepwalk_starts(5, 3)) == [0, 1, 2, 0, 1]
-    assert list(lt_inputs.deepwalk_starts(3, 4, first_walk=6)) == [2, 3, 0]
+    assert list(lt_inputs.deepwalk_starts(3, 4, first_walk_id=6)) == [2, 3, 0]
     assert list(lt_inputs.ppr_starts(3, 7)) == [7, 7, 7]
 
 
