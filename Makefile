@@ -12,7 +12,12 @@ LT_CU     := $(wildcard $(CSRC)/*.cu)
 LT_CPP    := $(wildcard $(CSRC)/*.cpp)
 LT_H      := $(wildcard $(CSRC)/*.h $(CSRC)/*.cuh) include/lt.h
 
-all: inputs oracle lt
+all: inputs oracle lt tools
+
+tools: tools/gather_bench
+
+tools/gather_bench: tools/gather_bench.cu
+	$(NVCC) $(ARCH) -O3 -lineinfo $< -o $@
 
 inputs: lt_inputs/libltgen.so
 oracle: oracle/liboracle.so
@@ -41,6 +46,6 @@ $(PKG)/liblt.so: $(LT_CU:.cu=.o) $(LT_CPP:.cpp=.o)
 	$(NVCC) $(ARCH) -shared $^ -o $@
 
 clean:
-	rm -f lt_inputs/*.o lt_inputs/*.so oracle/*.so $(CSRC)/*.o $(CSRC)/*.ptxas.txt $(PKG)/*.so
+	rm -f tools/gather_bench lt_inputs/*.o lt_inputs/*.so oracle/*.so $(CSRC)/*.o $(CSRC)/*.ptxas.txt $(PKG)/*.so
 
-.PHONY: all inputs oracle lt clean
+.PHONY: all inputs oracle lt tools clean

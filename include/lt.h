@@ -65,6 +65,12 @@ typedef enum {
   LT_INSERT_DIRECT = 1           /* one global atomic per walk ("direct write") */
 } lt_insert_mode;
 
+typedef enum {
+  LT_LAYOUT_AUTO = 0, /* ADJ when 16 B x m fits in half of the free device memory, else CSR */
+  LT_LAYOUT_CSR = 1,  /* steps gather row_ptr[v], row_ptr[v+1] and col[row_ptr[v] + i] */
+  LT_LAYOUT_ADJ = 2   /* steps gather adj[row_ptr[v] + i] = {u, deg(u), row_ptr[u]}: one access per step */
+} lt_layout;
+
 typedef struct lt_config {
   int device;                 /* CUDA ordinal */
   void* stream;               /* cudaStream_t to run on; NULL -> the legacy default stream */
@@ -75,7 +81,18 @@ typedef struct lt_config {
   uint32_t timing;            /* 1 -> CUDA events around every update launch (lt_stats.update_ms) */
   uint32_t block_threads;     /* update kernel block size (multiple of 32); 0 -> 256 */
   uint32_t blocks_per_sm;     /* update kernel resident blocks per SM for the grid; 0 -> occupancy */
-  uint32_t reserved[8];
+  uint32_t l2_fetch_bytes;    /* cudaLimitMaxL2FetchGranularity set at create: 0 -> 32 (random
+                                 sector gathers); 0xFFFFFFFF -> leave the device limit untouched */
+  uint32_t gather_mode;       /* L2 hints of the CSR gathers: 0 none, 1 col evict_first, 2 +row_ptr
+                                 evict_last, 3 col evict_first + L2::64B
+                                 ...; lt_config_default sets 3 */
+  uint32_t ilp;               /* walks advanced in lockstep per lane: 1, 2 or 4; 0 -> auto (1 with
+                                 the ADJ layout, 2 with CSR: the measured best) */
+  uint32_t layout;            /* lt_layout of the device graph the steps gather from */
+  uint32_t path_mode;         /* 0: path entries buffered and written as full 32-B sectors;
+                                 1: one 4-B store per step; 2: ABLATION, no path stores (paths
+                                 invalid; lengths and stats still exact) */
+  uint32_t reserved[3];
 } lt_config;
 
 typedef struct lt_stats {
@@ -93,9 +110,13 @@ typedef struct lt_stats {
   double update_ms;            /* sum of CUDA-event durations of update launches (if timing) */
   double run_ms;               /* CUDA-event duration of the last lt_run (first launch..last) */
   double init_ms;              /* CUDA-event duration of the last lt_walks_init* */
+  double graph_prep_ms;        /* device-side graph preparation in the last lt_graph_load* (ADJ build) */
+  uint32_t layout;             /* lt_layout in use (LT_LAYOUT_CSR or LT_LAYOUT_ADJ) */
+  uint32_t reserved;
 } lt_stats;
 
-/* Fill *cfg with defaults (device 0, library stream, C=8192, L_max=127, selective, aggregated). */
+/* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,
+ * gather_mode 3, ilp auto, layout auto, buffered path stores). */
 lt_status lt_config_default(lt_config* cfg);
 
 /* Create a context on cfg->device. No graph or walk memory is reserved yet. */

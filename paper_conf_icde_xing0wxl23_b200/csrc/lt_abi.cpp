@@ -55,6 +55,8 @@ struct lt_ctx {
   unsigned long long* d_row_ptr = nullptr;
   uint32_t* d_col = nullptr;
   bool own_graph = false;
+  uint4* d_adj = nullptr;  // augmented adjacency (layout ADJ), owned
+  size_t adj_cap = 0;
   std::vector<uint32_t> h_bounds;
   uint32_t* d_bounds = nullptr;
   size_t bounds_cap = 0;
@@ -63,7 +65,7 @@ struct lt_ctx {
   bool ran = false;
   uint64_t W = 0, first = 0, seed = 0;
   lt_app app = LT_APP_DEEPWALK;
-  uint32_t length = 0, T = 0, lmax = 127, stride = 1;
+  uint32_t length = 0, T = 0, lmax = 127, stride = 1, pitch = 8;
   uint32_t* d_paths = nullptr;
   size_t paths_cap = 0;
   uint32_t* d_lengths = nullptr;
@@ -100,6 +102,7 @@ lt_status lt_config_default(lt_config* cfg) {
   std::memset(cfg, 0, sizeof(*cfg));
   cfg->chunk_walks = 8192;
   cfg->ppr_max_len = 127;
+  cfg->gather_mode = 3;
   return LT_OK;
 }
 
@@ -114,7 +117,11 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.ppr_max_len == 0) c.ppr_max_len = 127;
   if (c.block_threads == 0) c.block_threads = 256;
   if (c.block_threads != 256) return fail(LT_ERR_INVALID, "block_threads must be 256 in this build");
-  if (c.policy > 1 || c.insert_mode > 1) return fail(LT_ERR_INVALID, "bad policy / insert_mode");
+  if (c.policy > 1 || c.insert_mode > 1 || c.gather_mode > 3)
+    return fail(LT_ERR_INVALID, "bad policy / insert_mode / gather_mode");
+  if (c.layout > 2) return fail(LT_ERR_INVALID, "bad layout");
+  if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
+  if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
   if (c.device < 0 || c.device >= ndev) return fail(LT_ERR_INVALID, "bad device ordinal");
@@ -124,7 +131,13 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   ctx->stream = (cudaStream_t)c.stream;
   ctx->block = c.block_threads;
   cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, c.device);
-  ctx->occ = c.blocks_per_sm ? (int)c.blocks_per_sm : lt::update_kernel_occupancy(ctx->block);
+  ctx->occ = 0;  // resolved per launch configuration in lt_walks_init
+  // Every gather on the path touches one random 32-B sector; a larger L2 fetch granularity only
+  // drags in neighbouring sectors nobody reads (measured: 2.5x DRAM read amplification at 64 B+).
+  if (c.l2_fetch_bytes != 0xFFFFFFFFu) {
+    size_t g = c.l2_fetch_bytes ? c.l2_fetch_bytes : 32;
+    CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, g));
+  }
   cudaError_t e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
   if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_ctr, sizeof(lt::Counters));
   if (e == cudaSuccess) e = cudaMallocHost((void**)&ctx->h_ctr, sizeof(lt::Counters));
@@ -143,6 +156,7 @@ void lt_destroy(lt_ctx* ctx) {
   cudaSetDevice(ctx->cfg.device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream); else cudaDeviceSynchronize();
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  cudaFree(ctx->d_adj);
   cudaFree(ctx->d_bounds);
   cudaFree(ctx->d_paths);
   cudaFree(ctx->d_lengths);
@@ -196,6 +210,24 @@ static lt_status validate_row_ptr(uint32_t n, uint64_t m, const uint64_t* row_pt
 }
 
 static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* h_row_ptr, uint32_t P) {
+  CK(cudaEventRecord(ctx->ev_a, ctx->stream));
+  // Layout: the augmented adjacency costs 16 B per CSR entry and saves one
+  // random DRAM access per step; auto-select it when it fits in half of the free device memory.
+  bool use_adj = ctx->cfg.layout == LT_LAYOUT_ADJ;
+  if (ctx->cfg.layout == LT_LAYOUT_AUTO) {
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    use_adj = m > 0 && (double)m * 16.0 <= 0.5 * (double)fr;
+  }
+  if (use_adj && m) {
+    CK(ensure(ctx->d_adj, ctx->adj_cap, m));
+    CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, m, ctx->d_adj, ctx->stream));
+  } else if (ctx->d_adj) {
+    cudaFree(ctx->d_adj);
+    ctx->d_adj = nullptr;
+    ctx->adj_cap = 0;
+  }
+  ctx->stats.layout = (use_adj && m) ? LT_LAYOUT_ADJ : LT_LAYOUT_CSR;
   std::vector<uint32_t> b(P + 1);
   lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
   if (s != LT_OK) return s;
@@ -208,6 +240,13 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     ctx->h_hc_cap = 0;
     CK(cudaMallocHost((void**)&ctx->h_hc, 2 * (size_t)P * sizeof(unsigned long long)));
     ctx->h_hc_cap = 2 * (size_t)P;
+  }
+  CK(cudaEventRecord(ctx->ev_b, ctx->stream));
+  CK(cudaEventSynchronize(ctx->ev_b));
+  {
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
+    ctx->stats.graph_prep_ms = ms;
   }
   ctx->h_bounds = std::move(b);
   ctx->n = n;
@@ -320,7 +359,8 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   const uint64_t ring_len = wc + 2;
   const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->P + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
-  CK(ensure(ctx->d_paths, ctx->paths_cap, std::max<uint64_t>(W, 1) * stride));
+  const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
+  CK(ensure(ctx->d_paths, ctx->paths_cap, std::max<uint64_t>(W, 1) * pitch));
   CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
   CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
   CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->P * ring_len));
@@ -336,10 +376,13 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   lt::Params& p = ctx->params;
   p.wk.row_ptr = ctx->d_row_ptr;
   p.wk.col = ctx->d_col;
+  p.wk.adj = ctx->d_adj;
   p.wk.bounds = ctx->d_bounds;
   p.wk.P = ctx->P;
   p.wk.paths = ctx->d_paths;
   p.wk.stride = stride;
+  p.wk.pitch = pitch;
+  p.wk.path_mode = ctx->cfg.path_mode;
   p.wk.lengths = ctx->d_lengths;
   p.wk.first_walk_id = first_walk_id;
   p.wk.seed_lo = (uint32_t)seed;
@@ -360,6 +403,10 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.pool.free_top = (int*)ctx->d_small;
   p.ctr = ctx->d_ctr;
   p.insert_mode = ctx->cfg.insert_mode;
+  p.gather_mode = ctx->cfg.gather_mode;
+  // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
+  p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : (ctx->d_adj ? 1u : 2u);
+  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp);
 
   ctx->W = W;
   ctx->first = first_walk_id;
@@ -369,6 +416,7 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   ctx->T = T;
   ctx->lmax = lmax;
   ctx->stride = stride;
+  ctx->pitch = pitch;
   ctx->stats.num_walks = W;
   ctx->stats.chunks_total = num_chunks;
   ctx->stats.kernel_launches = 0;
@@ -436,7 +484,8 @@ lt_status lt_run(lt_ctx* ctx) {
       // walks present at launch time <= pending now + everything launched before in this sweep
       const uint64_t bound = pend + earlier;
       earlier += pend;
-      const uint64_t grid = std::min<uint64_t>(std::max<uint64_t>((bound + ctx->block - 1) / ctx->block, 1), max_grid);
+      const uint64_t per_block = (uint64_t)ctx->block * p.ilp;
+      const uint64_t grid = std::min<uint64_t>(std::max<uint64_t>((bound + per_block - 1) / per_block, 1), max_grid);
       if (ctx->cfg.timing) {
         while (ctx->events.size() < nev + 2) {
           cudaEvent_t ev;
@@ -499,7 +548,8 @@ lt_status lt_get_paths(lt_ctx* ctx, uint32_t* paths, uint32_t* lengths) {
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
   if (paths && ctx->W) {
-    CK(cudaMemcpyAsync(paths, ctx->d_paths, ctx->W * ctx->stride * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpy2DAsync(paths, ctx->stride * sizeof(uint32_t), ctx->d_paths, ctx->pitch * sizeof(uint32_t),
+                         ctx->stride * sizeof(uint32_t), ctx->W, cudaMemcpyDeviceToHost, s));
     ctx->stats.d2h_bytes += ctx->W * ctx->stride * 4;
   }
   if (lengths && ctx->W) {
@@ -543,7 +593,8 @@ lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_length
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
   if (d_paths && ctx->W)
-    CK(cudaMemcpyAsync(d_paths, ctx->d_paths, ctx->W * ctx->stride * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    CK(cudaMemcpy2DAsync(d_paths, ctx->stride * sizeof(uint32_t), ctx->d_paths, ctx->pitch * sizeof(uint32_t),
+                         ctx->stride * sizeof(uint32_t), ctx->W, cudaMemcpyDeviceToDevice, s));
   if (d_lengths && ctx->W)
     CK(cudaMemcpyAsync(d_lengths, ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
   CK(cudaStreamSynchronize(s));

@@ -33,10 +33,13 @@ struct Pool {
 struct Walk {
   const unsigned long long* row_ptr;
   const uint32_t* col;
+  const uint4* adj;               // [m] augmented adjacency {u, deg(u), row_ptr[u]} or nullptr (CSR)
   const uint32_t* bounds;         // [P+1]
   uint32_t P;
   uint32_t* paths;
-  uint64_t stride;
+  uint64_t stride;                // logical row length: l+1 (DeepWalk) or L_max+1 (PPR)
+  uint64_t pitch;                 // physical row pitch in u32: stride rounded up to 8 (32-B sectors)
+  uint32_t path_mode;             // 0 buffered full-sector stores, 1 one store per step, 2 no stores (ablation)
   uint32_t* lengths;
   uint64_t first_walk_id;
   uint32_t seed_lo, seed_hi;
@@ -54,6 +57,8 @@ struct Params {
   Pool pool;
   Counters* ctr;
   uint32_t insert_mode;
+  uint32_t gather_mode;
+  uint32_t ilp;
 };
 
 // launchers (lt_kernels.cu); all asynchronous on `s`
@@ -65,7 +70,9 @@ cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, 
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
-int update_kernel_occupancy(uint32_t block);   // resident blocks per SM for the update kernel
+cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
+                             cudaStream_t s);
+int update_kernel_occupancy(uint32_t block, uint32_t ilp);  // resident blocks per SM (update kernel)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

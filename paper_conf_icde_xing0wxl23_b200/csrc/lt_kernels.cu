@@ -203,7 +203,7 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
     uint32_t dest = 0;
     if (have) {
       const uint32_t v = starts[i];
-      wk.paths[i * wk.stride] = v;
+      wk.paths[i * wk.pitch] = v;
       rec = make_uint4((uint32_t)i, v, 0u, 0u);
       dest = find_partition(B, wk.P, v);
     }
@@ -212,9 +212,50 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
   last_cta_retire(p, -1, 0, 0);
 }
 
+// Gather loads. GM selects L2 cache hints:
+//   0: plain ld.global.nc everywhere
+//   3: the per-step neighbour gather (col / adj) with an L2 evict_first policy (those lines are
+//      never reused) and the L2::64B prefetch-size hint (halves the DRAM bytes of each miss); the
+//      row_ptr gathers keep the default policy so the hot vertices' offsets stay in L2.
+struct Policies {
+  uint64_t first;
+};
+__device__ __forceinline__ Policies make_policies() {
+  Policies p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p.first));
+  return p;
+}
+template <int GM>
+__device__ __forceinline__ uint32_t ld_col(const uint32_t* p, const Policies& pol) {
+  if (GM == 0) return __ldg(p);
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol.first));
+  return v;
+}
+template <int GM>
+__device__ __forceinline__ uint4 ld_adj(const uint4* p, const Policies& pol) {
+  if (GM == 0) return __ldg(p);
+  uint4 v;
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p), "l"(pol.first));
+  return v;
+}
+
 // ------------------------------------------------------------------------------- a3 + a4 + a5
-template <int APP>
-__global__ void __launch_bounds__(256, 4) k_update(Params p, uint32_t k) {
+// ILP walks per lane: a warp takes 32*ILP consecutive records; each lane advances its ILP walks in
+// lockstep so their dependent gathers are in flight together (memory-level parallelism is what
+// bounds this kernel: the measured random-access rate of the HBM).
+// LAY selects the graph layout the step gathers from:
+//   0 (CSR): per step row_ptr[v], row_ptr[v+1] (one line) then col[off + i] (one line);
+//   1 (ADJ): per step ONE 16-B gather adj[off + i] = {u, deg(u), row_ptr[u]} that carries the next
+//            vertex's degree and offset, so only a visit's first step reads row_ptr.
+template <int ILP> struct MinBlocks { static constexpr int v = 4; };
+template <> struct MinBlocks<2> { static constexpr int v = 3; };
+template <> struct MinBlocks<4> { static constexpr int v = 2; };
+
+template <int APP, int GM, int ILP, int LAY>
+__global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
   const Pool& pl = p.pool;
@@ -226,55 +267,155 @@ __global__ void __launch_bounds__(256, 4) k_update(Params p, uint32_t k) {
   const uint32_t lane = threadIdx.x & 31u;
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
+  const Policies pol = make_policies();
   unsigned long long my_steps = 0, my_trunc = 0;
 
-  for (unsigned long long base = head + ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32;
-       base < tail; base += nwarps * 32) {
-    const unsigned long long pos = base + lane;
-    const bool have = pos < tail;
-    uint4 rec = make_uint4(0, 0, 0, 0);
-    bool left = false;
-    uint32_t dest = 0;
-    if (have) {
-      const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
-      rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
-      const uint32_t row = rec.x;
-      uint32_t v = rec.y, t = rec.z;
-      const uint64_t wid = wk.first_walk_id + row;
-      const uint32_t wlo = (uint32_t)wid, whi = (uint32_t)(wid >> 32);
-      uint32_t* prow = wk.paths + (uint64_t)row * wk.stride;
-      bool trunc = false;
-      for (;;) {
-        if (APP == 0) {
-          if (t == wk.length) break;
-        } else {
-          if (t == wk.lmax) { trunc = true; break; }
-        }
-        const uint4 b = philox10(make_uint4(t, 0u, wlo, whi), wk.seed_lo, wk.seed_hi);
-        if (APP == 1 && b.x < wk.T) break;
-        const unsigned long long off = __ldg(wk.row_ptr + v);
-        const unsigned long long end = __ldg(wk.row_ptr + v + 1);
-        const uint32_t d = (uint32_t)(end - off);
-        if (d == 0) break;
-        const uint64_t m = (uint64_t)b.y * d;
-        const uint32_t idx = ((uint32_t)m < d) ? lemire_slow(d, b, t, wlo, whi, wk.seed_lo, wk.seed_hi)
-                                               : (uint32_t)(m >> 32);
-        v = __ldg(wk.col + off + idx);
-        ++t;
-        prow[t] = v;
-        if (v - lo >= span) { left = true; break; }
+  for (unsigned long long base = head + ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * (32 * ILP);
+       base < tail; base += nwarps * (32 * ILP)) {
+    uint4 rec[ILP];  // .x = row, .y = current vertex v, .z = walked steps t
+    bool alive[ILP], left[ILP], trunc[ILP];
+    uint32_t* prow[ILP];
+    // Path entries are buffered per walk in a shift register (pb[s][7] = newest, entry t) and written
+    // as full 32-B sectors (two 16-B stores) whenever entry t closes a sector (t % 8 == 7); `nb`
+    // counts the buffered entries not yet in memory. The visit's first vertex (entry t0, already in
+    // memory) seeds the buffer so a sector that starts at t0 can still be written whole.
+    uint32_t pb[ILP][8];
+    uint32_t nb[ILP];
+    unsigned long long off[ILP];
+    uint32_t d[ILP];
+#pragma unroll
+    for (int s = 0; s < ILP; ++s) {
+      const unsigned long long pos = base + s * 32 + lane;
+      alive[s] = pos < tail;
+      left[s] = false;
+      trunc[s] = false;
+      rec[s] = make_uint4(0, 0, 0, 0);
+      if (alive[s]) {
+        const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
+        rec[s] = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
       }
-      if (left) {
-        dest = find_partition(B, wk.P, v);
-        rec.y = v;
-        rec.z = t;
-      } else {
-        wk.lengths[row] = t + 1;
-        my_steps += t;
-        my_trunc += trunc ? 1 : 0;
+      prow[s] = wk.paths + (uint64_t)rec[s].x * wk.pitch;
+      off[s] = 0;
+      d[s] = 0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) pb[s][q] = 0;
+      pb[s][7] = rec[s].y;
+      nb[s] = (alive[s] && (rec[s].z & 7u) == 0) ? 1u : 0u;  // entry t0 opens its sector: rewrite it too
+      if (LAY == 1 && alive[s]) {  // the visit's first vertex: its offset and degree from row_ptr
+        off[s] = __ldg(wk.row_ptr + rec[s].y);
+        d[s] = (uint32_t)(__ldg(wk.row_ptr + rec[s].y + 1) - off[s]);
       }
     }
-    insert_warp(p, left, dest, rec);
+    for (;;) {
+      bool any = false;
+#pragma unroll
+      for (int s = 0; s < ILP; ++s) {
+        if (alive[s]) {
+          if (APP == 0) {
+            if (rec[s].z == wk.length) alive[s] = false;
+          } else if (rec[s].z == wk.lmax) {
+            trunc[s] = true;
+            alive[s] = false;
+          }
+        }
+        any |= alive[s];
+      }
+      if (!any) break;
+      if (LAY == 0) {
+#pragma unroll
+        for (int s = 0; s < ILP; ++s) {  // issue every row_ptr gather first
+          if (alive[s]) {
+            off[s] = __ldg(wk.row_ptr + rec[s].y);
+            d[s] = (uint32_t)(__ldg(wk.row_ptr + rec[s].y + 1) - off[s]);
+          }
+        }
+      }
+      uint4 b[ILP];
+#pragma unroll
+      for (int s = 0; s < ILP; ++s) {  // Philox overlaps the gather latency (it needs only w and t)
+        const uint64_t wid = wk.first_walk_id + rec[s].x;
+        b[s] = philox10(make_uint4(rec[s].z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
+      }
+      uint32_t nv[ILP];
+#pragma unroll
+      for (int s = 0; s < ILP; ++s) {
+        nv[s] = 0;
+        if (APP == 1 && alive[s] && b[s].x < wk.T) alive[s] = false;  // terminate before moving
+        if (alive[s] && d[s] == 0) alive[s] = false;                   // dead end
+        if (alive[s]) {
+          const uint64_t m = (uint64_t)b[s].y * d[s];
+          const uint64_t wid = wk.first_walk_id + rec[s].x;
+          const uint32_t idx = ((uint32_t)m < d[s])
+                                   ? lemire_slow(d[s], b[s], rec[s].z, (uint32_t)wid, (uint32_t)(wid >> 32),
+                                                 wk.seed_lo, wk.seed_hi)
+                                   : (uint32_t)(m >> 32);
+          if (LAY == 0) {
+            nv[s] = ld_col<GM>(wk.col + off[s] + idx, pol);
+          } else {
+            const uint4 e = ld_adj<GM>(wk.adj + off[s] + idx, pol);
+            nv[s] = e.x;
+            d[s] = e.y;
+            off[s] = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+          }
+        }
+      }
+#pragma unroll
+      for (int s = 0; s < ILP; ++s) {
+        if (alive[s]) {
+          rec[s].y = nv[s];
+          rec[s].z += 1;
+          const uint32_t t = rec[s].z;
+          if (wk.path_mode == 0) {
+#pragma unroll
+            for (int q = 0; q < 7; ++q) pb[s][q] = pb[s][q + 1];
+            pb[s][7] = nv[s];
+            nb[s] += 1;
+            if ((t & 7u) == 7u) {  // entry t closes sector [t-7, t]
+              if (nb[s] == 8) {
+                uint4* dst = reinterpret_cast<uint4*>(prow[s] + (t - 7));
+                dst[0] = make_uint4(pb[s][0], pb[s][1], pb[s][2], pb[s][3]);
+                dst[1] = make_uint4(pb[s][4], pb[s][5], pb[s][6], pb[s][7]);
+              } else {
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                  if ((uint32_t)q < nb[s]) prow[s][t - q] = pb[s][7 - q];
+              }
+              nb[s] = 0;
+            }
+          } else if (wk.path_mode == 1) {
+            prow[s][t] = nv[s];
+          }
+          if (nv[s] - lo >= span) {
+            left[s] = true;
+            alive[s] = false;
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int s = 0; s < ILP; ++s) {  // flush the entries of an unfinished sector
+      if (wk.path_mode == 0) {
+        const uint32_t t = rec[s].z;
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          if ((uint32_t)q < nb[s]) prow[s][t - q] = pb[s][7 - q];
+      }
+    }
+#pragma unroll
+    for (int s = 0; s < ILP; ++s) {
+      const bool had = base + s * 32 + lane < tail;
+      uint32_t dest = 0;
+      if (had) {
+        if (left[s]) {
+          dest = find_partition(B, wk.P, rec[s].y);
+        } else {
+          wk.lengths[rec[s].x] = rec[s].z + 1;
+          my_steps += rec[s].z;
+          my_trunc += trunc[s] ? 1 : 0;
+        }
+      }
+      insert_warp(p, had && left[s], dest, rec[s]);
+    }
   }
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
@@ -296,7 +437,7 @@ __global__ void k_finalize(Params p, uint64_t W) {
       const int j = __ffs(todo) - 1;
       todo &= todo - 1;
       const uint32_t Lj = __shfl_sync(kFull, L, j);
-      uint32_t* prow = wk.paths + (base + j) * wk.stride;
+      uint32_t* prow = wk.paths + (base + j) * wk.pitch;
       for (uint64_t t = Lj + lane; t < wk.stride; t += 32) prow[t] = kEmpty;
     }
   }
@@ -309,7 +450,7 @@ __global__ void k_gather_rows(Params p, const unsigned long long* rows, uint64_t
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
        i += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t r = i / wk.stride, t = i % wk.stride;
-    out[i] = wk.paths[rows[r] * wk.stride + t];
+    out[i] = wk.paths[rows[r] * wk.pitch + t];
     if (t == 0) out_len[r] = wk.lengths[rows[r]];
   }
 }
@@ -352,12 +493,30 @@ int num_sms() {
 
 uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 
-int update_kernel_occupancy(uint32_t block) {
+int update_kernel_occupancy(uint32_t block, uint32_t ilp) {
   int nb = 0;
-  cudaFuncSetAttribute(k_update<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-  cudaFuncSetAttribute(k_update<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0>, (int)block, 0);
+  if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1>, (int)block, 0);
+  else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1>, (int)block, 0);
+  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1>, (int)block, 0);
   return nb > 0 ? nb : 1;
+}
+
+// Augmented adjacency (LAY 1): adj[i] = {u, deg(u), row_ptr[u] lo, row_ptr[u] hi} for u = col[i].
+__global__ void k_build_adj(const unsigned long long* __restrict__ row_ptr, const uint32_t* __restrict__ col,
+                            uint64_t m, uint4* __restrict__ adj) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = col[i];
+    const unsigned long long o = __ldg(row_ptr + u);
+    const uint32_t dg = (uint32_t)(__ldg(row_ptr + u + 1) - o);
+    adj[i] = make_uint4(u, dg, (uint32_t)o, (uint32_t)(o >> 32));
+  }
+}
+
+cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
+                             cudaStream_t s) {
+  if (!m) return cudaSuccess;
+  k_build_adj<<<num_sms() * 8, 256, 0, s>>>(row_ptr, col, m, adj);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cudaStream_t s) {
@@ -368,9 +527,41 @@ cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cud
   return cudaGetLastError();
 }
 
+template <int APP, int GM, int ILP, int LAY>
+void launch_update_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_update<APP, GM, ILP, LAY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         kSmemBoundsCap * 4);
+    attr = true;
+  }
+  k_update<APP, GM, ILP, LAY><<<grid, block, bounds_smem(p), s>>>(p, k);
+}
+
+template <int APP, int GM, int LAY>
+void launch_update_ilp(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  switch (p.ilp) {
+    case 1: launch_update_t<APP, GM, 1, LAY>(p, k, grid, block, s); break;
+    case 4: launch_update_t<APP, GM, 4, LAY>(p, k, grid, block, s); break;
+    default: launch_update_t<APP, GM, 2, LAY>(p, k, grid, block, s); break;
+  }
+}
+
+template <int APP>
+void launch_update_app(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  const bool adj = p.wk.adj != nullptr;
+  if (p.gather_mode == 0) {
+    if (adj) launch_update_ilp<APP, 0, 1>(p, k, grid, block, s);
+    else launch_update_ilp<APP, 0, 0>(p, k, grid, block, s);
+  } else {
+    if (adj) launch_update_ilp<APP, 3, 1>(p, k, grid, block, s);
+    else launch_update_ilp<APP, 3, 0>(p, k, grid, block, s);
+  }
+}
+
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  if (p.wk.app == 0) k_update<0><<<grid, block, bounds_smem(p), s>>>(p, k);
-  else k_update<1><<<grid, block, bounds_smem(p), s>>>(p, k);
+  if (p.wk.app == 0) launch_update_app<0>(p, k, grid, block, s);
+  else launch_update_app<1>(p, k, grid, block, s);
   return cudaGetLastError();
 }
 

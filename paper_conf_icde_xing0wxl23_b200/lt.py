@@ -14,7 +14,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "liblt.so")
+LIB_PATH = os.environ.get("LT_LIBRARY") or os.path.join(_HERE, "liblt.so")  # override: experiments only
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build the CUDA extension first (`make lt` or "
@@ -25,6 +25,7 @@ LT_OK, LT_ERR_INVALID, LT_ERR_STATE, LT_ERR_OOM, LT_ERR_CUDA, LT_ERR_NCCL = rang
 DEEPWALK, PPR = 0, 1
 POLICY_SELECTIVE, POLICY_ROUND_ROBIN = 0, 1
 INSERT_WARP_AGGREGATED, INSERT_DIRECT = 0, 1
+LAYOUT_AUTO, LAYOUT_CSR, LAYOUT_ADJ = 0, 1, 2
 EMPTY = 0xFFFFFFFF
 
 EXPORTED = [
@@ -45,7 +46,12 @@ class Config(ctypes.Structure):
         ("timing", ctypes.c_uint32),
         ("block_threads", ctypes.c_uint32),
         ("blocks_per_sm", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 8),
+        ("l2_fetch_bytes", ctypes.c_uint32),
+        ("gather_mode", ctypes.c_uint32),
+        ("ilp", ctypes.c_uint32),
+        ("layout", ctypes.c_uint32),
+        ("path_mode", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 3),
     ]
 
 
@@ -53,7 +59,8 @@ class Stats(ctypes.Structure):
     _fields_ = [(name, ctypes.c_uint64) for name in (
         "num_walks", "steps", "visits", "truncated", "sweeps", "update_launches", "kernel_launches",
         "chunks_total", "chunks_free_min", "h2d_bytes", "d2h_bytes")] + [
-        ("update_ms", ctypes.c_double), ("run_ms", ctypes.c_double), ("init_ms", ctypes.c_double)]
+        ("update_ms", ctypes.c_double), ("run_ms", ctypes.c_double), ("init_ms", ctypes.c_double),
+        ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
 class PoolState(ctypes.Structure):
@@ -133,7 +140,9 @@ class Engine:
 
     def __init__(self, device: int = 0, chunk_walks: int = 8192, ppr_max_len: int = 127,
                  policy: int = POLICY_SELECTIVE, insert_mode: int = INSERT_WARP_AGGREGATED,
-                 timing: bool = False, stream=None, blocks_per_sm: int = 0):
+                 timing: bool = False, stream=None, blocks_per_sm: int = 0, l2_fetch_bytes: int = 0,
+                 gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
+                 path_mode: int = 0):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -144,6 +153,11 @@ class Engine:
         cfg.insert_mode = insert_mode
         cfg.timing = int(bool(timing))
         cfg.blocks_per_sm = blocks_per_sm
+        cfg.l2_fetch_bytes = l2_fetch_bytes
+        cfg.gather_mode = gather_mode
+        cfg.ilp = ilp
+        cfg.layout = layout
+        cfg.path_mode = path_mode
         h = _vp()
         _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))
         self._h = h

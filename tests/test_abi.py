@@ -98,4 +98,4 @@ def test_create_without_gpu_fails_cleanly():
 def test_struct_layout_matches_header():
     # lt_config: int + pad + void* + 7 u32 + 8 u32 -> 8 + 8 + 60 = 76 -> 80 with alignment
     assert ctypes.sizeof(ltmod.Config) == 80
-    assert ctypes.sizeof(ltmod.Stats) == 11 * 8 + 3 * 8
+    assert ctypes.sizeof(ltmod.Stats) == 11 * 8 + 4 * 8 + 8

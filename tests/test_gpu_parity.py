@@ -223,3 +223,34 @@ def test_pool_invariants(gpu, cfg1, P, chunk):
         # only partially consumed chunks (at most one per partition) may stay installed
         assert s1["ring_chunks"] <= P, s1
         assert s1["free_chunks"] + s1["ring_chunks"] == s1["total_chunks"], s1
+
+
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("ilp", [1, 2, 4])
+@pytest.mark.parametrize("gather_mode", [0, 3])
+@pytest.mark.parametrize("P", [1, 8])
+def test_kernel_variants_exact(gpu, cfg1, layout, ilp, gather_mode, P):
+    """Layout (CSR vs augmented adjacency), walks per lane and cache hints change only how the
+    gathers are issued, never which neighbour is chosen."""
+    kw = dict(layout=layout, ilp=ilp, gather_mode=gather_mode, chunk_walks=256)
+    assert_parity(cfg1, lt_inputs.deepwalk_starts(3000, cfg1.n), LT.DEEPWALK, 12, 7, P=P, **kw)
+    assert_parity(cfg1, lt_inputs.ppr_starts(3000, cfg1.argmax_deg), LT.PPR, 0.2, 7, P=P, **kw)
+    g = lt_inputs.small_graph([(0, 1), (1, 3), (3, 4)], n=6)
+    assert_parity(g, np.array([0, 2, 5, 4, 1, 2], dtype=np.uint32), LT.DEEPWALK, 9, 1, P=min(P, 6), **kw)
+
+
+@pytest.mark.parametrize("path_mode", [0, 1])
+@pytest.mark.parametrize("P", [1, 3, 16])
+@pytest.mark.parametrize("length", [0, 1, 7, 8, 9, 15, 16, 17, 80])
+def test_path_store_modes_and_sector_edges(gpu, cfg1, path_mode, P, length):
+    """Buffered full-sector path stores vs one store per step, at lengths around the 8-entry sector
+    boundaries, with visits that start mid-sector (P > 1)."""
+    assert_parity(cfg1, lt_inputs.deepwalk_starts(1500, cfg1.n), LT.DEEPWALK, length, 3, P=P, path_mode=path_mode)
+
+
+def test_path_mode_off_keeps_lengths(gpu, cfg1):
+    starts = lt_inputs.deepwalk_starts(2000, cfg1.n)
+    paths, lengths, st, _ = run_gpu(cfg1, starts, LT.PPR, 0.15, 4, P=4, path_mode=2)
+    _, ol, osteps, _ = run_oracle(cfg1, starts, LT.PPR, 0.15, 4)
+    np.testing.assert_array_equal(lengths, ol)
+    assert st["steps"] == osteps
