@@ -11,10 +11,13 @@ a3-a7). Workload (default): BASELINE.json configs[3], the Friendster-shaped R-MA
             on the stream the library launches on, max over ranks.
   e2e       the same metric through the C ABI with HOST buffers: pinned starts copied H2D inside
             lt_walks_init, and every path and length copied D2H by lt_get_paths, per step.
-  roofline  the update kernel (the dominant kernel): algorithmic bytes per launch (DESIGN.md
-            "Roofline": 32 B row_ptr sector + 32 B col sector + 4 B path entry per step, 16 B record
-            read per visit, 16 B record write per partition change, 4 B length per finished walk)
-            / its CUDA-event-timed average launch duration, against MEASURED_PEAKS.json hbm_gbs.
+  roofline  the update kernel (the dominant kernel): algorithmic bytes per launch / its CUDA-event
+            timed average launch duration, against MEASURED_PEAKS.json hbm_gbs. Algorithmic bytes are
+            SURVEY.md §8(d)'s per-unit figures at 32-B sector granularity with no cache reuse (DESIGN.md
+            "Roofline"): 104 B per step (row_ptr pair 40 + col 32 + path entry 32) plus 16 B per
+            record read (every visit) and 16 B per record write (every partition change).
+            `gather` adds the measured random-access view: DRAM-missing gathers per second against
+            the ceiling tools/gather_bench measured on this pool (profiles/gather_ceiling.json).
   cpu_baseline  the CPU oracle (oracle/, as it stands) on this box's host cores over a bounded
             sample of the same workload's walks (rank 0, N=1 only).
 
@@ -59,6 +62,9 @@ def parse():
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
+    ap.add_argument("--layout", type=int, default=0, help="0 auto, 1 CSR, 2 ADJ (lt_layout)")
+    ap.add_argument("--ilp", type=int, default=0)
+    ap.add_argument("--path-mode", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", default="", help="comma list of P values to time (extra key)")
@@ -142,7 +148,7 @@ def oracle_sample(c, g_host, W, first, seconds, threads=0):
     kw = dict(app=app, length=int(c.get("length", 0)), alpha=float(c.get("alpha", 0.15)), seed=c["seed"],
               threads=threads)
     # calibrate on a small prefix, then size the sample for ~`seconds` of work
-    n0 = min(W, 20_000)
+    n0 = min(W, 200_000)
     st = starts_for(c, g_host, n0, first)
     t0 = time.perf_counter()
     O.walks(g_host.row_ptr, g_host.col, st, ids=np.arange(first, first + n0, dtype=np.uint64), **kw)
@@ -259,8 +265,10 @@ def main():
     starts_d = torch.from_numpy(starts_h.view(np.int32)).cuda(local)
 
     eng = LT.Engine(device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
-                    timing=True)
+                    timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode)
+    t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
+    load_s = time.time() - t0
 
     def barrier():
         torch.cuda.synchronize()
@@ -303,7 +311,7 @@ def main():
     visits = sum(s["visits"] for s in stats)
     steps_k = steps_local
     moves = visits - len(stats) * W  # each walk's final visit ends in termination, every other visit in a move
-    alg_bytes = steps_k * (32 + 32 + 4) + visits * 16 + moves * 16 + len(stats) * W * 4
+    alg_bytes = steps_k * 104 + visits * 16 + moves * 16
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
     if os.path.exists(peaks_path):
@@ -313,18 +321,31 @@ def main():
     prof = os.path.join(ROOT, "profiles", "update_kernel_traffic.json")
     if os.path.exists(prof):
         pj = json.load(open(prof))
-        if pj.get("config_key") == f"cfg{args.config}-P{P}-C{args.chunk_walks}":
+        if pj.get("config_key") == f"cfg{args.config}-P{P}-layout{args.layout}":
             traffic = pj.get("dram_bytes_per_launch")
+    layout = stats[-1]["layout"]
+    # DRAM-missing random gathers issued by the update kernel: one per step (ADJ: adj entry;
+    # CSR: col entry) + the row_ptr line per step (CSR) or per visit (ADJ)
+    gathers = steps_k * (1 if layout == LT.LAYOUT_ADJ else 2) + (visits if layout == LT.LAYOUT_ADJ else 0)
+    gather = None
+    gc_path = os.path.join(ROOT, "profiles", "gather_ceiling.json")
+    if upd_ms > 0:
+        gather = {"gathers_per_s": gathers / (upd_ms / 1000.0), "per_step": gathers / max(1, steps_k)}
+        if os.path.exists(gc_path):
+            gc = json.load(open(gc_path))
+            gather["ceiling_per_s"] = gc["ceiling_gathers_per_s"]
+            gather["frac"] = gather["gathers_per_s"] / gc["ceiling_gathers_per_s"]
+            gather["ceiling_source"] = "profiles/gather_ceiling.json (tools/gather_bench)"
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "kernel": "k_update", "launches": upd_launches, "avg_launch_ms": upd_ms / max(1, upd_launches),
             "alg_bytes_per_step": alg_bytes / max(1, steps_k), "peak_source": peak_src,
-            "update_share_of_step": upd_ms / ms}
+            "update_share_of_step": upd_ms / ms, "gather": gather}
 
     # ---- extra partition-count sweep (context; the headline uses P above)
     sweep = {}
     for ps in [int(x) for x in args.sweep.split(",") if x.strip()]:
-        with LT.Engine(device=local, chunk_walks=args.chunk_walks, timing=True) as e2:
+        with LT.Engine(device=local, chunk_walks=args.chunk_walks, timing=True, layout=args.layout) as e2:
             e2.graph_load(g.row_ptr, g.col, ps)
             for _ in range(2):
                 e2.walks_init(starts_d, app, param, args.seed, first)
@@ -406,7 +427,9 @@ def main():
                                              "insert_mode": "warp_aggregated" if args.insert_mode == 0 else "direct",
                                              "parallelism": f"replicas{world}" if world > 1 else "single",
                                              "l2": "inputs larger than L2 (CSR >> 126 MB); no flush",
-                                             "graph_gen_s": round(gen_s, 2)}),
+                                             "layout": "adj" if layout == LT.LAYOUT_ADJ else "csr",
+                                             "graph_gen_s": round(gen_s, 2), "graph_load_s": round(load_s, 2),
+                                             "graph_prep_ms": stats[-1]["graph_prep_ms"]}),
                 "clocks": ck, "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "parity_sample": parity,
                 "per_step": {"steps": last["steps"], "visits": last["visits"], "sweeps": last["sweeps"],
