@@ -56,8 +56,15 @@ typedef enum {
 } lt_app;
 
 typedef enum {
-  LT_POLICY_SELECTIVE = 0,  /* partitions in descending pending-walk order */
-  LT_POLICY_ROUND_ROBIN = 1 /* partitions in ID order (the ablation baseline) */
+  /* Partition scheduling policy; Table III's four columns.
+   * Resident mode uses only the order: selective = descending pending walks, else ID order.
+   * Out-of-core mode: selective = load the partition with the most walks and evict the resident one
+   * with the fewest; preemptive = run ready resident partitions while a load is in
+   * flight; round robin = load in ID order, evict FIFO, no preemption. */
+  LT_POLICY_SELECTIVE = 0,        /* PS + SS (LightTraffic's default) */
+  LT_POLICY_ROUND_ROBIN = 1,      /* baseline: round robin + FIFO */
+  LT_POLICY_SELECTIVE_ONLY = 2,   /* SS */
+  LT_POLICY_PREEMPTIVE_ONLY = 3   /* PS with round-robin loading + FIFO eviction */
 } lt_policy;
 
 typedef enum {
@@ -92,7 +99,14 @@ typedef struct lt_config {
   uint32_t path_mode;         /* 0: path entries buffered and written as full 32-B sectors;
                                  1: one 4-B store per step; 2: ABLATION, no path stores (paths
                                  invalid; lengths and stats still exact) */
-  uint32_t reserved[3];
+  uint32_t zero_copy;         /* out-of-core: 1 -> adaptive zero copy when alpha*w < S_p */
+  uint32_t zc_alpha_bytes;    /* alpha, bytes per walk; 0 -> 256 */
+  uint32_t pad0;
+  uint64_t graph_pool_bytes;  /* 0 -> HBM-resident graph; > 0 -> out-of-core: the CSR stays in pinned
+                                 host memory and a device graph pool of this many bytes caches
+                                 partitions. Every partition must fit one block
+                                 (block = the largest partition's CSR slice). */
+  uint32_t reserved[4];
 } lt_config;
 
 typedef struct lt_stats {
@@ -112,7 +126,16 @@ typedef struct lt_stats {
   double init_ms;              /* CUDA-event duration of the last lt_walks_init* */
   double graph_prep_ms;        /* device-side graph preparation in the last lt_graph_load* (ADJ build) */
   uint32_t layout;             /* lt_layout in use (LT_LAYOUT_CSR or LT_LAYOUT_ADJ) */
-  uint32_t reserved;
+  uint32_t out_of_core;        /* 1 if the graph is host-resident with a device graph pool */
+  /* out-of-core scheduler counters of the last lt_run (Table III) */
+  uint64_t iterations;         /* partitions selected by scheduler.iteration() */
+  uint64_t explicit_copies;    /* partitions copied into the graph pool */
+  uint64_t pool_hits;          /* selections whose partition was already resident */
+  uint64_t zero_copy_launches; /* selections served through zero copy */
+  uint64_t preemptive_launches;/* ready partitions run while a load was in flight */
+  uint64_t graph_h2d_bytes;    /* CSR bytes copied host -> device by the scheduler */
+  uint64_t pool_blocks;        /* m_g */
+  uint64_t pool_block_bytes;
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

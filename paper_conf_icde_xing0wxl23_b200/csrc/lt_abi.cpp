@@ -1,10 +1,11 @@
-// lt_abi.cpp — the C ABI (include/lt.h): context, validation, range partitioner (a1), pool
-// reservation (a6 sizing), and the host partition scheduler (a7; Alg. 2).
-#include "lt.h"
-#include "lt_internal.h"
+// lt_abi.cpp — the C ABI (include/lt.h): context, validation, range partitioner (a1), graph
+// loading (resident or out-of-core), pool reservation (a6 sizing) and outputs. The partition
+// scheduler (a7; Alg. 2) is in lt_sched.cpp.
+#include "lt_ctx.h"
 
 #include <algorithm>
 #include <cmath>
+#include <thread>
 #include <cstdio>
 #include <cstring>
 #include <numeric>
@@ -12,86 +13,17 @@
 #include <vector>
 
 namespace {
-
 thread_local std::string g_err;
+}  // namespace
 
+namespace lt {
 lt_status fail(lt_status s, const std::string& msg) {
   g_err = msg;
   return s;
 }
-
-#define CK(call)                                                                        \
-  do {                                                                                  \
-    cudaError_t _e = (call);                                                            \
-    if (_e != cudaSuccess)                                                              \
-      return fail(_e == cudaErrorMemoryAllocation ? LT_ERR_OOM : LT_ERR_CUDA,           \
-                  std::string(#call) + ": " + cudaGetErrorString(_e));                  \
-  } while (0)
-
-template <class T>
-cudaError_t ensure(T*& p, size_t& cap, size_t count) {
-  if (count <= cap && p) return cudaSuccess;
-  if (p) cudaFree(p);
-  p = nullptr;
-  cap = 0;
-  cudaError_t e = cudaMalloc((void**)&p, std::max<size_t>(count, 1) * sizeof(T));
-  if (e == cudaSuccess) cap = count;
-  return e;
-}
-
-}  // namespace
-
-struct lt_ctx {
-  lt_config cfg{};
-  cudaStream_t stream = nullptr;
-  int num_sms = 148;
-  int occ = 1;
-  uint32_t block = 256;
-  // graph
-  bool graph_loaded = false;
-  uint32_t n = 0;
-  uint64_t m = 0;
-  uint32_t P = 0;
-  unsigned long long* d_row_ptr = nullptr;
-  uint32_t* d_col = nullptr;
-  bool own_graph = false;
-  uint4* d_adj = nullptr;  // augmented adjacency (layout ADJ), owned
-  size_t adj_cap = 0;
-  std::vector<uint32_t> h_bounds;
-  uint32_t* d_bounds = nullptr;
-  size_t bounds_cap = 0;
-  // walks
-  bool walks_ready = false;
-  bool ran = false;
-  uint64_t W = 0, first = 0, seed = 0;
-  lt_app app = LT_APP_DEEPWALK;
-  uint32_t length = 0, T = 0, lmax = 127, stride = 1, pitch = 8;
-  uint32_t* d_paths = nullptr;
-  size_t paths_cap = 0;
-  uint32_t* d_lengths = nullptr;
-  size_t lengths_cap = 0;
-  uint32_t* d_starts = nullptr;
-  size_t starts_cap = 0;
-  // pool
-  uint4* d_slots = nullptr;
-  size_t slots_cap = 0;
-  uint32_t* d_ring = nullptr;
-  size_t ring_cap = 0;
-  unsigned long long* d_hc = nullptr;  // head[P] then cursor[P]
-  size_t hc_cap = 0;
-  uint32_t* d_free = nullptr;
-  size_t free_cap = 0;
-  uint32_t* d_small = nullptr;  // [0]=free_top [1]=unused [2..3]=scratch flags
-  lt::Counters* d_ctr = nullptr;
-  // pinned staging
-  unsigned long long* h_hc = nullptr;
-  size_t h_hc_cap = 0;
-  lt::Counters* h_ctr = nullptr;
-  lt::Params params{};
-  lt_stats stats{};
-  std::vector<cudaEvent_t> events;
-  cudaEvent_t ev_a = nullptr, ev_b = nullptr;
-};
+}  // namespace lt
+using lt::fail;
+using lt::ensure;
 
 extern "C" {
 
@@ -117,7 +49,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.ppr_max_len == 0) c.ppr_max_len = 127;
   if (c.block_threads == 0) c.block_threads = 256;
   if (c.block_threads != 256) return fail(LT_ERR_INVALID, "block_threads must be 256 in this build");
-  if (c.policy > 1 || c.insert_mode > 1 || c.gather_mode > 3)
+  if (c.policy > 3 || c.insert_mode > 1 || c.gather_mode > 3 || c.zero_copy > 1)
     return fail(LT_ERR_INVALID, "bad policy / insert_mode / gather_mode");
   if (c.layout > 2) return fail(LT_ERR_INVALID, "bad layout");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
@@ -151,10 +83,23 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   return LT_OK;
 }
 
+static void free_ooc(lt_ctx* ctx) {
+  lt::OutOfCore& o = ctx->ooc;
+  if (o.load_stream) cudaStreamSynchronize(o.load_stream);
+  for (auto e : o.ev_ready) cudaEventDestroy(e);
+  for (auto e : o.ev_used) cudaEventDestroy(e);
+  if (o.load_stream) cudaStreamDestroy(o.load_stream);
+  if (o.d_gpool) cudaFree(o.d_gpool);
+  if (o.h_row_ptr) cudaFreeHost(o.h_row_ptr);
+  if (o.h_col) cudaFreeHost(o.h_col);
+  ctx->ooc = lt::OutOfCore();
+}
+
 void lt_destroy(lt_ctx* ctx) {
   if (!ctx) return;
   cudaSetDevice(ctx->cfg.device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream); else cudaDeviceSynchronize();
+  free_ooc(ctx);
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   cudaFree(ctx->d_adj);
   cudaFree(ctx->d_bounds);
@@ -213,8 +158,8 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   CK(cudaEventRecord(ctx->ev_a, ctx->stream));
   // Layout: the augmented adjacency costs 16 B per CSR entry and saves one
   // random DRAM access per step; auto-select it when it fits in half of the free device memory.
-  bool use_adj = ctx->cfg.layout == LT_LAYOUT_ADJ;
-  if (ctx->cfg.layout == LT_LAYOUT_AUTO) {
+  bool use_adj = ctx->cfg.layout == LT_LAYOUT_ADJ && !ctx->ooc.on;
+  if (ctx->cfg.layout == LT_LAYOUT_AUTO && !ctx->ooc.on) {
     size_t fr = 0, tot = 0;
     CK(cudaMemGetInfo(&fr, &tot));
     use_adj = m > 0 && (double)m * 16.0 <= 0.5 * (double)fr;
@@ -228,6 +173,7 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     ctx->adj_cap = 0;
   }
   ctx->stats.layout = (use_adj && m) ? LT_LAYOUT_ADJ : LT_LAYOUT_CSR;
+  ctx->stats.out_of_core = ctx->ooc.on ? 1 : 0;
   std::vector<uint32_t> b(P + 1);
   lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
   if (s != LT_OK) return s;
@@ -258,6 +204,63 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   return LT_OK;
 }
 
+// Out-of-core graph (a7/a8): G_cpu is a pinned, mapped host copy of the CSR;
+// the device graph pool holds m_g blocks, each big enough for the largest partition's row_ptr slice
+// (at offset 0) plus col slice (at rp_bytes).
+static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row_ptr, const uint32_t* col,
+                                   bool src_on_device, uint32_t P) {
+  free_ooc(ctx);
+  lt::OutOfCore& o = ctx->ooc;
+  CK(cudaHostAlloc((void**)&o.h_row_ptr, ((size_t)n + 1) * 8, cudaHostAllocMapped | cudaHostAllocPortable));
+  CK(cudaHostAlloc((void**)&o.h_col, std::max<uint64_t>(m, 1) * 4, cudaHostAllocMapped | cudaHostAllocPortable));
+  if (src_on_device) {
+    CK(cudaMemcpy(o.h_row_ptr, row_ptr, ((size_t)n + 1) * 8, cudaMemcpyDeviceToHost));
+    if (m) CK(cudaMemcpy(o.h_col, col, m * 4, cudaMemcpyDeviceToHost));
+  } else {
+    std::memcpy(o.h_row_ptr, row_ptr, ((size_t)n + 1) * 8);
+    const unsigned nt = 8;
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < nt; ++t)
+      th.emplace_back([&, t] {
+        const uint64_t a = m * t / nt, b = m * (t + 1) / nt;
+        if (b > a) std::memcpy(o.h_col + a, col + a, (b - a) * 4);
+      });
+    for (auto& x : th) x.join();
+  }
+  CK(cudaHostGetDevicePointer((void**)&o.d_map_row_ptr, o.h_row_ptr, 0));
+  CK(cudaHostGetDevicePointer((void**)&o.d_map_col, o.h_col, 0));
+  std::vector<uint32_t> b(P + 1);
+  lt_status s = lt_partition_bounds(n, (const uint64_t*)o.h_row_ptr, P, b.data());
+  if (s != LT_OK) return s;
+  uint64_t rp_max = 0, col_max = 0;
+  for (uint32_t k = 0; k < P; ++k) {
+    rp_max = std::max<uint64_t>(rp_max, 8ull * (b[k + 1] - b[k] + 1));
+    col_max = std::max<uint64_t>(col_max, 4ull * (o.h_row_ptr[b[k + 1]] - o.h_row_ptr[b[k]]));
+  }
+  o.rp_bytes = (rp_max + 255) & ~255ull;
+  o.block_bytes = (o.rp_bytes + col_max + 255) & ~255ull;
+  uint64_t mg = ctx->cfg.graph_pool_bytes / o.block_bytes;
+  if (mg == 0)
+    return fail(LT_ERR_INVALID, "graph pool smaller than one partition (" + std::to_string(o.block_bytes) +
+                                    " B): raise num_partitions or graph_pool_bytes");
+  o.m_g = (uint32_t)std::min<uint64_t>(mg, P);
+  CK(cudaMalloc((void**)&o.d_gpool, (size_t)o.m_g * o.block_bytes));
+  o.block_of.assign(P, -1);
+  o.part_in.assign(o.m_g, -1);
+  o.loaded_at.assign(o.m_g, 0);
+  o.ev_ready.resize(o.m_g);
+  o.ev_used.resize(o.m_g);
+  for (uint32_t q = 0; q < o.m_g; ++q) {
+    CK(cudaEventCreateWithFlags(&o.ev_ready[q], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&o.ev_used[q], cudaEventDisableTiming));
+  }
+  CK(cudaStreamCreateWithFlags(&o.load_stream, cudaStreamNonBlocking));
+  o.on = true;
+  ctx->stats.pool_blocks = o.m_g;
+  ctx->stats.pool_block_bytes = o.block_bytes;
+  return LT_OK;
+}
+
 lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row_ptr, const uint32_t* col,
                         uint32_t P) {
   if (!ctx || !row_ptr || (m && !col)) return fail(LT_ERR_INVALID, "NULL argument");
@@ -270,8 +273,15 @@ lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   ctx->d_row_ptr = nullptr;
   ctx->d_col = nullptr;
-  ctx->own_graph = true;
   ctx->graph_loaded = false;
+  free_ooc(ctx);
+  if (ctx->cfg.graph_pool_bytes) {
+    ctx->own_graph = false;
+    lt_status so = setup_out_of_core(ctx, n, m, row_ptr, col, false, P);
+    if (so != LT_OK) return so;
+    return finish_graph_load(ctx, n, m, row_ptr, P);
+  }
+  ctx->own_graph = true;
   CK(cudaMalloc((void**)&ctx->d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t)));
   CK(cudaMalloc((void**)&ctx->d_col, std::max<uint64_t>(m, 1) * sizeof(uint32_t)));
   CK(cudaMemcpy(ctx->d_row_ptr, row_ptr, ((size_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
@@ -297,6 +307,15 @@ lt_status lt_graph_load_device(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64
   if (bad) return fail(LT_ERR_INVALID, "col entry >= n");
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   ctx->own_graph = false;
+  ctx->graph_loaded = false;
+  free_ooc(ctx);
+  if (ctx->cfg.graph_pool_bytes) {  // host-resident copy of the caller's device CSR
+    ctx->d_row_ptr = nullptr;
+    ctx->d_col = nullptr;
+    lt_status so = setup_out_of_core(ctx, n, m, d_row_ptr, d_col, true, P);
+    if (so != LT_OK) return so;
+    return finish_graph_load(ctx, n, m, h.data(), P);
+  }
   ctx->d_row_ptr = (unsigned long long*)d_row_ptr;
   ctx->d_col = (uint32_t*)d_col;
   return finish_graph_load(ctx, n, m, h.data(), P);
@@ -376,7 +395,9 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   lt::Params& p = ctx->params;
   p.wk.row_ptr = ctx->d_row_ptr;
   p.wk.col = ctx->d_col;
-  p.wk.adj = ctx->d_adj;
+  p.wk.vbase = 0;
+  p.wk.ebase = 0;
+  p.wk.adj = ctx->ooc.on ? nullptr : ctx->d_adj;
   p.wk.bounds = ctx->d_bounds;
   p.wk.P = ctx->P;
   p.wk.paths = ctx->d_paths;
@@ -439,10 +460,6 @@ lt_status lt_run(lt_ctx* ctx) {
   if (ctx->ran) return fail(LT_ERR_STATE, "lt_run already done for these walks; call lt_walks_init again");
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
-  lt::Params& p = ctx->params;
-  const uint32_t P = ctx->P;
-  const uint64_t max_grid = (uint64_t)ctx->num_sms * ctx->occ;
-  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
   {
     float ms = 0;
     CK(cudaEventSynchronize(ctx->ev_b));
@@ -452,59 +469,18 @@ lt_status lt_run(lt_ctx* ctx) {
   ctx->stats.sweeps = 0;
   ctx->stats.update_launches = 0;
   ctx->stats.update_ms = 0;
+  ctx->stats.iterations = 0;
+  ctx->stats.explicit_copies = 0;
+  ctx->stats.pool_hits = 0;
+  ctx->stats.zero_copy_launches = 0;
+  ctx->stats.preemptive_launches = 0;
+  ctx->stats.graph_h2d_bytes = 0;
   ctx->stats.chunks_free_min = ctx->stats.chunks_total;
-  size_t nev = 0;
-  std::vector<uint32_t> order;
-  order.reserve(P);
+  ctx->nev = 0;
   CK(cudaEventRecord(ctx->ev_a, s));
-  for (;;) {
-    // pending-walk counts at the sweep boundary (one small D2H + sync per sweep)
-    CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)P * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
-    uint32_t free_top = 0;
-    CK(cudaMemcpyAsync(&free_top, ctx->d_small, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    if (ctx->h_ctr->err) break;
-    ctx->stats.chunks_free_min = std::min<uint64_t>(ctx->stats.chunks_free_min, (uint64_t)(int)free_top);
-    const unsigned long long* head = ctx->h_hc;
-    const unsigned long long* cur = ctx->h_hc + P;
-    order.clear();
-    uint64_t total = 0;
-    for (uint32_t k = 0; k < P; ++k)
-      if (cur[k] > head[k]) { order.push_back(k); total += cur[k] - head[k]; }
-    if (total == 0) break;
-    if (ctx->stats.sweeps > max_len + 2)
-      return fail(LT_ERR_CUDA, "scheduler did not converge (walk count not decreasing)");
-    if (ctx->cfg.policy == LT_POLICY_SELECTIVE)  // most pending walks first
-      std::stable_sort(order.begin(), order.end(),
-                       [&](uint32_t a, uint32_t b) { return cur[a] - head[a] > cur[b] - head[b]; });
-    uint64_t earlier = 0;
-    for (uint32_t k : order) {
-      const uint64_t pend = cur[k] - head[k];
-      // walks present at launch time <= pending now + everything launched before in this sweep
-      const uint64_t bound = pend + earlier;
-      earlier += pend;
-      const uint64_t per_block = (uint64_t)ctx->block * p.ilp;
-      const uint64_t grid = std::min<uint64_t>(std::max<uint64_t>((bound + per_block - 1) / per_block, 1), max_grid);
-      if (ctx->cfg.timing) {
-        while (ctx->events.size() < nev + 2) {
-          cudaEvent_t ev;
-          CK(cudaEventCreate(&ev));
-          ctx->events.push_back(ev);
-        }
-        CK(cudaEventRecord(ctx->events[nev], s));
-      }
-      CK(lt::launch_update(p, k, (uint32_t)grid, ctx->block, s));
-      if (ctx->cfg.timing) {
-        CK(cudaEventRecord(ctx->events[nev + 1], s));
-        nev += 2;
-      }
-      ctx->stats.update_launches++;
-      ctx->stats.kernel_launches++;
-    }
-    ctx->stats.sweeps++;
-  }
-  CK(lt::launch_finalize_paths(p, ctx->W, s));
+  lt_status st = ctx->ooc.on ? lt::run_out_of_core(ctx) : lt::run_resident(ctx);
+  if (st != LT_OK) return st;
+  CK(lt::launch_finalize_paths(ctx->params, ctx->W, s));
   ctx->stats.kernel_launches++;
   CK(cudaEventRecord(ctx->ev_b, s));
   CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
@@ -514,7 +490,7 @@ lt_status lt_run(lt_ctx* ctx) {
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
     ctx->stats.run_ms = ms;
     double tot = 0;
-    for (size_t i = 0; i + 1 < nev; i += 2) {
+    for (size_t i = 0; i + 1 < ctx->nev; i += 2) {
       CK(cudaEventElapsedTime(&ms, ctx->events[i], ctx->events[i + 1]));
       tot += ms;
     }

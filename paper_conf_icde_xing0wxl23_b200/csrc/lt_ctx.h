@@ -1,0 +1,113 @@
+// lt_ctx.h — the library context behind the opaque lt_ctx handle (private to csrc/).
+#pragma once
+#include "lt.h"
+#include "lt_internal.h"
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+namespace lt {
+
+lt_status fail(lt_status s, const std::string& msg);
+
+template <class T>
+cudaError_t ensure(T*& p, size_t& cap, size_t count) {
+  if (count <= cap && p) return cudaSuccess;
+  if (p) cudaFree(p);
+  p = nullptr;
+  cap = 0;
+  cudaError_t e = cudaMalloc((void**)&p, std::max<size_t>(count, 1) * sizeof(T));
+  if (e == cudaSuccess) cap = count;
+  return e;
+}
+
+// Out-of-core graph state: the CSR lives in
+// pinned, mapped host memory (G_cpu); a graph pool of m_g equal blocks caches partitions on the
+// device; a load stream copies partitions in while the compute stream runs resident ones.
+struct OutOfCore {
+  bool on = false;
+  unsigned long long* h_row_ptr = nullptr;  // pinned + mapped, n+1
+  uint32_t* h_col = nullptr;                // pinned + mapped, m
+  unsigned long long* d_map_row_ptr = nullptr;  // device views of the mapped host arrays (zero copy)
+  uint32_t* d_map_col = nullptr;
+  char* d_gpool = nullptr;   // m_g blocks of block_bytes
+  size_t block_bytes = 0;
+  size_t rp_bytes = 0;       // bytes reserved for the row_ptr slice at the start of each block
+  uint32_t m_g = 0;
+  std::vector<int> block_of;   // partition -> block (-1: not resident)
+  std::vector<int> part_in;    // block -> partition (-1: free)
+  std::vector<uint64_t> loaded_at;  // block -> load sequence number (FIFO eviction)
+  std::vector<cudaEvent_t> ev_ready, ev_used;  // per block: load finished / last compute use
+  cudaStream_t load_stream = nullptr;
+};
+
+}  // namespace lt
+
+struct lt_ctx {
+  lt_config cfg{};
+  cudaStream_t stream = nullptr;
+  int num_sms = 148;
+  int occ = 1;
+  uint32_t block = 256;
+  // graph
+  bool graph_loaded = false;
+  uint32_t n = 0;
+  uint64_t m = 0;
+  uint32_t P = 0;
+  unsigned long long* d_row_ptr = nullptr;
+  uint32_t* d_col = nullptr;
+  bool own_graph = false;
+  uint4* d_adj = nullptr;  // augmented adjacency (layout ADJ), owned
+  size_t adj_cap = 0;
+  std::vector<uint32_t> h_bounds;
+  uint32_t* d_bounds = nullptr;
+  size_t bounds_cap = 0;
+  lt::OutOfCore ooc;
+  // walks
+  bool walks_ready = false;
+  bool ran = false;
+  uint64_t W = 0, first = 0, seed = 0;
+  lt_app app = LT_APP_DEEPWALK;
+  uint32_t length = 0, T = 0, lmax = 127, stride = 1, pitch = 8;
+  uint32_t* d_paths = nullptr;
+  size_t paths_cap = 0;
+  uint32_t* d_lengths = nullptr;
+  size_t lengths_cap = 0;
+  uint32_t* d_starts = nullptr;
+  size_t starts_cap = 0;
+  // pool
+  uint4* d_slots = nullptr;
+  size_t slots_cap = 0;
+  uint32_t* d_ring = nullptr;
+  size_t ring_cap = 0;
+  unsigned long long* d_hc = nullptr;  // head[P] then cursor[P]
+  size_t hc_cap = 0;
+  uint32_t* d_free = nullptr;
+  size_t free_cap = 0;
+  uint32_t* d_small = nullptr;  // [0]=free_top [1]=unused [2..3]=scratch flags
+  lt::Counters* d_ctr = nullptr;
+  // pinned staging
+  unsigned long long* h_hc = nullptr;
+  size_t h_hc_cap = 0;
+  lt::Counters* h_ctr = nullptr;
+  lt::Params params{};
+  lt_stats stats{};
+  std::vector<cudaEvent_t> events;
+  size_t nev = 0;
+  cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+};
+
+#define CK(call)                                                                        \
+  do {                                                                                  \
+    cudaError_t _e = (call);                                                            \
+    if (_e != cudaSuccess)                                                              \
+      return lt::fail(_e == cudaErrorMemoryAllocation ? LT_ERR_OOM : LT_ERR_CUDA,       \
+                      std::string(#call) + ": " + cudaGetErrorString(_e));              \
+  } while (0)
+
+namespace lt {
+lt_status run_resident(lt_ctx* ctx);
+lt_status run_out_of_core(lt_ctx* ctx);
+lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound);
+}  // namespace lt

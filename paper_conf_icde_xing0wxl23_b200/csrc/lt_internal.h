@@ -31,8 +31,13 @@ struct Pool {
 };
 
 struct Walk {
+  // The graph the update launch gathers from. Resident mode: the whole CSR (vbase = ebase = 0).
+  // Out-of-core mode: one partition's slice in a graph-pool block, row_ptr[0] is vertex vbase's
+  // offset and col[0] is CSR entry ebase (or the whole CSR mapped from pinned host for zero copy).
   const unsigned long long* row_ptr;
   const uint32_t* col;
+  uint32_t vbase;
+  unsigned long long ebase;
   const uint4* adj;               // [m] augmented adjacency {u, deg(u), row_ptr[u]} or nullptr (CSR)
   const uint32_t* bounds;         // [P+1]
   uint32_t P;

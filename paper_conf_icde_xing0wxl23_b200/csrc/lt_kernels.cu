@@ -325,8 +325,11 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
 #pragma unroll
         for (int s = 0; s < ILP; ++s) {  // issue every row_ptr gather first
           if (alive[s]) {
-            off[s] = __ldg(wk.row_ptr + rec[s].y);
-            d[s] = (uint32_t)(__ldg(wk.row_ptr + rec[s].y + 1) - off[s]);
+            // the loaded graph may be one partition's slice (out-of-core pool block or a zero-copy
+            // host view): row_ptr is indexed from vbase and col from ebase
+            const unsigned long long* rp = wk.row_ptr + (rec[s].y - wk.vbase);
+            off[s] = __ldg(rp) - wk.ebase;
+            d[s] = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
           }
         }
       }

@@ -1,0 +1,243 @@
+// lt_sched.cpp — the host partition scheduler (Alg. 2).
+//
+// Resident mode (the graph is in HBM): sweeps over the partitions with pending walks, in descending
+// pending order (selective) or ID order (round robin, :341), one update launch each.
+//
+// Out-of-core mode (cfg.graph_pool_bytes > 0): the CSR lives in pinned host memory (G_cpu, :112,
+// :214); a graph pool of m_g blocks caches partitions on the device (:112-118). Each iteration
+// picks a partition (selective: the most pending walks; round robin otherwise), makes it resident
+// by an explicit cudaMemcpyAsync on the load stream into a free block or the block of the resident
+// partition with the fewest pending walks (selective) / the oldest one (FIFO) (:200), or reads it
+// through zero copy when alpha * w < S_p (adaptive scheduling, :263-265); while the load is in
+// flight it runs ready resident partitions (preemptive scheduling, :194-198, Alg. 2 l.7-10).
+// Cross-stream dependencies use events: a block is overwritten only after its last compute use,
+// and a partition is computed only after its load finished (:208).
+#include "lt_ctx.h"
+
+#include <cstring>
+
+namespace lt {
+
+namespace {
+
+lt_status read_counts(lt_ctx* ctx) {
+  cudaStream_t s = ctx->stream;
+  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)ctx->P * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+  int free_top = 0;
+  CK(cudaMemcpyAsync(&free_top, ctx->d_small, sizeof(int), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  ctx->stats.chunks_free_min = std::min<uint64_t>(ctx->stats.chunks_free_min, (uint64_t)std::max(free_top, 0));
+  return LT_OK;
+}
+
+inline uint64_t pending(const lt_ctx* ctx, uint32_t k) { return ctx->h_hc[ctx->P + k] - ctx->h_hc[k]; }
+
+// cudaEventQuery without leaving cudaErrorNotReady behind for the next launch check
+bool event_done(cudaEvent_t e) {
+  const cudaError_t r = cudaEventQuery(e);
+  if (r == cudaErrorNotReady) (void)cudaGetLastError();
+  return r == cudaSuccess;
+}
+
+}  // namespace
+
+lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
+  cudaStream_t s = ctx->stream;
+  const uint64_t max_grid = (uint64_t)ctx->num_sms * ctx->occ;
+  const uint64_t per_block = (uint64_t)ctx->block * p.ilp;
+  const uint64_t grid = std::min<uint64_t>(std::max<uint64_t>((walks_bound + per_block - 1) / per_block, 1), max_grid);
+  if (ctx->cfg.timing) {
+    while (ctx->events.size() < ctx->nev + 2) {
+      cudaEvent_t ev;
+      CK(cudaEventCreate(&ev));
+      ctx->events.push_back(ev);
+    }
+    CK(cudaEventRecord(ctx->events[ctx->nev], s));
+  }
+  CK(launch_update(p, k, (uint32_t)grid, ctx->block, s));
+  if (ctx->cfg.timing) {
+    CK(cudaEventRecord(ctx->events[ctx->nev + 1], s));
+    ctx->nev += 2;
+  }
+  ctx->stats.update_launches++;
+  ctx->stats.kernel_launches++;
+  return LT_OK;
+}
+
+lt_status run_resident(lt_ctx* ctx) {
+  const uint32_t P = ctx->P;
+  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
+  std::vector<uint32_t> order;
+  order.reserve(P);
+  for (;;) {
+    lt_status st = read_counts(ctx);  // one small D2H + sync per sweep
+    if (st != LT_OK) return st;
+    if (ctx->h_ctr->err) return LT_OK;
+    order.clear();
+    uint64_t total = 0;
+    for (uint32_t k = 0; k < P; ++k)
+      if (pending(ctx, k)) { order.push_back(k); total += pending(ctx, k); }
+    if (total == 0) return LT_OK;
+    // every live walk advances >= 1 step per sweep, so sweeps <= max_len + 1
+    if (ctx->stats.sweeps > max_len + 2) return fail(LT_ERR_CUDA, "scheduler did not converge");
+    if (ctx->cfg.policy == LT_POLICY_SELECTIVE || ctx->cfg.policy == LT_POLICY_SELECTIVE_ONLY)
+      std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return pending(ctx, a) > pending(ctx, b); });
+    uint64_t earlier = 0;
+    for (uint32_t k : order) {
+      // walks present at launch time <= pending now + everything launched before in this sweep
+      const uint64_t bound = pending(ctx, k) + earlier;
+      earlier += pending(ctx, k);
+      st = launch_update_timed(ctx, ctx->params, k, bound);
+      if (st != LT_OK) return st;
+    }
+    ctx->stats.sweeps++;
+  }
+}
+
+// ------------------------------------------------------------------------------- out-of-core
+namespace {
+
+uint64_t partition_bytes(const lt_ctx* ctx, uint32_t k) {
+  const uint32_t v0 = ctx->h_bounds[k], v1 = ctx->h_bounds[k + 1];
+  return 8ull * (v1 - v0 + 1) + 4ull * (ctx->ooc.h_row_ptr[v1] - ctx->ooc.h_row_ptr[v0]);
+}
+
+// Params whose graph view is partition k's slice in block b, or the whole mapped host CSR.
+Params view_block(const lt_ctx* ctx, uint32_t k, int b) {
+  Params p = ctx->params;
+  const uint32_t v0 = ctx->h_bounds[k];
+  char* base = ctx->ooc.d_gpool + (size_t)b * ctx->ooc.block_bytes;
+  p.wk.row_ptr = reinterpret_cast<const unsigned long long*>(base);
+  p.wk.col = reinterpret_cast<const uint32_t*>(base + ctx->ooc.rp_bytes);
+  p.wk.vbase = v0;
+  p.wk.ebase = ctx->ooc.h_row_ptr[v0];
+  p.wk.adj = nullptr;
+  return p;
+}
+
+Params view_zero_copy(const lt_ctx* ctx) {
+  Params p = ctx->params;
+  p.wk.row_ptr = ctx->ooc.d_map_row_ptr;
+  p.wk.col = ctx->ooc.d_map_col;
+  p.wk.vbase = 0;
+  p.wk.ebase = 0;
+  p.wk.adj = nullptr;
+  return p;
+}
+
+lt_status load_partition(lt_ctx* ctx, uint32_t k, int b, uint64_t seq) {
+  OutOfCore& o = ctx->ooc;
+  const uint32_t v0 = ctx->h_bounds[k], v1 = ctx->h_bounds[k + 1];
+  const uint64_t e0 = o.h_row_ptr[v0], e1 = o.h_row_ptr[v1];
+  char* base = o.d_gpool + (size_t)b * o.block_bytes;
+  CK(cudaStreamWaitEvent(o.load_stream, o.ev_used[b], 0));  // the block's last reader is done
+  CK(cudaMemcpyAsync(base, o.h_row_ptr + v0, 8ull * (v1 - v0 + 1), cudaMemcpyHostToDevice, o.load_stream));
+  if (e1 > e0)
+    CK(cudaMemcpyAsync(base + o.rp_bytes, o.h_col + e0, 4ull * (e1 - e0), cudaMemcpyHostToDevice, o.load_stream));
+  CK(cudaEventRecord(o.ev_ready[b], o.load_stream));
+  if (o.part_in[b] >= 0) o.block_of[o.part_in[b]] = -1;
+  o.part_in[b] = (int)k;
+  o.block_of[k] = b;
+  o.loaded_at[b] = seq;
+  ctx->stats.explicit_copies++;
+  ctx->stats.graph_h2d_bytes += partition_bytes(ctx, k);
+  ctx->stats.h2d_bytes += partition_bytes(ctx, k);
+  return LT_OK;
+}
+
+lt_status compute_block(lt_ctx* ctx, uint32_t k) {
+  OutOfCore& o = ctx->ooc;
+  const int b = o.block_of[k];
+  CK(cudaStreamWaitEvent(ctx->stream, o.ev_ready[b], 0));
+  lt_status st = launch_update_timed(ctx, view_block(ctx, k, b), k, pending(ctx, k));
+  if (st != LT_OK) return st;
+  CK(cudaEventRecord(o.ev_used[b], ctx->stream));
+  return LT_OK;
+}
+
+}  // namespace
+
+lt_status run_out_of_core(lt_ctx* ctx) {
+  OutOfCore& o = ctx->ooc;
+  const uint32_t P = ctx->P;
+  const uint32_t pol = ctx->cfg.policy;
+  const bool selective = pol == LT_POLICY_SELECTIVE || pol == LT_POLICY_SELECTIVE_ONLY;
+  const bool preemptive = pol == LT_POLICY_SELECTIVE || pol == LT_POLICY_PREEMPTIVE_ONLY;
+  const uint64_t alpha = ctx->cfg.zc_alpha_bytes ? ctx->cfg.zc_alpha_bytes : 256;
+  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
+  // each iteration consumes >= 1 visit and a walk makes <= max_len + 1 visits
+  const uint64_t max_iters = ctx->W * (max_len + 1) + P + 64;
+  uint64_t seq = 0;
+  uint32_t rr = P - 1;  // round-robin cursor
+  for (;;) {
+    lt_status st = read_counts(ctx);  // Alg. 2 line 1: while active walks exist
+    if (st != LT_OK) return st;
+    if (ctx->h_ctr->err) return LT_OK;
+    uint64_t total = 0;
+    for (uint32_t k = 0; k < P; ++k) total += pending(ctx, k);
+    if (total == 0) return LT_OK;
+    if (ctx->stats.iterations > max_iters) return fail(LT_ERR_CUDA, "out-of-core scheduler did not converge");
+    // scheduler.iteration(): select partition i
+    uint32_t i = 0;
+    if (selective) {
+      for (uint32_t k = 1; k < P; ++k)
+        if (pending(ctx, k) > pending(ctx, i)) i = k;
+    } else {
+      do { rr = (rr + 1) % P; } while (!pending(ctx, rr));
+      i = rr;
+    }
+    ctx->stats.iterations++;
+    if (o.block_of[i] >= 0) {  // graph-pool hit
+      ctx->stats.pool_hits++;
+      st = compute_block(ctx, i);
+      if (st != LT_OK) return st;
+      continue;
+    }
+    // adaptive scheduling: zero copy when alpha * w < S_p (Alg. 2 l.3-4)
+    if (ctx->cfg.zero_copy && alpha * pending(ctx, i) < partition_bytes(ctx, i)) {
+      ctx->stats.zero_copy_launches++;
+      st = launch_update_timed(ctx, view_zero_copy(ctx), i, pending(ctx, i));
+      if (st != LT_OK) return st;
+      continue;
+    }
+    // explicit copy (Alg. 2 l.6): a free block, else evict (fewest pending walks / FIFO)
+    int b = -1;
+    for (uint32_t q = 0; q < o.m_g && b < 0; ++q)
+      if (o.part_in[q] < 0) b = (int)q;
+    if (b < 0) {
+      for (uint32_t q = 0; q < o.m_g; ++q) {
+        if (b < 0) { b = (int)q; continue; }
+        if (selective ? pending(ctx, o.part_in[q]) < pending(ctx, o.part_in[b]) : o.loaded_at[q] < o.loaded_at[b])
+          b = (int)q;
+      }
+    }
+    st = load_partition(ctx, i, b, ++seq);
+    if (st != LT_OK) return st;
+    // preemptive scheduling (Alg. 2 l.7-10): while the load stream is busy, run ready partitions
+    while (preemptive && !event_done(o.ev_ready[b])) {
+      int j = -1;
+      // prefer a full batch whose partition holds the fewest walks, else the most walks
+      const uint64_t full = ctx->params.pool.C;
+      for (uint32_t q = 0; q < o.m_g; ++q) {
+        const int k = o.part_in[q];
+        if (k < 0 || (uint32_t)k == i || !pending(ctx, k)) continue;
+        if (!event_done(o.ev_ready[q])) continue;
+        if (j < 0) { j = k; continue; }
+        const bool kf = pending(ctx, k) >= full, jf = pending(ctx, j) >= full;
+        if (kf != jf ? kf : (kf ? pending(ctx, k) < pending(ctx, j) : pending(ctx, k) > pending(ctx, j))) j = k;
+      }
+      if (j < 0) break;
+      ctx->stats.preemptive_launches++;
+      st = compute_block(ctx, (uint32_t)j);
+      if (st != LT_OK) return st;
+      st = read_counts(ctx);  // Alg. 2 l.10: cudaStreamSynchronize(compStream)
+      if (st != LT_OK) return st;
+      if (ctx->h_ctr->err) return LT_OK;
+    }
+    st = compute_block(ctx, i);
+    if (st != LT_OK) return st;
+  }
+}
+
+}  // namespace lt

@@ -23,7 +23,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 LT_OK, LT_ERR_INVALID, LT_ERR_STATE, LT_ERR_OOM, LT_ERR_CUDA, LT_ERR_NCCL = range(6)
 DEEPWALK, PPR = 0, 1
-POLICY_SELECTIVE, POLICY_ROUND_ROBIN = 0, 1
+POLICY_SELECTIVE, POLICY_ROUND_ROBIN, POLICY_SELECTIVE_ONLY, POLICY_PREEMPTIVE_ONLY = 0, 1, 2, 3
 INSERT_WARP_AGGREGATED, INSERT_DIRECT = 0, 1
 LAYOUT_AUTO, LAYOUT_CSR, LAYOUT_ADJ = 0, 1, 2
 EMPTY = 0xFFFFFFFF
@@ -51,7 +51,11 @@ class Config(ctypes.Structure):
         ("ilp", ctypes.c_uint32),
         ("layout", ctypes.c_uint32),
         ("path_mode", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 3),
+        ("zero_copy", ctypes.c_uint32),
+        ("zc_alpha_bytes", ctypes.c_uint32),
+        ("pad0", ctypes.c_uint32),
+        ("graph_pool_bytes", ctypes.c_uint64),
+        ("reserved", ctypes.c_uint32 * 4),
     ]
 
 
@@ -60,7 +64,10 @@ class Stats(ctypes.Structure):
         "num_walks", "steps", "visits", "truncated", "sweeps", "update_launches", "kernel_launches",
         "chunks_total", "chunks_free_min", "h2d_bytes", "d2h_bytes")] + [
         ("update_ms", ctypes.c_double), ("run_ms", ctypes.c_double), ("init_ms", ctypes.c_double),
-        ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+        ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
+        (name, ctypes.c_uint64) for name in (
+            "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes")]
 
 
 class PoolState(ctypes.Structure):
@@ -142,7 +149,8 @@ class Engine:
                  policy: int = POLICY_SELECTIVE, insert_mode: int = INSERT_WARP_AGGREGATED,
                  timing: bool = False, stream=None, blocks_per_sm: int = 0, l2_fetch_bytes: int = 0,
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
-                 path_mode: int = 0):
+                 path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
+                 zc_alpha_bytes: int = 0):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -158,6 +166,9 @@ class Engine:
         cfg.ilp = ilp
         cfg.layout = layout
         cfg.path_mode = path_mode
+        cfg.graph_pool_bytes = graph_pool_bytes
+        cfg.zero_copy = int(bool(zero_copy))
+        cfg.zc_alpha_bytes = zc_alpha_bytes
         h = _vp()
         _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))
         self._h = h

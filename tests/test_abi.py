@@ -95,7 +95,15 @@ def test_create_without_gpu_fails_cleanly():
     assert ei.value.status in (ltmod.LT_ERR_CUDA, ltmod.LT_ERR_INVALID)
 
 
-def test_struct_layout_matches_header():
-    # lt_config: int + pad + void* + 7 u32 + 8 u32 -> 8 + 8 + 60 = 76 -> 80 with alignment
-    assert ctypes.sizeof(ltmod.Config) == 80
-    assert ctypes.sizeof(ltmod.Stats) == 11 * 8 + 4 * 8 + 8
+def test_struct_layout_matches_header(tmp_path):
+    """The ctypes mirrors of lt_config / lt_stats / lt_pool_state match the C compiler's layout."""
+    import subprocess
+    src = tmp_path / "sz.c"
+    src.write_text('#include <stdio.h>\n#include <stddef.h>\n#include "lt.h"\nint main(){printf("%zu %zu %zu %zu %zu\\n",'
+                   ' sizeof(lt_config), sizeof(lt_stats), sizeof(lt_pool_state), offsetof(lt_config, graph_pool_bytes),'
+                   ' offsetof(lt_stats, iterations));}\n')
+    exe = tmp_path / "sz"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)], check=True)
+    sizes = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
+    assert sizes == [ctypes.sizeof(ltmod.Config), ctypes.sizeof(ltmod.Stats), ctypes.sizeof(ltmod.PoolState),
+                     ltmod.Config.graph_pool_bytes.offset, ltmod.Stats.iterations.offset]
