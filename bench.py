@@ -68,6 +68,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", default="", help="comma list of P values to time (extra key)")
+    ap.add_argument("--graph-pool-gb", type=float, default=0.0,
+                    help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
+    ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
     return ap.parse_args()
 
 
@@ -264,8 +267,10 @@ def main():
     starts_h = starts_for(c, g, W, first)
     starts_d = torch.from_numpy(starts_h.view(np.int32)).cuda(local)
 
+    ooc = args.graph_pool_gb > 0
     eng = LT.Engine(device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
-                    timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode)
+                    timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
+                    graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy))
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
@@ -365,6 +370,32 @@ def main():
                               "sweeps": sts[-1]["sweeps"], "update_launches": sts[-1]["update_launches"]}
 
     # ---- e2e through the C ABI with host buffers (pinned), H2D + D2H inside the timed region
+    # ---- out-of-core: host-link traffic of the timed steps against the measured pinned H2D bandwidth
+    host_link = None
+    if ooc:
+        gb = sum(s["graph_h2d_bytes"] for s in stats)
+        hb = torch.empty(1 << 30, dtype=torch.uint8, pin_memory=True)
+        db = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+        for _ in range(2):
+            db.copy_(hb, non_blocking=True)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(5):
+            db.copy_(hb, non_blocking=True)
+        b.record()
+        torch.cuda.synchronize()
+        h2d_peak = 5 * (1 << 30) / (a.elapsed_time(b) / 1000) / 1e9
+        del hb, db
+        last = stats[-1]
+        host_link = {"achieved_gbs": gb / (ms / 1000) / 1e9, "peak_gbs": h2d_peak,
+                     "peak_source": "pinned 1 GiB H2D copy, measured in this run",
+                     "frac": gb / (ms / 1000) / 1e9 / h2d_peak, "graph_h2d_bytes_per_step": gb / len(stats),
+                     "pool_blocks": last["pool_blocks"], "pool_block_bytes": last["pool_block_bytes"],
+                     "iterations": last["iterations"], "explicit_copies": last["explicit_copies"],
+                     "pool_hits": last["pool_hits"], "zero_copy_launches": last["zero_copy_launches"],
+                     "preemptive_launches": last["preemptive_launches"],
+                     "hit_rate": last["pool_hits"] / max(1, last["iterations"])}
+
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0:
         S = int(c["length"]) + 1 if c["app"] == "deepwalk" else 128
@@ -426,6 +457,8 @@ def main():
                                              "policy": "selective" if args.policy == 0 else "round_robin",
                                              "insert_mode": "warp_aggregated" if args.insert_mode == 0 else "direct",
                                              "parallelism": f"replicas{world}" if world > 1 else "single",
+                                             "mode": "out_of_core" if ooc else "hbm_resident",
+                                             "graph_pool_gb": args.graph_pool_gb if ooc else None,
                                              "l2": "inputs larger than L2 (CSR >> 126 MB); no flush",
                                              "layout": "adj" if layout == LT.LAYOUT_ADJ else "csr",
                                              "graph_gen_s": round(gen_s, 2), "graph_load_s": round(load_s, 2),
@@ -436,6 +469,8 @@ def main():
                              "update_launches": last["update_launches"], "run_ms": last["run_ms"],
                              "init_ms": last["init_ms"], "update_ms": last["update_ms"],
                              "chunks_total": last["chunks_total"], "chunks_free_min": last["chunks_free_min"]}}
+        if host_link:
+            line["host_link"] = host_link
         if sweep:
             line["partition_sweep"] = sweep
         print(json.dumps(line), flush=True)

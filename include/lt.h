@@ -106,7 +106,8 @@ typedef struct lt_config {
                                  host memory and a device graph pool of this many bytes caches
                                  partitions. Every partition must fit one block
                                  (block = the largest partition's CSR slice). */
-  uint32_t reserved[4];
+  uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
+  uint32_t reserved[2];
 } lt_config;
 
 typedef struct lt_stats {
@@ -192,6 +193,26 @@ lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, u
 lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_lengths);
 
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out);
+
+/* ---- Range ownership across GPUs (the north star's multi-GPU mode, not
+ * in the paper). With cfg.world = R > 1, rank r owns partitions [floor(P r / R), floor(P (r+1) / R));
+ * every rank calls every function with identical arguments. lt_walks_init keeps the walks whose
+ * start partition this rank owns. lt_run advances local walks until no owned bucket holds a walk;
+ * a walk whose next partition belongs to rank q is appended to send bucket q instead. The caller
+ * then runs a superstep exchange (paper_conf_icde_xing0wxl23_b200/dist.py):
+ *   lt_exchange_pack -> all-to-all of counts and 16-B records (NCCL via torch.distributed) ->
+ *   lt_exchange_insert -> lt_run ... until the global count of live walks is 0.
+ * Path rows then hold only the entries this rank wrote (others 0xFFFFFFFF) and lengths only the
+ * walks that ended here (others 0): the merged result is the element-wise min of the paths and the
+ * max of the lengths over ranks. Walk records carry walk indices, identical on every rank. */
+/* Walks waiting in owned buckets (*local) and in the send bucket of each rank (outgoing[world]). */
+lt_status lt_pending(lt_ctx* ctx, uint64_t* local, uint64_t* outgoing);
+/* Move every send bucket into d_send (device, 16-B records, grouped by destination rank in rank
+ * order); counts[world] (host) receives the number of records per destination (0 for this rank).
+ * LT_ERR_INVALID if capacity (records) is too small. */
+lt_status lt_exchange_pack(lt_ctx* ctx, void* d_send, uint64_t capacity, uint64_t* counts);
+/* Insert `count` received records (device memory) into the owned buckets. */
+lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count);
 
 /* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:
  * pending + finished == num_walks; free_chunks + ring_chunks == total_chunks. */

@@ -52,6 +52,8 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.policy > 3 || c.insert_mode > 1 || c.gather_mode > 3 || c.zero_copy > 1)
     return fail(LT_ERR_INVALID, "bad policy / insert_mode / gather_mode");
   if (c.layout > 2) return fail(LT_ERR_INVALID, "bad layout");
+  if (c.world == 0) c.world = 1;
+  if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
@@ -62,6 +64,8 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   ctx->cfg = c;
   ctx->stream = (cudaStream_t)c.stream;
   ctx->block = c.block_threads;
+  ctx->rank = c.rank;
+  ctx->world = c.world;
   cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, c.device);
   ctx->occ = 0;  // resolved per launch configuration in lt_walks_init
   // Every gather on the path touches one random 32-B sector; a larger L2 fetch granularity only
@@ -103,6 +107,7 @@ void lt_destroy(lt_ctx* ctx) {
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   cudaFree(ctx->d_adj);
   cudaFree(ctx->d_bounds);
+  cudaFree(ctx->d_owner);
   cudaFree(ctx->d_paths);
   cudaFree(ctx->d_lengths);
   cudaFree(ctx->d_starts);
@@ -179,13 +184,29 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   if (s != LT_OK) return s;
   CK(ensure(ctx->d_bounds, ctx->bounds_cap, P + 1));
   CK(cudaMemcpy(ctx->d_bounds, b.data(), (P + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice));
-  CK(ensure(ctx->d_hc, ctx->hc_cap, 2 * (size_t)P));
-  if (ctx->h_hc_cap < 2 * (size_t)P) {
+  // range ownership: rank r owns partitions [floor(P r / R), floor(P (r+1) / R))
+  const uint32_t R = ctx->world;
+  if (R > P) return fail(LT_ERR_INVALID, "need num_partitions >= world");
+  ctx->own_lo = (uint32_t)((uint64_t)P * ctx->rank / R);
+  ctx->own_hi = (uint32_t)((uint64_t)P * (ctx->rank + 1) / R);
+  ctx->nb = P + (R > 1 ? R : 0);
+  if (ctx->d_owner) cudaFree(ctx->d_owner);
+  ctx->d_owner = nullptr;
+  if (R > 1) {
+    std::vector<uint16_t> own(P);
+    for (uint32_t r = 0; r < R; ++r)
+      for (uint64_t q = (uint64_t)P * r / R; q < (uint64_t)P * (r + 1) / R; ++q) own[q] = (uint16_t)r;
+    CK(cudaMalloc((void**)&ctx->d_owner, P * sizeof(uint16_t)));
+    CK(cudaMemcpy(ctx->d_owner, own.data(), P * sizeof(uint16_t), cudaMemcpyHostToDevice));
+  }
+  const size_t nb = ctx->nb;
+  CK(ensure(ctx->d_hc, ctx->hc_cap, 2 * nb));
+  if (ctx->h_hc_cap < 2 * nb) {
     if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
     ctx->h_hc = nullptr;
     ctx->h_hc_cap = 0;
-    CK(cudaMallocHost((void**)&ctx->h_hc, 2 * (size_t)P * sizeof(unsigned long long)));
-    ctx->h_hc_cap = 2 * (size_t)P;
+    CK(cudaMallocHost((void**)&ctx->h_hc, 2 * nb * sizeof(unsigned long long)));
+    ctx->h_hc_cap = 2 * nb;
   }
   CK(cudaEventRecord(ctx->ev_b, ctx->stream));
   CK(cudaEventSynchronize(ctx->ev_b));
@@ -376,13 +397,13 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   while ((1ull << c_shift) < C) ++c_shift;
   const uint64_t wc = (W + C - 1) / C;
   const uint64_t ring_len = wc + 2;
-  const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->P + 64;
+  const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
   const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
   CK(ensure(ctx->d_paths, ctx->paths_cap, std::max<uint64_t>(W, 1) * pitch));
   CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
   CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
-  CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->P * ring_len));
+  CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
   CK(ensure(ctx->d_free, ctx->free_cap, num_chunks));
   if (on_device && W) {
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
@@ -418,8 +439,12 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.pool.num_chunks = (uint32_t)num_chunks;
   p.pool.ring = ctx->d_ring;
   p.pool.ring_len = (uint32_t)ring_len;
+  p.pool.nbuckets = ctx->nb;
   p.pool.head = ctx->d_hc;
-  p.pool.cursor = ctx->d_hc + ctx->P;
+  p.pool.cursor = ctx->d_hc + ctx->nb;
+  p.own.own_lo = ctx->own_lo;
+  p.own.own_hi = ctx->own_hi;
+  p.own.owner = ctx->d_owner;
   p.pool.free_list = ctx->d_free;
   p.pool.free_top = (int*)ctx->d_small;
   p.ctr = ctx->d_ctr;
@@ -445,6 +470,9 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   CK(lt::launch_pool_reset(p, s));
   ctx->stats.kernel_launches++;
   if (W) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
+  // with range ownership each rank writes only its share of every row: unwritten entries must
+  // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
+  if (W && ctx->world > 1) CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
   if (W) {
     CK(lt::launch_init(p, d_starts, W, s));
     ctx->stats.kernel_launches++;
@@ -457,10 +485,11 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
 lt_status lt_run(lt_ctx* ctx) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "lt_run before lt_walks_init");
-  if (ctx->ran) return fail(LT_ERR_STATE, "lt_run already done for these walks; call lt_walks_init again");
+  if (ctx->ran && ctx->world == 1)
+    return fail(LT_ERR_STATE, "lt_run already done for these walks; call lt_walks_init again");
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
-  {
+  if (!ctx->ran) {
     float ms = 0;
     CK(cudaEventSynchronize(ctx->ev_b));
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
@@ -480,8 +509,10 @@ lt_status lt_run(lt_ctx* ctx) {
   CK(cudaEventRecord(ctx->ev_a, s));
   lt_status st = ctx->ooc.on ? lt::run_out_of_core(ctx) : lt::run_resident(ctx);
   if (st != LT_OK) return st;
-  CK(lt::launch_finalize_paths(ctx->params, ctx->W, s));
-  ctx->stats.kernel_launches++;
+  if (ctx->world == 1) {  // with ownership the rows are pre-filled and merged by the caller
+    CK(lt::launch_finalize_paths(ctx->params, ctx->W, s));
+    ctx->stats.kernel_launches++;
+  }
   CK(cudaEventRecord(ctx->ev_b, s));
   CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
@@ -588,19 +619,67 @@ lt_status lt_get_pool_state(lt_ctx* ctx, lt_pool_state* out) {
   CK(cudaMemcpy(small, ctx->d_small, sizeof(small), cudaMemcpyDeviceToHost));
   lt::Counters c;
   CK(cudaMemcpy(&c, ctx->d_ctr, sizeof(c), cudaMemcpyDeviceToHost));
-  std::vector<uint32_t> ring((size_t)ctx->P * p.pool.ring_len);
+  std::vector<uint32_t> ring((size_t)ctx->nb * p.pool.ring_len);
   CK(cudaMemcpy(ring.data(), ctx->d_ring, ring.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
-  std::vector<unsigned long long> hc(2 * (size_t)ctx->P);
+  std::vector<unsigned long long> hc(2 * (size_t)ctx->nb);
   CK(cudaMemcpy(hc.data(), ctx->d_hc, hc.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
   std::vector<uint32_t> len(ctx->W);
   if (ctx->W) CK(cudaMemcpy(len.data(), ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToHost));
   out->free_chunks = small[0];
   out->total_chunks = p.pool.num_chunks;
   for (uint32_t r : ring) out->ring_chunks += (r != lt::kEmpty);
-  for (uint32_t k = 0; k < ctx->P; ++k) out->pending += hc[ctx->P + k] - hc[k];
+  for (uint32_t k = 0; k < ctx->nb; ++k) out->pending += hc[ctx->nb + k] - hc[k];
   if (ctx->ran) out->finished = ctx->W;  // every walk terminated
   else for (uint32_t l : len) out->finished += (l != 0 && l != lt::kEmpty);
   out->device_err = c.err;
+  return LT_OK;
+}
+
+lt_status lt_pending(lt_ctx* ctx, uint64_t* local, uint64_t* outgoing) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  CK(cudaSetDevice(ctx->cfg.device));
+  const size_t nb = ctx->nb;
+  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * nb * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  uint64_t loc = 0;
+  for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k) loc += ctx->h_hc[nb + k] - ctx->h_hc[k];
+  if (local) *local = loc;
+  if (outgoing)
+    for (uint32_t r = 0; r < ctx->world; ++r)
+      outgoing[r] = ctx->world > 1 ? ctx->h_hc[nb + ctx->P + r] - ctx->h_hc[ctx->P + r] : 0;
+  return LT_OK;
+}
+
+lt_status lt_exchange_pack(lt_ctx* ctx, void* d_send, uint64_t capacity, uint64_t* counts) {
+  if (!ctx || !counts) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  std::vector<uint64_t> out(ctx->world, 0);
+  lt_status st = lt_pending(ctx, nullptr, out.data());
+  if (st != LT_OK) return st;
+  uint64_t total = 0;
+  for (uint64_t c : out) total += c;
+  if (total > capacity) return fail(LT_ERR_INVALID, "send buffer too small: need " + std::to_string(total));
+  if (total && !d_send) return fail(LT_ERR_INVALID, "NULL send buffer");
+  uint64_t off = 0;
+  for (uint32_t r = 0; r < ctx->world; ++r) {
+    counts[r] = out[r];
+    if (!out[r]) continue;
+    CK(lt::launch_pack(ctx->params, ctx->P + r, (uint4*)d_send + off, out[r], ctx->stream));
+    ctx->stats.kernel_launches++;
+    off += out[r];
+  }
+  CK(cudaStreamSynchronize(ctx->stream));
+  return LT_OK;
+}
+
+lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  if (count && !d_recv) return fail(LT_ERR_INVALID, "NULL receive buffer");
+  CK(lt::launch_insert_records(ctx->params, (const uint4*)d_recv, count, ctx->stream));
+  if (count) ctx->stats.kernel_launches++;
+  CK(cudaStreamSynchronize(ctx->stream));
   return LT_OK;
 }
 

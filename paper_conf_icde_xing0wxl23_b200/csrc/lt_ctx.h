@@ -55,6 +55,9 @@ struct lt_ctx {
   uint32_t n = 0;
   uint64_t m = 0;
   uint32_t P = 0;
+  uint32_t nb = 0;             // buckets: P + (world > 1 ? world : 0)
+  uint32_t rank = 0, world = 1, own_lo = 0, own_hi = 0;
+  uint16_t* d_owner = nullptr;  // [P] owner rank per partition (world > 1)
   unsigned long long* d_row_ptr = nullptr;
   uint32_t* d_col = nullptr;
   bool own_graph = false;

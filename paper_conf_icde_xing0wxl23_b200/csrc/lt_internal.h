@@ -24,8 +24,9 @@ struct Pool {
   uint32_t num_chunks;            // + 1 trash chunk at index num_chunks (writes after OOM)
   uint32_t* ring;
   uint32_t ring_len;
-  unsigned long long* head;       // [P]
-  unsigned long long* cursor;     // [P]
+  uint32_t nbuckets;              // P partition buckets + one send bucket per other rank
+  unsigned long long* head;       // [nbuckets]
+  unsigned long long* cursor;     // [nbuckets]
   uint32_t* free_list;            // [num_chunks]
   int* free_top;
 };
@@ -57,10 +58,19 @@ struct Counters {
   uint32_t done_ctas;
 };
 
+// Range ownership across ranks (north star 8-GPU mode): this rank owns partitions
+// [own_lo, own_hi); a walk whose next partition q is owned elsewhere goes to the send bucket
+// P + owner[q]. world == 1: own_lo = 0, own_hi = P, no send buckets.
+struct Owner {
+  uint32_t own_lo, own_hi;
+  const uint16_t* owner;  // [P] rank of each partition (nullptr when world == 1)
+};
+
 struct Params {
   Walk wk;
   Pool pool;
   Counters* ctr;
+  Owner own;
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;
@@ -68,6 +78,8 @@ struct Params {
 
 // launchers (lt_kernels.cu); all asynchronous on `s`
 cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cudaStream_t s);
+cudaError_t launch_insert_records(const Params& p, const uint4* recs, uint64_t count, cudaStream_t s);
+cudaError_t launch_pack(const Params& p, uint32_t bucket, uint4* out, uint64_t count, cudaStream_t s);
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s);
 cudaError_t launch_finalize_paths(const Params& p, uint64_t W, cudaStream_t s);
 cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, uint64_t count,

@@ -188,7 +188,15 @@ __device__ __forceinline__ const uint32_t* stage_bounds(const Walk& wk, uint32_t
   return wk.bounds;
 }
 
+// Bucket of partition q seen from this rank: q itself when owned, else the send bucket of its owner.
+__device__ __forceinline__ uint32_t bucket_of(const Params& p, uint32_t q) {
+  if (q >= p.own.own_lo && q < p.own.own_hi) return q;
+  return p.wk.P + p.own.owner[q];
+}
+
 // ------------------------------------------------------------------------------------------ a2
+// Walk init: path[w][0] and insertion into the start partition's bucket. With range ownership
+// (world > 1) every rank sees every start and keeps the walks whose start partition it owns.
 __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restrict__ starts, uint64_t W) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
@@ -198,18 +206,58 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
   for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; base < W;
        base += nwarps * 32) {
     const uint64_t i = base + lane;
-    const bool have = i < W;
+    bool have = i < W;
     uint4 rec = make_uint4(0, 0, 0, 0);
     uint32_t dest = 0;
     if (have) {
       const uint32_t v = starts[i];
-      wk.paths[i * wk.pitch] = v;
-      rec = make_uint4((uint32_t)i, v, 0u, 0u);
       dest = find_partition(B, wk.P, v);
+      have = dest >= p.own.own_lo && dest < p.own.own_hi;
+      if (have) {
+        wk.paths[i * wk.pitch] = v;
+        rec = make_uint4((uint32_t)i, v, 0u, 0u);
+      }
     }
     insert_warp(p, have, dest, rec);
   }
   last_cta_retire(p, -1, 0, 0);
+}
+
+// a9 receive side: records that arrived from other ranks go into the buckets of their (owned)
+// partitions with the same warp-aggregated insertion.
+__global__ void __launch_bounds__(256) k_insert_records(Params p, const uint4* __restrict__ recs, uint64_t count) {
+  extern __shared__ uint32_t s_bounds[];
+  const Walk& wk = p.wk;
+  const uint32_t* B = stage_bounds(wk, s_bounds);
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; base < count;
+       base += nwarps * 32) {
+    const uint64_t i = base + lane;
+    const bool have = i < count;
+    uint4 rec = make_uint4(0, 0, 0, 0);
+    uint32_t dest = 0;
+    if (have) {
+      rec = recs[i];
+      dest = bucket_of(p, find_partition(B, wk.P, rec.y));
+    }
+    insert_warp(p, have, dest, rec);
+  }
+  last_cta_retire(p, -1, 0, 0);
+}
+
+// a9 send side: copy send bucket `bucket` ([head, cursor), read at launch) contiguously to `out`
+// and retire its chunks.
+__global__ void __launch_bounds__(256) k_pack(Params p, uint32_t bucket, uint4* __restrict__ out) {
+  const Pool& pl = p.pool;
+  const unsigned long long head = pl.head[bucket], tail = pl.cursor[bucket];
+  const uint32_t* ring_b = pl.ring + (uint64_t)bucket * pl.ring_len;
+  for (unsigned long long pos = head + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; pos < tail;
+       pos += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = ring_b[(pos >> pl.c_shift) % pl.ring_len];
+    out[pos - head] = pl.slots[((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))];
+  }
+  last_cta_retire(p, (int)bucket, head, tail);
 }
 
 // Gather loads. GM selects L2 cache hints:
@@ -410,7 +458,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
       uint32_t dest = 0;
       if (had) {
         if (left[s]) {
-          dest = find_partition(B, wk.P, rec[s].y);
+          dest = bucket_of(p, find_partition(B, wk.P, rec[s].y));
         } else {
           wk.lengths[rec[s].x] = rec[s].z + 1;
           my_steps += rec[s].z;
@@ -468,9 +516,9 @@ __global__ void k_pool_reset(Params p) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   for (uint64_t i = tid; i < pl.num_chunks; i += stride) pl.free_list[i] = (uint32_t)i;
-  const uint64_t nring = (uint64_t)p.wk.P * pl.ring_len;
+  const uint64_t nring = (uint64_t)pl.nbuckets * pl.ring_len;
   for (uint64_t i = tid; i < nring; i += stride) pl.ring[i] = kEmpty;
-  for (uint64_t i = tid; i < p.wk.P; i += stride) { pl.head[i] = 0; pl.cursor[i] = 0; }
+  for (uint64_t i = tid; i < pl.nbuckets; i += stride) { pl.head[i] = 0; pl.cursor[i] = 0; }
   if (tid == 0) {
     *pl.free_top = (int)pl.num_chunks;
     p.ctr->steps = 0; p.ctr->visits = 0; p.ctr->truncated = 0; p.ctr->err = 0; p.ctr->done_ctas = 0;
@@ -519,6 +567,23 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
                              cudaStream_t s) {
   if (!m) return cudaSuccess;
   k_build_adj<<<num_sms() * 8, 256, 0, s>>>(row_ptr, col, m, adj);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_insert_records(const Params& p, const uint4* recs, uint64_t count, cudaStream_t s) {
+  if (!count) return cudaSuccess;
+  uint64_t want = (count + 255) / 256;
+  uint32_t grid = (uint32_t)std::min<uint64_t>(want, (uint64_t)num_sms() * 8);
+  cudaFuncSetAttribute(k_insert_records, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
+  k_insert_records<<<grid, 256, bounds_smem(p), s>>>(p, recs, count);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pack(const Params& p, uint32_t bucket, uint4* out, uint64_t count, cudaStream_t s) {
+  if (!count) return cudaSuccess;
+  uint64_t want = (count + 255) / 256;
+  uint32_t grid = (uint32_t)std::min<uint64_t>(want, (uint64_t)num_sms() * 8);
+  k_pack<<<grid, 256, 0, s>>>(p, bucket, out);
   return cudaGetLastError();
 }
 

@@ -22,7 +22,7 @@ namespace {
 
 lt_status read_counts(lt_ctx* ctx) {
   cudaStream_t s = ctx->stream;
-  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)ctx->P * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)ctx->nb * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
   CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
   int free_top = 0;
   CK(cudaMemcpyAsync(&free_top, ctx->d_small, sizeof(int), cudaMemcpyDeviceToHost, s));
@@ -31,7 +31,7 @@ lt_status read_counts(lt_ctx* ctx) {
   return LT_OK;
 }
 
-inline uint64_t pending(const lt_ctx* ctx, uint32_t k) { return ctx->h_hc[ctx->P + k] - ctx->h_hc[k]; }
+inline uint64_t pending(const lt_ctx* ctx, uint32_t k) { return ctx->h_hc[ctx->nb + k] - ctx->h_hc[k]; }
 
 // cudaEventQuery without leaving cudaErrorNotReady behind for the next launch check
 bool event_done(cudaEvent_t e) {
@@ -66,17 +66,16 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
 }
 
 lt_status run_resident(lt_ctx* ctx) {
-  const uint32_t P = ctx->P;
   const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
   std::vector<uint32_t> order;
-  order.reserve(P);
+  order.reserve(ctx->P);
   for (;;) {
     lt_status st = read_counts(ctx);  // one small D2H + sync per sweep
     if (st != LT_OK) return st;
     if (ctx->h_ctr->err) return LT_OK;
     order.clear();
     uint64_t total = 0;
-    for (uint32_t k = 0; k < P; ++k)
+    for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k)  // owned partitions (all when world == 1)
       if (pending(ctx, k)) { order.push_back(k); total += pending(ctx, k); }
     if (total == 0) return LT_OK;
     // every live walk advances >= 1 step per sweep, so sweeps <= max_len + 1
@@ -169,22 +168,23 @@ lt_status run_out_of_core(lt_ctx* ctx) {
   // each iteration consumes >= 1 visit and a walk makes <= max_len + 1 visits
   const uint64_t max_iters = ctx->W * (max_len + 1) + P + 64;
   uint64_t seq = 0;
-  uint32_t rr = P - 1;  // round-robin cursor
+  const uint32_t lo = ctx->own_lo, hi = ctx->own_hi;  // owned partitions (all when world == 1)
+  uint32_t rr = hi - 1;  // round-robin cursor
   for (;;) {
     lt_status st = read_counts(ctx);  // Alg. 2 line 1: while active walks exist
     if (st != LT_OK) return st;
     if (ctx->h_ctr->err) return LT_OK;
     uint64_t total = 0;
-    for (uint32_t k = 0; k < P; ++k) total += pending(ctx, k);
+    for (uint32_t k = lo; k < hi; ++k) total += pending(ctx, k);
     if (total == 0) return LT_OK;
     if (ctx->stats.iterations > max_iters) return fail(LT_ERR_CUDA, "out-of-core scheduler did not converge");
     // scheduler.iteration(): select partition i
-    uint32_t i = 0;
+    uint32_t i = lo;
     if (selective) {
-      for (uint32_t k = 1; k < P; ++k)
+      for (uint32_t k = lo + 1; k < hi; ++k)
         if (pending(ctx, k) > pending(ctx, i)) i = k;
     } else {
-      do { rr = (rr + 1) % P; } while (!pending(ctx, rr));
+      do { rr = (rr + 1 >= hi) ? lo : rr + 1; } while (!pending(ctx, rr));
       i = rr;
     }
     ctx->stats.iterations++;

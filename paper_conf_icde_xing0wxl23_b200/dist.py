@@ -1,0 +1,149 @@
+"""Multi-GPU range-ownership mode (the north star's 8-GPU mode, not in
+the paper): the superstep exchange around the C ABI.
+
+Rank r owns a contiguous range of partitions (lt_config.rank/world). Each superstep:
+  1. lt_run            advance every walk in the owned buckets until it ends or leaves the range
+                       (walks for rank q collect in send bucket q);
+  2. lt_exchange_pack  move the send buckets into one device buffer, grouped by destination;
+  3. all-to-all        of the per-rank counts, then of the 16-B walk records (NCCL over NVLink via
+                       torch.distributed; gloo on CPU in the tests);
+  4. lt_exchange_insert the received walks into the owned buckets (warp-aggregated insertion);
+until no walk crossed ranks in a superstep (every live walk is then in some owned bucket, and lt_run
+ended them all). Paths are merged once at the end: element-wise unsigned min of the path rows
+(unwritten entries are 0xFFFFFFFF) and max of the lengths.
+
+The exchange is the only data-path collective; this module only sequences ABI calls and
+collectives (plumbing), every walk step runs in the CUDA kernels behind the ABI.
+"""
+from __future__ import annotations
+
+import threading
+
+SIGN = -0x80000000  # int32 with only the sign bit: x ^ SIGN maps unsigned order onto signed order
+
+
+class TorchComm:
+    """Collectives over a torch.distributed process group (NCCL for CUDA tensors, gloo for CPU)."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+
+    def alltoall_counts(self, counts, device):
+        import torch
+        t = torch.tensor(counts, dtype=torch.int64, device=device)
+        out = torch.empty_like(t)
+        self.dist.all_to_all_single(out, t, group=self.group)
+        return [int(x) for x in out.tolist()]
+
+    def alltoallv(self, send, send_counts, recv_counts):
+        """send: int32 [sum(send_counts), 4]; returns int32 [sum(recv_counts), 4]."""
+        import torch
+        recv = torch.empty((sum(recv_counts), 4), dtype=torch.int32, device=send.device)
+        self.dist.all_to_all_single(recv.view(-1), send[: sum(send_counts)].reshape(-1).contiguous(),
+                                    output_split_sizes=[4 * c for c in recv_counts],
+                                    input_split_sizes=[4 * c for c in send_counts], group=self.group)
+        return recv
+
+    def allreduce_sum(self, x: int, device) -> int:
+        import torch
+        t = torch.tensor([x], dtype=torch.int64, device=device)
+        self.dist.all_reduce(t, group=self.group)
+        return int(t.item())
+
+    def allreduce_(self, t, op: str):
+        self.dist.all_reduce(t, op={"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX}[op], group=self.group)
+
+
+class ThreadComm:
+    """In-process collectives between `world` threads (each driving one Engine), used to exercise
+    the ownership mode with several engines on one GPU. Create one shared ThreadComm.Hub and a
+    ThreadComm(hub, rank) per thread."""
+
+    class Hub:
+        def __init__(self, world):
+            self.world = world
+            self.barrier = threading.Barrier(world)
+            self.slots = [None] * world
+
+    def __init__(self, hub, rank):
+        self.hub, self.rank, self.world = hub, rank, hub.world
+
+    def _gather(self, x):
+        self.hub.barrier.wait()
+        self.hub.slots[self.rank] = x
+        self.hub.barrier.wait()
+        allv = list(self.hub.slots)
+        self.hub.barrier.wait()
+        return allv
+
+    def alltoall_counts(self, counts, device):
+        allc = self._gather(list(counts))
+        return [allc[r][self.rank] for r in range(self.world)]
+
+    def alltoallv(self, send, send_counts, recv_counts):
+        import torch
+        offs = [0]
+        for c in send_counts:
+            offs.append(offs[-1] + c)
+        allv = self._gather((send, offs))
+        parts = [allv[r][0][allv[r][1][self.rank]: allv[r][1][self.rank + 1]] for r in range(self.world)]
+        parts = [p.to(send.device) for p in parts]
+        return torch.cat(parts) if parts else send[:0]
+
+    def allreduce_sum(self, x: int, device) -> int:
+        return sum(self._gather(int(x)))
+
+    def allreduce_(self, t, op: str):
+        allv = self._gather(t.clone())
+        acc = allv[0].to(t.device)
+        for o in allv[1:]:
+            o = o.to(t.device)
+            acc = (acc.minimum(o) if op == "min" else acc.maximum(o))
+        t.copy_(acc)
+
+
+def send_buffer(engine, device, cache: dict):
+    """A device buffer large enough for every walk this rank holds in its send buckets."""
+    import torch
+    _, out = engine.pending()
+    need = max(sum(out), 1)
+    buf = cache.get("send")
+    if buf is None or buf.shape[0] < need:
+        buf = torch.empty((max(need, 2 * (0 if buf is None else buf.shape[0])), 4), dtype=torch.int32, device=device)
+        cache["send"] = buf
+    return buf
+
+
+def run_supersteps(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
+    """Drive lt_run + exchange until no walk is alive on any rank. Returns counters."""
+    cache: dict = {}
+    supersteps, moved = 0, 0
+    while True:
+        engine.run()
+        buf = send_buffer(engine, device, cache)
+        counts = engine.exchange_pack(buf)
+        recv_counts = comm.alltoall_counts(counts, device)
+        recv = comm.alltoallv(buf, counts, recv_counts)
+        engine.exchange_insert(recv, sum(recv_counts))
+        crossed = comm.allreduce_sum(sum(recv_counts), device)
+        supersteps += 1
+        moved += sum(counts)
+        if crossed == 0:
+            return {"supersteps": supersteps, "records_sent": moved}
+        if supersteps >= max_supersteps:
+            raise RuntimeError("ownership supersteps did not converge")
+
+
+def merge_paths(engine, comm):
+    """Cross-rank merge of the partial path matrices: unsigned min of entries, max of lengths.
+    Returns CUDA/CPU int32 tensors (paths [W, stride], lengths [W]) identical on every rank."""
+    paths, lengths = engine.partial_paths()
+    paths ^= SIGN
+    comm.allreduce_(paths, "min")
+    paths ^= SIGN
+    comm.allreduce_(lengths, "max")
+    return paths, lengths

@@ -32,6 +32,7 @@ EXPORTED = [
     "lt_config_default", "lt_create", "lt_destroy", "lt_last_error", "lt_partition_bounds", "lt_graph_load",
     "lt_graph_load_device", "lt_get_bounds", "lt_walks_init", "lt_walks_init_ex", "lt_run", "lt_path_stride",
     "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
+    "lt_pending", "lt_exchange_pack", "lt_exchange_insert",
 ]
 
 
@@ -55,7 +56,9 @@ class Config(ctypes.Structure):
         ("zc_alpha_bytes", ctypes.c_uint32),
         ("pad0", ctypes.c_uint32),
         ("graph_pool_bytes", ctypes.c_uint64),
-        ("reserved", ctypes.c_uint32 * 4),
+        ("rank", ctypes.c_uint32),
+        ("world", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 2),
     ]
 
 
@@ -96,6 +99,9 @@ _lib.lt_get_paths_rows.argtypes = [_vp, _vp, _u64, _vp, _vp]
 _lib.lt_get_paths_device.argtypes = [_vp, _vp, _vp]
 _lib.lt_get_stats.argtypes = [_vp, ctypes.POINTER(Stats)]
 _lib.lt_get_pool_state.argtypes = [_vp, ctypes.POINTER(PoolState)]
+_lib.lt_pending.argtypes = [_vp, ctypes.POINTER(_u64), _vp]
+_lib.lt_exchange_pack.argtypes = [_vp, _vp, _u64, _vp]
+_lib.lt_exchange_insert.argtypes = [_vp, _vp, _u64]
 
 
 class LTError(RuntimeError):
@@ -150,7 +156,7 @@ class Engine:
                  timing: bool = False, stream=None, blocks_per_sm: int = 0, l2_fetch_bytes: int = 0,
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
-                 zc_alpha_bytes: int = 0):
+                 zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -169,6 +175,9 @@ class Engine:
         cfg.graph_pool_bytes = graph_pool_bytes
         cfg.zero_copy = int(bool(zero_copy))
         cfg.zc_alpha_bytes = zc_alpha_bytes
+        cfg.rank = rank
+        cfg.world = world
+        self.rank, self.world, self.device = rank, world, device
         h = _vp()
         _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))
         self._h = h
@@ -259,6 +268,41 @@ class Engine:
         if (d_paths is not None and not dp) or (d_lengths is not None and not dl):
             raise ValueError("get_paths_device needs CUDA tensors")
         _check(_lib.lt_get_paths_device(self._h, pp, pl))
+
+    # ---- range ownership across ranks (include/lt.h "Range ownership"; driven by dist.py)
+    def pending(self):
+        """(walks in owned buckets, [walks in the send bucket of each rank])"""
+        loc = _u64()
+        out = np.zeros(self.world, dtype=np.uint64)
+        _check(_lib.lt_pending(self._h, ctypes.byref(loc), out.ctypes.data))
+        return int(loc.value), [int(x) for x in out]
+
+    def exchange_pack(self, d_send):
+        """Move every send bucket into the CUDA int32 tensor d_send [capacity, 4] (16-B records grouped
+        by destination rank); returns the per-rank record counts."""
+        pp, dev, keep = _ptr(d_send, np.uint32)
+        if d_send is not None and not dev:
+            raise ValueError("exchange_pack needs a CUDA tensor")
+        cap = keep.numel() // 4 if keep is not None else 0
+        counts = np.zeros(self.world, dtype=np.uint64)
+        _check(_lib.lt_exchange_pack(self._h, pp, cap, counts.ctypes.data))
+        return [int(x) for x in counts]
+
+    def exchange_insert(self, d_recv, count: int):
+        pp, dev, _ = _ptr(d_recv, np.uint32)
+        if d_recv is not None and count and not dev:
+            raise ValueError("exchange_insert needs a CUDA tensor")
+        _check(_lib.lt_exchange_insert(self._h, pp, count))
+
+    def partial_paths(self):
+        """This rank's share of paths (CUDA int32 tensors [W, stride], [W]) for the cross-rank merge."""
+        import torch
+        W, S = self.num_walks, self.stride()
+        paths = torch.empty((W, S), dtype=torch.int32, device=f"cuda:{self.device}")
+        lengths = torch.empty(W, dtype=torch.int32, device=f"cuda:{self.device}")
+        if W:
+            self.get_paths_device(paths, lengths)
+        return paths, lengths
 
     def pool_state(self) -> dict:
         s = PoolState()

@@ -1,0 +1,111 @@
+"""Test-only CPU stand-in for one rank of the range-ownership mode (include/lt.h "Range ownership").
+
+It implements the Engine methods dist.run_supersteps / dist.merge_paths call (run, pending,
+exchange_pack, exchange_insert, partial_paths) with per-visit stepping built on the ORACLE's
+primitives (Philox and Lemire from oracle/), so the multi-process protocol (ownership ranges,
+send buckets, count + payload all-to-all, termination, min/max merge) can run on CPU under gloo.
+It is not the product: the product's kernels are exercised by tests/test_gpu_ownership.py.
+"""
+import numpy as np
+
+import oracle as O
+import paper_conf_icde_xing0wxl23_b200 as LT
+
+EMPTY = 0xFFFFFFFF
+
+
+class CpuOwnerEngine:
+    def __init__(self, g, P, rank, world):
+        self.g, self.P, self.rank, self.world = g, P, rank, world
+        self.bounds = LT.partition_bounds(g.row_ptr, P)
+        self.own_lo = P * rank // world
+        self.own_hi = P * (rank + 1) // world
+        self.owner = np.zeros(P, dtype=np.int64)
+        for r in range(world):
+            self.owner[P * r // world: P * (r + 1) // world] = r
+
+    def _part(self, v):
+        return int(np.searchsorted(self.bounds, v, side="right") - 1)
+
+    def _bucket(self, q):
+        return q if self.own_lo <= q < self.own_hi else self.P + int(self.owner[q])
+
+    def walks_init(self, starts, app, param, seed, lmax=127):
+        W = len(starts)
+        self.app, self.param, self.seed, self.lmax = app, param, seed, lmax
+        self.T = O.ppr_threshold(param) if app == LT.PPR else 0
+        self.stride = int(param) + 1 if app == LT.DEEPWALK else lmax + 1
+        self.num_walks = W
+        self.paths = np.full((W, self.stride), EMPTY, dtype=np.uint32)
+        self.lengths = np.zeros(W, dtype=np.uint32)
+        self.buckets = {b: [] for b in range(self.P + self.world)}
+        for w in range(W):
+            q = self._part(int(starts[w]))
+            if self.own_lo <= q < self.own_hi:
+                self.paths[w, 0] = starts[w]
+                self.buckets[q].append((w, int(starts[w]), 0))
+
+    def _visit(self, rec, lo, hi):
+        w, v, t = rec
+        rp, col = self.g.row_ptr, self.g.col
+        while True:
+            if self.app == LT.DEEPWALK and t == int(self.param):
+                break
+            if self.app == LT.PPR and t == self.lmax:
+                break
+            if self.app == LT.PPR:
+                x0 = O.philox4x32_10([t, 0, w & 0xFFFFFFFF, w >> 32], [self.seed & 0xFFFFFFFF, self.seed >> 32])[0]
+                if x0 < self.T:
+                    break
+            d = int(rp[v + 1] - rp[v])
+            if d == 0:
+                break
+            idx, _ = O.lemire(self.seed, w, t, d)
+            v = int(col[int(rp[v]) + idx])
+            t += 1
+            self.paths[w, t] = v
+            if not (lo <= v < hi):
+                return (w, v, t)
+        self.lengths[w] = t + 1
+        return None
+
+    def run(self):
+        while True:
+            ks = [k for k in range(self.own_lo, self.own_hi) if self.buckets[k]]
+            if not ks:
+                return
+            for k in ks:
+                lo, hi = int(self.bounds[k]), int(self.bounds[k + 1])
+                recs, self.buckets[k] = self.buckets[k], []
+                for rec in recs:
+                    out = self._visit(rec, lo, hi)
+                    if out is not None:
+                        self.buckets[self._bucket(self._part(out[1]))].append(out)
+
+    def pending(self):
+        loc = sum(len(self.buckets[k]) for k in range(self.own_lo, self.own_hi))
+        return loc, [len(self.buckets[self.P + r]) if self.world > 1 else 0 for r in range(self.world)]
+
+    def exchange_pack(self, buf):
+        counts, off = [], 0
+        for r in range(self.world):
+            recs = self.buckets[self.P + r]
+            self.buckets[self.P + r] = []
+            for i, (w, v, t) in enumerate(recs):
+                buf[off + i, 0] = w
+                buf[off + i, 1] = int(np.uint32(v).view(np.int32))
+                buf[off + i, 2] = t
+                buf[off + i, 3] = 0
+            counts.append(len(recs))
+            off += len(recs)
+        return counts
+
+    def exchange_insert(self, recv, count):
+        arr = recv[:count].numpy().view(np.uint32)
+        for w, v, t, _ in arr:
+            self.buckets[self._bucket(self._part(int(v)))].append((int(w), int(v), int(t)))
+
+    def partial_paths(self):
+        import torch
+        return (torch.from_numpy(self.paths.view(np.int32).copy()),
+                torch.from_numpy(self.lengths.view(np.int32).copy()))
