@@ -65,12 +65,17 @@ def parse():
     ap.add_argument("--layout", type=int, default=0, help="0 auto, 1 CSR, 2 ADJ (lt_layout)")
     ap.add_argument("--ilp", type=int, default=0)
     ap.add_argument("--path-mode", type=int, default=0)
+    ap.add_argument("--refill", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", default="", help="comma list of P values to time (extra key)")
     ap.add_argument("--graph-pool-gb", type=float, default=0.0,
                     help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
     ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
+    ap.add_argument("--mode", default="replicas", choices=["replicas", "own"],
+                    help="N>1: replicas (each rank its own |V| walks, no collective, weak scaling) or own "
+                         "(range ownership: |V| walks in total, NCCL all-to-all of crossing walks per "
+                         "superstep, strong scaling)")
     return ap.parse_args()
 
 
@@ -262,7 +267,10 @@ def main():
     g = make_graph(c, local)
     gen_s = time.time() - t0
     W = num_walks(c, g)
-    first = rank * W
+    own = args.mode == "own" and world > 1
+    if own and args.partitions is None:
+        P = c["partitions"] = world  # one contiguous partition per rank: fewest crossings
+    first = 0 if own else rank * W
     app, param = app_param(c)
     starts_h = starts_for(c, g, W, first)
     starts_d = torch.from_numpy(starts_h.view(np.int32)).cuda(local)
@@ -270,7 +278,8 @@ def main():
     ooc = args.graph_pool_gb > 0
     eng = LT.Engine(device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
-                    graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy))
+                    graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
+                    rank=rank if own else 0, world=world if own else 1, refill=args.refill)
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
@@ -281,9 +290,18 @@ def main():
             dist.barrier()
             torch.cuda.synchronize()
 
+    comm = None
+    if own:
+        from paper_conf_icde_xing0wxl23_b200 import dist as ltdist
+        comm = ltdist.TorchComm()
+    superstep_counters = {}
+
     def one_step():
         eng.walks_init(starts_d, app, param, args.seed, first)
-        eng.run()
+        if own:
+            superstep_counters.update(ltdist.run_supersteps(eng, comm, f"cuda:{local}"))
+        else:
+            eng.run()
         return eng.stats()
 
     for _ in range(args.warmup):
@@ -315,7 +333,8 @@ def main():
     upd_launches = sum(s["update_launches"] for s in stats)
     visits = sum(s["visits"] for s in stats)
     steps_k = steps_local
-    moves = visits - len(stats) * W  # each walk's final visit ends in termination, every other visit in a move
+    finished = sum(s["num_walks"] for s in stats) if not own else len(stats) * W // world
+    moves = max(0, visits - finished)  # a walk's final visit ends in termination, every other in a move
     alg_bytes = steps_k * 104 + visits * 16 + moves * 16
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
@@ -349,8 +368,9 @@ def main():
 
     # ---- extra partition-count sweep (context; the headline uses P above)
     sweep = {}
-    for ps in [int(x) for x in args.sweep.split(",") if x.strip()]:
-        with LT.Engine(device=local, chunk_walks=args.chunk_walks, timing=True, layout=args.layout) as e2:
+    for ps in ([int(x) for x in args.sweep.split(",") if x.strip()] if not own else []):
+        with LT.Engine(device=local, chunk_walks=args.chunk_walks, timing=True, layout=args.layout,
+                       refill=args.refill) as e2:
             e2.graph_load(g.row_ptr, g.col, ps)
             for _ in range(2):
                 e2.walks_init(starts_d, app, param, args.seed, first)
@@ -397,7 +417,7 @@ def main():
                      "hit_rate": last["pool_hits"] / max(1, last["iterations"])}
 
     e2e = None
-    if not args.no_e2e and args.e2e_steps > 0:
+    if not args.no_e2e and args.e2e_steps > 0 and not own:
         S = int(c["length"]) + 1 if c["app"] == "deepwalk" else 128
         try:
             h_paths = torch.empty((W, S), dtype=torch.int32, pin_memory=True)
@@ -452,11 +472,11 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "steps/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "scaling": "strong" if own else "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
                 "config": cfg_json(c, g, W, {"partitions": P, "chunk_walks": args.chunk_walks,
                                              "policy": "selective" if args.policy == 0 else "round_robin",
                                              "insert_mode": "warp_aggregated" if args.insert_mode == 0 else "direct",
-                                             "parallelism": f"replicas{world}" if world > 1 else "single",
+                                             "parallelism": (f"own{world}" if own else f"replicas{world}") if world > 1 else "single",
                                              "mode": "out_of_core" if ooc else "hbm_resident",
                                              "graph_pool_gb": args.graph_pool_gb if ooc else None,
                                              "l2": "inputs larger than L2 (CSR >> 126 MB); no flush",
@@ -471,6 +491,8 @@ def main():
                              "chunks_total": last["chunks_total"], "chunks_free_min": last["chunks_free_min"]}}
         if host_link:
             line["host_link"] = host_link
+        if own:
+            line["ownership"] = dict(superstep_counters)
         if sweep:
             line["partition_sweep"] = sweep
         print(json.dumps(line), flush=True)

@@ -55,6 +55,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.world == 0) c.world = 1;
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
+  if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -200,7 +201,7 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     CK(cudaMemcpy(ctx->d_owner, own.data(), P * sizeof(uint16_t), cudaMemcpyHostToDevice));
   }
   const size_t nb = ctx->nb;
-  CK(ensure(ctx->d_hc, ctx->hc_cap, 2 * nb));
+  CK(ensure(ctx->d_hc, ctx->hc_cap, 3 * nb));  // head, cursor, refill claim
   if (ctx->h_hc_cap < 2 * nb) {
     if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
     ctx->h_hc = nullptr;
@@ -442,6 +443,7 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.pool.nbuckets = ctx->nb;
   p.pool.head = ctx->d_hc;
   p.pool.cursor = ctx->d_hc + ctx->nb;
+  p.pool.claim = ctx->d_hc + 2 * (size_t)ctx->nb;
   p.own.own_lo = ctx->own_lo;
   p.own.own_hi = ctx->own_hi;
   p.own.owner = ctx->d_owner;
@@ -452,6 +454,10 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.gather_mode = ctx->cfg.gather_mode;
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
   p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : (ctx->d_adj ? 1u : 2u);
+  // lane refill (k_update_rf) pays off when walks end at different steps inside a launch: several
+  // partitions (visits end at the partition edge) or PPR (geometric lengths)
+  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && (ctx->P > 1 || app == LT_APP_PPR)) ? 1u : 0u;
+  if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp);
 
   ctx->W = W;

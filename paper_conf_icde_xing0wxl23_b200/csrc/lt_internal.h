@@ -27,6 +27,7 @@ struct Pool {
   uint32_t nbuckets;              // P partition buckets + one send bucket per other rank
   unsigned long long* head;       // [nbuckets]
   unsigned long long* cursor;     // [nbuckets]
+  unsigned long long* claim;      // [nbuckets] refill claims within a launch (== head between launches)
   uint32_t* free_list;            // [num_chunks]
   int* free_top;
 };
@@ -74,6 +75,7 @@ struct Params {
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;
+  uint32_t refill;  // 1: lane-refill update kernel (k_update_rf)
 };
 
 // launchers (lt_kernels.cu); all asynchronous on `s`

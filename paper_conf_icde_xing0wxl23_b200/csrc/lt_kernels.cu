@@ -172,6 +172,7 @@ __device__ void last_cta_retire(const Params& p, int k, unsigned long long head,
   if (threadIdx.x == 0) {
     if (k >= 0) {
       pl.head[k] = tail;
+      pl.claim[k] = tail;  // refill claims may have run past the snapshot
       atomicAdd(&p.ctr->visits, tail - head);
     }
     *(volatile uint32_t*)&p.ctr->done_ctas = 0;
@@ -475,6 +476,158 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
   last_cta_retire(p, (int)k, head, tail);
 }
 
+// ------------------------------------------------------------------- a3 + a4 + a5, lane refill
+// Same step, gathers and insertion as k_update, but a lane whose walk ended (terminated or left the
+// partition) takes the next record of the bucket at once instead of idling until the warp's
+// longest walk is done. Walk lengths inside a partition are geometric when P > 1 and for PPR, so
+// without refill most lanes of a warp idle most of the time. A warp claims kRefill positions of the
+// bucket at a time (one atomic per kRefill walks) and hands them to its idle lanes.
+constexpr uint32_t kRefill = 64;
+
+template <int APP, int GM, int LAY>
+__global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
+  extern __shared__ uint32_t s_bounds[];
+  const Walk& wk = p.wk;
+  const Pool& pl = p.pool;
+  const uint32_t* B = stage_bounds(wk, s_bounds);
+  const unsigned long long head = pl.head[k];
+  const unsigned long long tail = pl.cursor[k];
+  const uint32_t lo = wk.bounds[k];
+  const uint32_t span = wk.bounds[k + 1] - lo;
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
+  unsigned long long* claim = pl.claim + k;
+  const Policies pol = make_policies();
+  unsigned long long my_steps = 0, my_trunc = 0;
+
+  bool has = false;
+  uint4 rec = make_uint4(0, 0, 0, 0);  // .x = row, .y = v, .z = t
+  uint32_t* prow = wk.paths;
+  uint32_t pb[8];
+  uint32_t nb = 0;
+  unsigned long long off = 0;
+  uint32_t d = 0;
+  unsigned long long q_cur = 0, q_end = 0;  // this warp's claimed, not yet handed out positions
+  bool drained = false;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) pb[q] = 0;
+
+  for (;;) {
+    // ---- refill idle lanes from the warp's claimed range (claim kRefill more when it runs out)
+    uint32_t need = __ballot_sync(kFull, !has);
+    while (need && !drained) {
+      if (q_cur >= q_end) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(claim, (unsigned long long)kRefill);
+        base = __shfl_sync(kFull, base, 0);
+        q_cur = base;
+        q_end = (base + kRefill < tail) ? base + kRefill : tail;
+        if (q_cur >= tail) { drained = true; break; }
+      }
+      const uint32_t avail = (q_end - q_cur < 32ull) ? (uint32_t)(q_end - q_cur) : 32u;
+      const uint32_t r = __popc(need & lanemask_lt());
+      if (!has && r < avail) {
+        const unsigned long long pos = q_cur + r;
+        const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
+        rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
+        has = true;
+        prow = wk.paths + (uint64_t)rec.x * wk.pitch;
+        pb[7] = rec.y;
+        nb = ((rec.z & 7u) == 0) ? 1u : 0u;
+        if (LAY == 1) {
+          off = __ldg(wk.row_ptr + rec.y);
+          d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
+        }
+      }
+      q_cur += (avail < (uint32_t)__popc(need)) ? avail : (uint32_t)__popc(need);
+      need = __ballot_sync(kFull, !has);
+    }
+    if (!__any_sync(kFull, has)) break;
+    // ---- one step of every lane that holds a walk
+    bool done = false, left = false, trunc = false;
+    if (has) {
+      if (APP == 0 && rec.z == wk.length) {
+        done = true;
+      } else if (APP == 1 && rec.z == wk.lmax) {
+        done = true;
+        trunc = true;
+      } else {
+        if (LAY == 0) {
+          const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
+          off = __ldg(rp) - wk.ebase;
+          d = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
+        }
+        const uint64_t wid = wk.first_walk_id + rec.x;
+        const uint4 b = philox10(make_uint4(rec.z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
+        if ((APP == 1 && b.x < wk.T) || d == 0) {
+          done = true;
+        } else {
+          const uint64_t m = (uint64_t)b.y * d;
+          const uint32_t idx = ((uint32_t)m < d) ? lemire_slow(d, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
+                                                              wk.seed_lo, wk.seed_hi)
+                                                 : (uint32_t)(m >> 32);
+          uint32_t nv;
+          if (LAY == 0) {
+            nv = ld_col<GM>(wk.col + off + idx, pol);
+          } else {
+            const uint4 e = ld_adj<GM>(wk.adj + off + idx, pol);
+            nv = e.x;
+            d = e.y;
+            off = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+          }
+          rec.y = nv;
+          rec.z += 1;
+          const uint32_t t = rec.z;
+          if (wk.path_mode == 0) {
+#pragma unroll
+            for (int q = 0; q < 7; ++q) pb[q] = pb[q + 1];
+            pb[7] = nv;
+            nb += 1;
+            if ((t & 7u) == 7u) {
+              if (nb == 8) {
+                uint4* dst = reinterpret_cast<uint4*>(prow + (t - 7));
+                dst[0] = make_uint4(pb[0], pb[1], pb[2], pb[3]);
+                dst[1] = make_uint4(pb[4], pb[5], pb[6], pb[7]);
+              } else {
+#pragma unroll
+                for (int q = 0; q < 8; ++q)
+                  if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
+              }
+              nb = 0;
+            }
+          } else if (wk.path_mode == 1) {
+            prow[t] = nv;
+          }
+          left = (nv - lo >= span);
+        }
+      }
+    }
+    // ---- retire the walks that ended this step
+    const bool ended = done || left;
+    if (ended && wk.path_mode == 0) {
+      const uint32_t t = rec.z;
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
+      nb = 0;
+    }
+    if (done) {
+      wk.lengths[rec.x] = rec.z + 1;
+      my_steps += rec.z;
+      my_trunc += trunc ? 1 : 0;
+    }
+    uint32_t dest = 0;
+    if (left) dest = bucket_of(p, find_partition(B, wk.P, rec.y));
+    insert_warp(p, left, dest, rec);
+    if (ended) has = false;
+  }
+  my_steps = warp_sum(my_steps);
+  my_trunc = warp_sum(my_trunc);
+  if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
+  if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
+  last_cta_retire(p, (int)k, head, tail);
+}
+
 // ---------------------------------------------------------------------------- output helpers
 __global__ void k_finalize(Params p, uint64_t W) {
   const Walk& wk = p.wk;
@@ -518,7 +671,7 @@ __global__ void k_pool_reset(Params p) {
   for (uint64_t i = tid; i < pl.num_chunks; i += stride) pl.free_list[i] = (uint32_t)i;
   const uint64_t nring = (uint64_t)pl.nbuckets * pl.ring_len;
   for (uint64_t i = tid; i < nring; i += stride) pl.ring[i] = kEmpty;
-  for (uint64_t i = tid; i < pl.nbuckets; i += stride) { pl.head[i] = 0; pl.cursor[i] = 0; }
+  for (uint64_t i = tid; i < pl.nbuckets; i += stride) { pl.head[i] = 0; pl.cursor[i] = 0; pl.claim[i] = 0; }
   if (tid == 0) {
     *pl.free_top = (int)pl.num_chunks;
     p.ctr->steps = 0; p.ctr->visits = 0; p.ctr->truncated = 0; p.ctr->err = 0; p.ctr->done_ctas = 0;
@@ -607,7 +760,21 @@ void launch_update_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block,
 }
 
 template <int APP, int GM, int LAY>
+void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(k_update_rf<APP, GM, LAY>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
+    attr = true;
+  }
+  k_update_rf<APP, GM, LAY><<<grid, block, bounds_smem(p), s>>>(p, k);
+}
+
+template <int APP, int GM, int LAY>
 void launch_update_ilp(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  if (p.refill) {
+    launch_update_rf<APP, GM, LAY>(p, k, grid, block, s);
+    return;
+  }
   switch (p.ilp) {
     case 1: launch_update_t<APP, GM, 1, LAY>(p, k, grid, block, s); break;
     case 4: launch_update_t<APP, GM, 4, LAY>(p, k, grid, block, s); break;

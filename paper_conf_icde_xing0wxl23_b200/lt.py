@@ -58,7 +58,8 @@ class Config(ctypes.Structure):
         ("graph_pool_bytes", ctypes.c_uint64),
         ("rank", ctypes.c_uint32),
         ("world", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 2),
+        ("refill", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 1),
     ]
 
 
@@ -156,7 +157,7 @@ class Engine:
                  timing: bool = False, stream=None, blocks_per_sm: int = 0, l2_fetch_bytes: int = 0,
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
-                 zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1):
+                 zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -177,6 +178,7 @@ class Engine:
         cfg.zc_alpha_bytes = zc_alpha_bytes
         cfg.rank = rank
         cfg.world = world
+        cfg.refill = refill
         self.rank, self.world, self.device = rank, world, device
         h = _vp()
         _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))

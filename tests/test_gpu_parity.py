@@ -226,13 +226,13 @@ def test_pool_invariants(gpu, cfg1, P, chunk):
 
 
 @pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
-@pytest.mark.parametrize("ilp", [1, 2, 4])
+@pytest.mark.parametrize("ilp,refill", [(1, 1), (2, 1), (4, 1), (1, 2)])
 @pytest.mark.parametrize("gather_mode", [0, 3])
 @pytest.mark.parametrize("P", [1, 8])
-def test_kernel_variants_exact(gpu, cfg1, layout, ilp, gather_mode, P):
-    """Layout (CSR vs augmented adjacency), walks per lane and cache hints change only how the
-    gathers are issued, never which neighbour is chosen."""
-    kw = dict(layout=layout, ilp=ilp, gather_mode=gather_mode, chunk_walks=256)
+def test_kernel_variants_exact(gpu, cfg1, layout, ilp, refill, gather_mode, P):
+    """Layout (CSR vs augmented adjacency), walks per lane, lane refill and cache hints change only
+    how the gathers are issued, never which neighbour is chosen."""
+    kw = dict(layout=layout, ilp=ilp, gather_mode=gather_mode, chunk_walks=256, refill=refill)
     assert_parity(cfg1, lt_inputs.deepwalk_starts(3000, cfg1.n), LT.DEEPWALK, 12, 7, P=P, **kw)
     assert_parity(cfg1, lt_inputs.ppr_starts(3000, cfg1.argmax_deg), LT.PPR, 0.2, 7, P=P, **kw)
     g = lt_inputs.small_graph([(0, 1), (1, 3), (3, 4)], n=6)
@@ -242,10 +242,12 @@ def test_kernel_variants_exact(gpu, cfg1, layout, ilp, gather_mode, P):
 @pytest.mark.parametrize("path_mode", [0, 1])
 @pytest.mark.parametrize("P", [1, 3, 16])
 @pytest.mark.parametrize("length", [0, 1, 7, 8, 9, 15, 16, 17, 80])
-def test_path_store_modes_and_sector_edges(gpu, cfg1, path_mode, P, length):
+@pytest.mark.parametrize("refill", [1, 2])
+def test_path_store_modes_and_sector_edges(gpu, cfg1, path_mode, P, length, refill):
     """Buffered full-sector path stores vs one store per step, at lengths around the 8-entry sector
-    boundaries, with visits that start mid-sector (P > 1)."""
-    assert_parity(cfg1, lt_inputs.deepwalk_starts(1500, cfg1.n), LT.DEEPWALK, length, 3, P=P, path_mode=path_mode)
+    boundaries, with visits that start mid-sector (P > 1), with and without lane refill."""
+    assert_parity(cfg1, lt_inputs.deepwalk_starts(1500, cfg1.n), LT.DEEPWALK, length, 3, P=P, path_mode=path_mode,
+                  refill=refill)
 
 
 def test_path_mode_off_keeps_lengths(gpu, cfg1):

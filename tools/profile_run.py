@@ -29,6 +29,7 @@ def main():
     ap.add_argument("--blocks-per-sm", type=int, default=0)
     ap.add_argument("--layout", type=int, default=0)
     ap.add_argument("--path-mode", type=int, default=0)
+    ap.add_argument("--refill", type=int, default=0)
     a = ap.parse_args()
     import torch
 
@@ -48,7 +49,8 @@ def main():
     sd = torch.from_numpy(st.view(np.int32)).cuda()
     with LT.Engine(chunk_walks=a.chunk_walks, l2_fetch_bytes=a.l2_fetch, timing=True,
                    gather_mode=a.gather_mode, ilp=a.ilp, blocks_per_sm=a.blocks_per_sm,
-                   layout=a.layout, path_mode=a.path_mode) as e:
+                   layout=a.layout, path_mode=a.path_mode,
+                   refill=a.refill) as e:
         e.graph_load(g.row_ptr, g.col, a.partitions)
         for _ in range(a.steps):
             e.walks_init(sd, app, prm, 1)
