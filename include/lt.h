@@ -107,8 +107,8 @@ typedef struct lt_config {
                                  partitions. Every partition must fit one block
                                  (block = the largest partition's CSR slice). */
   uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
-  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P > 1 or PPR),
-                                 1 off, 2 on */
+  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P == 1, the measured
+                                 best), 1 off, 2 on */
   uint32_t reserved[1];
 } lt_config;
 

@@ -454,9 +454,9 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.gather_mode = ctx->cfg.gather_mode;
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
   p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : (ctx->d_adj ? 1u : 2u);
-  // lane refill (k_update_rf) pays off when walks end at different steps inside a launch: several
-  // partitions (visits end at the partition edge) or PPR (geometric lengths)
-  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && (ctx->P > 1 || app == LT_APP_PPR)) ? 1u : 0u;
+  // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
+  // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
+  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
   if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp);
 

@@ -484,6 +484,16 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
 // bucket at a time (one atomic per kRefill walks) and hands them to its idle lanes.
 constexpr uint32_t kRefill = 64;
 
+// Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
+__device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
+  const uint32_t lane = threadIdx.x & 31u;
+  for (uint32_t r = 0; r < cnt; r += 32) {
+    const bool act = r + lane < cnt;
+    insert_warp(p, act, act ? qd[r + lane] : 0u, act ? qr[r + lane] : make_uint4(0, 0, 0, 0));
+  }
+  __syncwarp();
+}
+
 template <int APP, int GM, int LAY>
 __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
@@ -509,6 +519,10 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
   uint32_t d = 0;
   unsigned long long q_cur = 0, q_end = 0;  // this warp's claimed, not yet handed out positions
   bool drained = false;
+  __shared__ uint4 s_qr[8][2 * 32];     // per-warp staging of departing walks (records)
+  __shared__ uint32_t s_qd[8][2 * 32];  // and their destination buckets
+  const uint32_t wib = threadIdx.x >> 5;
+  uint32_t q_cnt = 0;
 #pragma unroll
   for (int q = 0; q < 8; ++q) pb[q] = 0;
 
@@ -616,11 +630,25 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
       my_steps += rec.z;
       my_trunc += trunc ? 1 : 0;
     }
-    uint32_t dest = 0;
-    if (left) dest = bucket_of(p, find_partition(B, wk.P, rec.y));
-    insert_warp(p, left, dest, rec);
+    // departing walks are staged per warp in shared memory and inserted 32-64 at a time, so the
+    // destination cursors see one atomic per (flush round, destination) instead of one per
+    // (step, destination): the warp-level form of the paper's local index
+    const uint32_t lm = __ballot_sync(kFull, left);
+    if (left) {
+      const uint32_t slot = q_cnt + __popc(lm & lanemask_lt());
+      s_qr[wib][slot] = rec;
+      s_qd[wib][slot] = bucket_of(p, find_partition(B, wk.P, rec.y));
+    }
+    q_cnt += __popc(lm);
+    if (q_cnt >= 32) {
+      __syncwarp();
+      flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
+      q_cnt = 0;
+    }
     if (ended) has = false;
   }
+  __syncwarp();
+  flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
   if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);

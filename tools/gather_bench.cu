@@ -51,7 +51,7 @@ __global__ void __launch_bounds__(256) k_gather(const uint4* __restrict__ buf, u
     uint32_t got[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      const uint64_t s = h[u] % slots;  // slot of WIDTH bytes
+      const uint64_t s = h[u] & (slots - 1);  // slot of WIDTH bytes (slots is a power of two)
       const char* p = (const char*)buf + s * WIDTH;
       uint32_t v;
       if (WIDTH == 4) v = ld4((const uint32_t*)p, g_mode);
@@ -67,7 +67,9 @@ __global__ void __launch_bounds__(256) k_gather(const uint4* __restrict__ buf, u
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       acc += got[u];
-      h[u] = DEP ? mix(h[u] + got[u]) : mix(h[u] + 0x632BE59BD9B4E019ULL);
+      // cheap next address (one IMAD + shift-xor): the benchmark must be bound by the gathers
+      h[u] = DEP ? (h[u] * 0x9E3779B97F4A7C15ULL + got[u]) ^ (h[u] >> 29)
+                 : (h[u] * 0x9E3779B97F4A7C15ULL + 0x632BE59BD9B4E019ULL) ^ (h[u] >> 29);
     }
   }
   if (acc == 0x12345678u) atomicAdd(sink, 1ull);
@@ -103,6 +105,7 @@ float dispatch_u(int U, bool dep, const uint4* buf, uint64_t bytes, int iters, i
 
 int main(int argc, char** argv) {
   uint64_t bytes = argc > 1 ? strtoull(argv[1], 0, 10) : (16ull << 30);
+  if (bytes & (bytes - 1)) { printf("bytes must be a power of two\n"); return 1; }
   int width = argc > 2 ? atoi(argv[2]) : 4;
   int U = argc > 3 ? atoi(argv[3]) : 4;
   int dep = argc > 4 ? atoi(argv[4]) : 0;
