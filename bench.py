@@ -61,6 +61,7 @@ def parse():
     ap.add_argument("--insert-mode", type=int, default=0)
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-chunks", type=int, default=16, help="lt_run_to_host walk ranges (copy-out overlap)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
     ap.add_argument("--layout", type=int, default=0, help="0 auto, 1 CSR, 2 ADJ (lt_layout)")
     ap.add_argument("--ilp", type=int, default=0)
@@ -434,9 +435,10 @@ def main():
         a.record()
         e_steps = 0
         for _ in range(args.e2e_steps):
-            eng.walks_init(h_starts, app, param, args.seed, first)
-            eng.run()
-            eng.get_paths(h_paths, h_len)
+            # lt_run_to_host: H2D of the starts, walks, and the D2H of every path and length, with the
+            # copy-out of walk range c overlapped with the walking of range c+1
+            eng.run_to_host(h_starts, app, param, args.seed, first, paths=h_paths, lengths=h_len,
+                            chunks=args.e2e_chunks)
             e_steps += eng.stats()["steps"]
         b.record()
         barrier()
@@ -446,9 +448,23 @@ def main():
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
             dist.all_reduce(es)
+        # the link the e2e copy-out rides on: pinned 1 GiB D2H, measured now
+        hb = torch.empty(1 << 30, dtype=torch.uint8, pin_memory=True)
+        db = torch.empty(1 << 30, dtype=torch.uint8, device="cuda")
+        hb.copy_(db, non_blocking=True)
+        a2, b2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a2.record()
+        for _ in range(4):
+            hb.copy_(db, non_blocking=True)
+        b2.record()
+        torch.cuda.synchronize()
+        d2h_gbs = 4 * (1 << 30) / (a2.elapsed_time(b2) / 1000) / 1e9
+        del hb, db
         e2e = {"value": float(es.item()) / (float(et.item()) / 1000), "unit": "steps/s",
+               "d2h_link_gbs": d2h_gbs,
+               "d2h_bound_steps_per_s": float(es.item()) / args.e2e_steps / ((W * S * 4 + W * 4) / (d2h_gbs * 1e9)),
                "h2d_bytes_per_step": W * 4, "d2h_bytes_per_step": W * S * 4 + W * 4, "pinned": pinned,
-               "steps": args.e2e_steps}
+               "steps": args.e2e_steps, "api": f"lt_run_to_host, {args.e2e_chunks} overlapped ranges"}
         del h_paths, h_len
 
     # ---- CPU oracle baseline on a bounded sample (rank 0, N=1) + sampled parity of that sample

@@ -196,6 +196,16 @@ lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_length
 
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out);
 
+/* End-to-end sampling into HOST buffers with the copy-out overlapped: the same result as
+ * lt_walks_init_ex(W, starts, host, first_walk_id, ...) + lt_run + lt_get_paths, computed in
+ * `chunks` consecutive walk ranges (0 -> 8) with two device path buffers: while range c+1 is walked,
+ * range c's paths and lengths stream to the host on a copy stream. paths is W x stride (stride as
+ * lt_path_stride would report: l+1 or L_max+1), lengths W; both should be pinned for the copies to
+ * overlap. Single-rank contexts only (world == 1). Stats afterwards cover all ranges. */
+lt_status lt_run_to_host(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, uint64_t first_walk_id,
+                         lt_app app, double length_or_alpha, uint64_t seed, uint32_t* paths, uint32_t* lengths,
+                         uint32_t chunks);
+
 /* ---- Range ownership across GPUs (the north star's multi-GPU mode, not
  * in the paper). With cfg.world = R > 1, rank r owns partitions [floor(P r / R), floor(P (r+1) / R));
  * every rank calls every function with identical arguments. lt_walks_init keeps the walks whose

@@ -77,7 +77,8 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   }
   cudaError_t e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
   if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_ctr, sizeof(lt::Counters));
-  if (e == cudaSuccess) e = cudaMallocHost((void**)&ctx->h_ctr, sizeof(lt::Counters));
+  if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_ctr, sizeof(lt::Counters), cudaHostAllocMapped);
+  if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_free, sizeof(int), cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaEventCreate(&ctx->ev_a);
   if (e == cudaSuccess) e = cudaEventCreate(&ctx->ev_b);
   if (e != cudaSuccess) {
@@ -111,6 +112,14 @@ void lt_destroy(lt_ctx* ctx) {
   cudaFree(ctx->d_owner);
   cudaFree(ctx->d_paths);
   cudaFree(ctx->d_lengths);
+  for (int i = 0; i < 2; ++i) {
+    if (ctx->d_paths2[i] && ctx->d_paths2[i] != ctx->d_paths) cudaFree(ctx->d_paths2[i]);
+    if (ctx->d_lengths2[i] && ctx->d_lengths2[i] != ctx->d_lengths) cudaFree(ctx->d_lengths2[i]);
+    if (ctx->d_dense2[i]) cudaFree(ctx->d_dense2[i]);
+    if (ctx->ev_computed[i]) cudaEventDestroy(ctx->ev_computed[i]);
+    if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+  }
+  if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
   cudaFree(ctx->d_starts);
   cudaFree(ctx->d_slots);
   cudaFree(ctx->d_ring);
@@ -120,6 +129,7 @@ void lt_destroy(lt_ctx* ctx) {
   cudaFree(ctx->d_ctr);
   if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
   if (ctx->h_ctr) cudaFreeHost(ctx->h_ctr);
+  if (ctx->h_free) cudaFreeHost(ctx->h_free);
   for (auto ev : ctx->events) cudaEventDestroy(ev);
   if (ctx->ev_a) cudaEventDestroy(ctx->ev_a);
   if (ctx->ev_b) cudaEventDestroy(ctx->ev_b);
@@ -206,7 +216,7 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
     ctx->h_hc = nullptr;
     ctx->h_hc_cap = 0;
-    CK(cudaMallocHost((void**)&ctx->h_hc, 2 * nb * sizeof(unsigned long long)));
+    CK(cudaHostAlloc((void**)&ctx->h_hc, 2 * nb * sizeof(unsigned long long), cudaHostAllocMapped));
     ctx->h_hc_cap = 2 * nb;
   }
   CK(cudaEventRecord(ctx->ev_b, ctx->stream));
@@ -520,8 +530,8 @@ lt_status lt_run(lt_ctx* ctx) {
     ctx->stats.kernel_launches++;
   }
   CK(cudaEventRecord(ctx->ev_b, s));
-  CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(lt::Counters), cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
+  st = lt::snapshot(ctx);
+  if (st != LT_OK) return st;
   {
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
@@ -646,8 +656,8 @@ lt_status lt_pending(lt_ctx* ctx, uint64_t* local, uint64_t* outgoing) {
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
   CK(cudaSetDevice(ctx->cfg.device));
   const size_t nb = ctx->nb;
-  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * nb * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
-  CK(cudaStreamSynchronize(ctx->stream));
+  lt_status sn = lt::snapshot(ctx);
+  if (sn != LT_OK) return sn;
   uint64_t loc = 0;
   for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k) loc += ctx->h_hc[nb + k] - ctx->h_hc[k];
   if (local) *local = loc;
@@ -686,6 +696,94 @@ lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count) {
   CK(lt::launch_insert_records(ctx->params, (const uint4*)d_recv, count, ctx->stream));
   if (count) ctx->stats.kernel_launches++;
   CK(cudaStreamSynchronize(ctx->stream));
+  return LT_OK;
+}
+
+lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64_t first_walk_id, lt_app app,
+                         double param, uint64_t seed, uint32_t* paths, uint32_t* lengths, uint32_t chunks) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if (ctx->world != 1) return fail(LT_ERR_INVALID, "lt_run_to_host needs a single-rank context");
+  if (W && (!starts || !paths || !lengths)) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_run_to_host before lt_graph_load");
+  CK(cudaSetDevice(ctx->cfg.device));
+  if (chunks == 0) chunks = 8;
+  const uint64_t wc = std::max<uint64_t>((W + chunks - 1) / chunks, 1);
+  if (!ctx->copy_stream) {
+    CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i) {
+      CK(cudaEventCreateWithFlags(&ctx->ev_computed[i], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming));
+      CK(cudaEventRecord(ctx->ev_copied[i], ctx->copy_stream));
+    }
+  }
+  // the chunk buffers stand in for the context's path/length arrays while this call runs
+  uint32_t* save_p = ctx->d_paths;
+  size_t save_pc = ctx->paths_cap;
+  uint32_t* save_l = ctx->d_lengths;
+  size_t save_lc = ctx->lengths_cap;
+  uint64_t steps = 0, visits = 0, trunc = 0, launches = 0, upd = 0, sweeps = 0, h2d = 0, d2h = 0;
+  double run_ms = 0, init_ms = 0, update_ms = 0;
+  lt_status st = LT_OK;
+  for (uint64_t a = 0, c = 0; a < W || (W == 0 && c == 0); a += wc, ++c) {
+    const uint64_t n = std::min<uint64_t>(wc, W - a);
+    const int b = (int)(c & 1);
+    CK(cudaEventSynchronize(ctx->ev_copied[b]));  // buffer b's previous chunk reached the host
+    ctx->d_paths = ctx->d_paths2[b];
+    ctx->paths_cap = ctx->paths2_cap[b];
+    ctx->d_lengths = ctx->d_lengths2[b];
+    ctx->lengths_cap = ctx->lengths2_cap[b];
+    st = lt_walks_init_ex(ctx, n, starts + a, 0, first_walk_id + a, app, param, seed);
+    if (st == LT_OK) st = lt_run(ctx);
+    ctx->d_paths2[b] = ctx->d_paths;  // (re)allocated by walks_init as needed
+    ctx->paths2_cap[b] = ctx->paths_cap;
+    ctx->d_lengths2[b] = ctx->d_lengths;
+    ctx->lengths2_cap[b] = ctx->lengths_cap;
+    if (st != LT_OK) break;
+    steps += ctx->stats.steps;
+    visits += ctx->stats.visits;
+    trunc += ctx->stats.truncated;
+    launches += ctx->stats.kernel_launches;
+    upd += ctx->stats.update_launches;
+    sweeps += ctx->stats.sweeps;
+    run_ms += ctx->stats.run_ms;
+    init_ms += ctx->stats.init_ms;
+    update_ms += ctx->stats.update_ms;
+    h2d += ctx->stats.h2d_bytes;
+    if (n) {  // stream chunk c out while chunk c+1 computes
+      // dense rows first (a 2-D copy of 324-B rows runs well below the link rate)
+      CK(ensure(ctx->d_dense2[b], ctx->dense2_cap[b], n * ctx->stride));
+      CK(lt::launch_compact_rows(ctx->d_paths2[b], ctx->pitch, ctx->stride, n, ctx->d_dense2[b], ctx->stream));
+      CK(cudaEventRecord(ctx->ev_computed[b], ctx->stream));
+      CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_computed[b], 0));
+      CK(cudaMemcpyAsync(paths + a * ctx->stride, ctx->d_dense2[b], n * ctx->stride * sizeof(uint32_t),
+                         cudaMemcpyDeviceToHost, ctx->copy_stream));
+      CK(cudaMemcpyAsync(lengths + a, ctx->d_lengths2[b], n * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                         ctx->copy_stream));
+      CK(cudaEventRecord(ctx->ev_copied[b], ctx->copy_stream));
+      d2h += n * (ctx->stride + 1) * 4;
+    }
+    if (W == 0) break;
+  }
+  CK(cudaStreamSynchronize(ctx->copy_stream));
+  ctx->d_paths = save_p;
+  ctx->paths_cap = save_pc;
+  ctx->d_lengths = save_l;
+  ctx->lengths_cap = save_lc;
+  ctx->walks_ready = false;  // the context's own path arrays do not hold these walks
+  ctx->ran = false;
+  if (st != LT_OK) return st;
+  ctx->stats.num_walks = W;
+  ctx->stats.steps = steps;
+  ctx->stats.visits = visits;
+  ctx->stats.truncated = trunc;
+  ctx->stats.kernel_launches = launches;
+  ctx->stats.update_launches = upd;
+  ctx->stats.sweeps = sweeps;
+  ctx->stats.run_ms = run_ms;
+  ctx->stats.init_ms = init_ms;
+  ctx->stats.update_ms = update_ms;
+  ctx->stats.h2d_bytes = h2d;
+  ctx->stats.d2h_bytes = d2h;
   return LT_OK;
 }
 

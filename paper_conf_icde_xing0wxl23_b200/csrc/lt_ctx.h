@@ -91,13 +91,23 @@ struct lt_ctx {
   uint32_t* d_small = nullptr;  // [0]=free_top [1]=unused [2..3]=scratch flags
   lt::Counters* d_ctr = nullptr;
   // pinned staging
-  unsigned long long* h_hc = nullptr;
+  unsigned long long* h_hc = nullptr;  // mapped pinned: head[nb], cursor[nb]
   size_t h_hc_cap = 0;
-  lt::Counters* h_ctr = nullptr;
+  lt::Counters* h_ctr = nullptr;       // mapped pinned
+  int* h_free = nullptr;               // mapped pinned: free-stack top
   lt::Params params{};
   lt_stats stats{};
   std::vector<cudaEvent_t> events;
   size_t nev = 0;
+  // lt_run_to_host double buffers
+  uint32_t* d_paths2[2] = {nullptr, nullptr};
+  size_t paths2_cap[2] = {0, 0};
+  uint32_t* d_lengths2[2] = {nullptr, nullptr};
+  size_t lengths2_cap[2] = {0, 0};
+  uint32_t* d_dense2[2] = {nullptr, nullptr};  // dense (stride-pitched) staging for the flat D2H
+  size_t dense2_cap[2] = {0, 0};
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_computed[2] = {nullptr, nullptr}, ev_copied[2] = {nullptr, nullptr};
   cudaEvent_t ev_a = nullptr, ev_b = nullptr;
 };
 
@@ -110,6 +120,7 @@ struct lt_ctx {
   } while (0)
 
 namespace lt {
+lt_status snapshot(lt_ctx* ctx);  // h_hc / h_ctr / h_free <- device, then sync the stream
 lt_status run_resident(lt_ctx* ctx);
 lt_status run_out_of_core(lt_ctx* ctx);
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound);

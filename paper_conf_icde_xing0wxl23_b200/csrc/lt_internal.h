@@ -86,6 +86,10 @@ cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t b
 cudaError_t launch_finalize_paths(const Params& p, uint64_t W, cudaStream_t s);
 cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, uint64_t count,
                                uint32_t* out_paths, uint32_t* out_lengths, cudaStream_t s);
+cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Counters* ctr, const int* free_top,
+                            unsigned long long* out_hc, Counters* out_ctr, int* out_free, cudaStream_t s);
+cudaError_t launch_compact_rows(const uint32_t* paths, uint64_t pitch, uint64_t stride, uint64_t n, uint32_t* out,
+                                cudaStream_t s);
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);

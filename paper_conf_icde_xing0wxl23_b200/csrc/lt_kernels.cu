@@ -687,6 +687,31 @@ __global__ void k_gather_rows(Params p, const unsigned long long* rows, uint64_t
   }
 }
 
+// Scheduler snapshot: head/cursor of every bucket, the counters and the free-stack top, written
+// by the SMs straight into mapped pinned host memory. A cudaMemcpy would queue behind a large D2H
+// on the same copy engine (lt_run_to_host's path copy-out) and serialise the pipeline.
+__global__ void k_snapshot(const unsigned long long* __restrict__ hc, uint64_t n, const Counters* __restrict__ ctr,
+                           const int* __restrict__ free_top, volatile unsigned long long* out_hc,
+                           volatile Counters* out_ctr, volatile int* out_free) {
+  for (uint64_t i = threadIdx.x; i < n; i += blockDim.x) out_hc[i] = hc[i];
+  if (threadIdx.x == 0) {
+    out_ctr->steps = ctr->steps;
+    out_ctr->visits = ctr->visits;
+    out_ctr->truncated = ctr->truncated;
+    out_ctr->err = ctr->err;
+    out_ctr->done_ctas = ctr->done_ctas;
+    *out_free = *free_top;
+  }
+}
+
+// Rows [0, n) of the pitched path matrix -> a dense n x stride buffer (one flat D2H afterwards).
+__global__ void k_compact_rows(const uint32_t* __restrict__ paths, uint64_t pitch, uint64_t stride, uint64_t n,
+                               uint32_t* __restrict__ out) {
+  const uint64_t total = n * stride;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = paths[(i / stride) * pitch + (i % stride)];
+}
+
 __global__ void k_check_range(const uint32_t* a, uint64_t cnt, uint32_t n, uint32_t* bad) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += (uint64_t)gridDim.x * blockDim.x)
     if (a[i] >= n) { atomicOr(bad, 1u); return; }
@@ -840,6 +865,19 @@ cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, 
   uint64_t want = (count * p.wk.stride + 255) / 256;
   uint32_t grid = (uint32_t)std::min<uint64_t>(want ? want : 1, (uint64_t)num_sms() * 8);
   k_gather_rows<<<grid, 256, 0, s>>>(p, rows, count, out_paths, out_lengths);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Counters* ctr, const int* free_top,
+                            unsigned long long* out_hc, Counters* out_ctr, int* out_free, cudaStream_t s) {
+  k_snapshot<<<1, 256, 0, s>>>(hc, n, ctr, free_top, out_hc, out_ctr, out_free);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_compact_rows(const uint32_t* paths, uint64_t pitch, uint64_t stride, uint64_t n, uint32_t* out,
+                                cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_compact_rows<<<num_sms() * 8, 256, 0, s>>>(paths, pitch, stride, n, out);
   return cudaGetLastError();
 }
 

@@ -21,13 +21,9 @@ namespace lt {
 namespace {
 
 lt_status read_counts(lt_ctx* ctx) {
-  cudaStream_t s = ctx->stream;
-  CK(cudaMemcpyAsync(ctx->h_hc, ctx->d_hc, 2 * (size_t)ctx->nb * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
-  CK(cudaMemcpyAsync(ctx->h_ctr, ctx->d_ctr, sizeof(Counters), cudaMemcpyDeviceToHost, s));
-  int free_top = 0;
-  CK(cudaMemcpyAsync(&free_top, ctx->d_small, sizeof(int), cudaMemcpyDeviceToHost, s));
-  CK(cudaStreamSynchronize(s));
-  ctx->stats.chunks_free_min = std::min<uint64_t>(ctx->stats.chunks_free_min, (uint64_t)std::max(free_top, 0));
+  lt_status st = snapshot(ctx);
+  if (st != LT_OK) return st;
+  ctx->stats.chunks_free_min = std::min<uint64_t>(ctx->stats.chunks_free_min, (uint64_t)std::max(*ctx->h_free, 0));
   return LT_OK;
 }
 
@@ -41,6 +37,19 @@ bool event_done(cudaEvent_t e) {
 }
 
 }  // namespace
+
+lt_status snapshot(lt_ctx* ctx) {
+  unsigned long long* dh = nullptr;
+  Counters* dc = nullptr;
+  int* df = nullptr;
+  CK(cudaHostGetDevicePointer((void**)&dh, ctx->h_hc, 0));
+  CK(cudaHostGetDevicePointer((void**)&dc, ctx->h_ctr, 0));
+  CK(cudaHostGetDevicePointer((void**)&df, ctx->h_free, 0));
+  CK(launch_snapshot(ctx->d_hc, 2 * (uint64_t)ctx->nb, ctx->d_ctr, (const int*)ctx->d_small, dh, dc, df, ctx->stream));
+  ctx->stats.kernel_launches++;
+  CK(cudaStreamSynchronize(ctx->stream));
+  return LT_OK;
+}
 
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
   cudaStream_t s = ctx->stream;

@@ -32,7 +32,7 @@ EXPORTED = [
     "lt_config_default", "lt_create", "lt_destroy", "lt_last_error", "lt_partition_bounds", "lt_graph_load",
     "lt_graph_load_device", "lt_get_bounds", "lt_walks_init", "lt_walks_init_ex", "lt_run", "lt_path_stride",
     "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
-    "lt_pending", "lt_exchange_pack", "lt_exchange_insert",
+    "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host",
 ]
 
 
@@ -103,6 +103,7 @@ _lib.lt_get_pool_state.argtypes = [_vp, ctypes.POINTER(PoolState)]
 _lib.lt_pending.argtypes = [_vp, ctypes.POINTER(_u64), _vp]
 _lib.lt_exchange_pack.argtypes = [_vp, _vp, _u64, _vp]
 _lib.lt_exchange_insert.argtypes = [_vp, _vp, _u64]
+_lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
 
 
 class LTError(RuntimeError):
@@ -179,6 +180,7 @@ class Engine:
         cfg.rank = rank
         cfg.world = world
         cfg.refill = refill
+        self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device
         h = _vp()
         _check(_lib.lt_create(ctypes.byref(cfg), ctypes.byref(h)))
@@ -235,6 +237,26 @@ class Engine:
 
     def run(self):
         _check(_lib.lt_run(self._h))
+
+    def run_to_host(self, starts, app: int = DEEPWALK, param: float = 80, seed: int = 1, first_walk_id: int = 0,
+                    paths=None, lengths=None, chunks: int = 0):
+        """Walk and copy every path to host buffers with the copy-out overlapped (lt_run_to_host).
+        starts/paths/lengths are host arrays (pinned torch tensors for overlapped copies)."""
+        ps, dev, keep = _ptr(starts, np.uint32)
+        if dev:
+            raise ValueError("run_to_host takes host starts")
+        W = keep.numel() if _is_torch(keep) else len(keep)
+        S = (int(param) + 1) if app == DEEPWALK else self._lmax + 1
+        if paths is None:
+            paths = np.empty((W, S), dtype=np.uint32)
+        if lengths is None:
+            lengths = np.empty(W, dtype=np.uint32)
+        pp, dp, kp = _ptr(paths, np.uint32)
+        pl, dl, kl = _ptr(lengths, np.uint32)
+        if dp or dl:
+            raise ValueError("run_to_host writes host buffers")
+        _check(_lib.lt_run_to_host(self._h, W, ps, first_walk_id, app, float(param), seed, pp, pl, chunks))
+        return paths, lengths
 
     def stride(self) -> int:
         s = _u32()

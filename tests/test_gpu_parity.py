@@ -256,3 +256,23 @@ def test_path_mode_off_keeps_lengths(gpu, cfg1):
     _, ol, osteps, _ = run_oracle(cfg1, starts, LT.PPR, 0.15, 4)
     np.testing.assert_array_equal(lengths, ol)
     assert st["steps"] == osteps
+
+
+@pytest.mark.parametrize("chunks", [1, 3, 8])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 11), (LT.PPR, 0.2)])
+def test_run_to_host_streamed(gpu, cfg1, chunks, app, param):
+    import torch
+    W = 5000
+    starts = lt_inputs.deepwalk_starts(W, cfg1.n) if app == LT.DEEPWALK else lt_inputs.ppr_starts(W, cfg1.argmax_deg)
+    S = param + 1 if app == LT.DEEPWALK else O.DEFAULT_LMAX + 1
+    paths = torch.empty((W, S), dtype=torch.int32, pin_memory=True)
+    lengths = torch.empty(W, dtype=torch.int32, pin_memory=True)
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 1)
+        e.run_to_host(torch.from_numpy(starts.view(np.int32)), app, param, 6, first_walk_id=17, paths=paths,
+                      lengths=lengths, chunks=chunks)
+        st = e.stats()
+    op, ol, osteps, _ = run_oracle(cfg1, starts, app, param, 6, first=17)
+    np.testing.assert_array_equal(lengths.numpy().view(np.uint32), ol)
+    np.testing.assert_array_equal(paths.numpy().view(np.uint32), op)
+    assert st["steps"] == osteps and st["num_walks"] == W
