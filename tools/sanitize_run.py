@@ -1,0 +1,53 @@
+#!/usr/bin/env python3
+"""Small runs of every kernel path for compute-sanitizer (memcheck / racecheck / synccheck /
+initcheck): resident P=1 (refill), P=4 (batch kernel, CSR and ADJ), PPR, out-of-core with zero copy,
+two-rank ownership, streamed run_to_host."""
+import os
+import sys
+import threading
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import lt_inputs  # noqa: E402
+import paper_conf_icde_xing0wxl23_b200 as LT  # noqa: E402
+from paper_conf_icde_xing0wxl23_b200 import dist as ltdist  # noqa: E402
+
+g = lt_inputs.rmat_cpu(12, 65_536, seed=1)
+starts = lt_inputs.deepwalk_starts(4096, g.n)
+pstarts = lt_inputs.ppr_starts(4096, g.argmax_deg)
+for kw in [dict(P=1), dict(P=4, layout=LT.LAYOUT_CSR), dict(P=4, layout=LT.LAYOUT_ADJ), dict(P=4, refill=2)]:
+    P = kw.pop("P")
+    with LT.Engine(chunk_walks=256, **kw) as e:
+        e.graph_load(g.row_ptr, g.col, P)
+        for st, app, prm in [(starts, LT.DEEPWALK, 10), (pstarts, LT.PPR, 0.15)]:
+            e.walks_init(st, app, prm, 1)
+            e.run()
+            e.get_paths()
+with LT.Engine(graph_pool_bytes=1 << 20, zero_copy=True, chunk_walks=256) as e:
+    e.graph_load(g.row_ptr, g.col, 8)
+    e.walks_init(starts, LT.DEEPWALK, 10, 1)
+    e.run()
+    e.get_paths()
+with LT.Engine() as e:
+    e.graph_load(g.row_ptr, g.col, 1)
+    e.run_to_host(starts, LT.DEEPWALK, 10, 1, chunks=3)
+hub = ltdist.ThreadComm.Hub(2)
+
+
+def rank(r):
+    with LT.Engine(rank=r, world=2, chunk_walks=256) as e:
+        e.graph_load(g.row_ptr, g.col, 4)
+        e.walks_init(starts, LT.DEEPWALK, 10, 1)
+        comm = ltdist.ThreadComm(hub, r)
+        ltdist.run_supersteps(e, comm, "cuda")
+        ltdist.merge_paths(e, comm)
+
+
+th = [threading.Thread(target=rank, args=(r,)) for r in range(2)]
+for t in th:
+    t.start()
+for t in th:
+    t.join()
+print("sanitize_run done")
