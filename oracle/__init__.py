@@ -17,6 +17,7 @@ _LIB = None
 
 DEEPWALK = 0
 PPR = 1
+PAGERANK = 2
 EMPTY = 0xFFFFFFFF
 DEFAULT_LMAX = 127  # DESIGN.md reading R6
 
@@ -43,6 +44,7 @@ def _lib():
                                      ctypes.c_uint32, _u32p, _u64p, ctypes.c_int]
         lib.oracle_walks.restype = ctypes.c_uint64
         lib.oracle_lemire_exhaustive.argtypes = [ctypes.c_uint32, _u64p, _u64p, ctypes.c_int]
+        lib.oracle_visit_counts.argtypes = [ctypes.c_uint64, _u32p, ctypes.c_uint32, _u32p, _u64p]
         _LIB = lib
     return _LIB
 
@@ -83,12 +85,23 @@ def lemire_exhaustive(d: int, threads: int = 0):
 
 
 def stride_for(app: int, length: int = 0, lmax: int = DEFAULT_LMAX) -> int:
-    return (length + 1) if app == DEEPWALK else (lmax + 1)
+    return (lmax + 1) if app == PPR else (length + 1)
+
+
+def visit_counts(paths, lengths, n):
+    """Visit frequency per vertex from path rows."""
+    paths = np.ascontiguousarray(paths, dtype=np.uint32)
+    lengths = np.ascontiguousarray(lengths, dtype=np.uint32)
+    counts = np.zeros(n, dtype=np.uint64)
+    _lib().oracle_visit_counts(len(lengths), _p(paths, _u32p), paths.shape[1] if paths.ndim == 2 else 1,
+                               _p(lengths, _u32p), _p(counts, _u64p))
+    return counts
 
 
 def walks(row_ptr, col, starts, app=DEEPWALK, length=80, alpha=0.15, lmax=DEFAULT_LMAX, seed=1,
           ids=None, threads=0):
-    """Run the oracle for walks `ids` (default 0..len(starts)-1) from `starts`.
+    """Run the oracle for walks `ids` (default 0..len(starts)-1) from `starts`. alpha is the PPR
+    termination probability or the PageRank restart probability.
     Returns (paths u32[count, stride], lengths u32[count], steps, truncated)."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.uint64)
     col = np.ascontiguousarray(col, dtype=np.uint32)
@@ -98,7 +111,7 @@ def walks(row_ptr, col, starts, app=DEEPWALK, length=80, alpha=0.15, lmax=DEFAUL
         ids = np.ascontiguousarray(ids, dtype=np.uint64)
         assert len(ids) == count
     n = len(row_ptr) - 1
-    T = ppr_threshold(alpha) if app == PPR else 0
+    T = ppr_threshold(alpha) if app in (PPR, PAGERANK) else 0
     stride = stride_for(app, length, lmax)
     paths = np.empty((count, stride), dtype=np.uint32)
     lengths = np.empty(count, dtype=np.uint32)

@@ -87,29 +87,41 @@ uint32_t oracle_lemire(uint64_t seed, uint64_t w, uint32_t t, uint32_t d, uint32
   }
 }
 
-/* One walk, SURVEY.md §8(c) "Definition":
+/* One walk, SURVEY.md §8(c) "Definition" (+ PageRank, reading R23):
  *   v = start; path[0] = v; t = 0
  *   loop: DeepWalk and t == l -> stop ("walked steps reaches l"; reading R1)
  *         PPR and t == L_max -> stop, truncated (reading R6)
  *         PPR and blk(w,t,0).x0 < T -> stop (terminate with probability p before moving; R2, R5)
  *         d = deg(v); d == 0 -> stop (dead end; reading R9)
  *         v = col[row_ptr[v] + lemire(d)]  (uniform neighbour); t += 1; path[t] = v
+ *   PageRank ("at each step, a walk has a probability p to restart at a random vertex,
+ *   instead of uniformly selecting one of the neighbors"): stop when t == l; if blk(w,t,0).x0 < T the
+ *   step goes to vertex lemire(n) (same word stream), else to a uniform neighbour as above.
  */
 uint32_t oracle_walk(uint32_t n, const uint64_t* row_ptr, const uint32_t* col, uint64_t w, uint32_t start,
                      int app, uint32_t length, uint32_t T, uint32_t lmax, uint64_t seed,
                      uint32_t* path, int* truncated) {
-  (void)n;
   uint32_t v = start;
   uint32_t t = 0;
   path[0] = v;
   *truncated = 0;
   for (;;) {
-    if (app == ORACLE_DEEPWALK && t == length) break;
+    if ((app == ORACLE_DEEPWALK || app == ORACLE_PAGERANK) && t == length) break;
     if (app == ORACLE_PPR && t == lmax) { *truncated = 1; break; }
     if (app == ORACLE_PPR) {
       uint32_t b[4];
       blk(seed, w, t, 0, b);
       if (b[0] < T) break;
+    }
+    if (app == ORACLE_PAGERANK) {
+      uint32_t b[4];
+      blk(seed, w, t, 0, b);
+      if (b[0] < T) {  /* restart at a uniform random vertex */
+        v = oracle_lemire(seed, w, t, n, NULL);
+        t += 1;
+        path[t] = v;
+        continue;
+      }
     }
     uint64_t d = row_ptr[v + 1] - row_ptr[v];
     if (d == 0) break;
@@ -144,6 +156,12 @@ uint64_t oracle_walks(uint32_t n, const uint64_t* row_ptr, const uint32_t* col, 
   }
   if (truncated) *truncated = trunc;
   return steps;
+}
+
+void oracle_visit_counts(uint64_t count, const uint32_t* paths, uint32_t stride, const uint32_t* lengths,
+                         uint64_t* counts) {
+  for (uint64_t r = 0; r < count; ++r)
+    for (uint32_t t = 0; t < lengths[r]; ++t) counts[paths[r * stride + t]] += 1;
 }
 
 void oracle_lemire_exhaustive(uint32_t d, uint64_t* hist, uint64_t* rejected, int threads) {

@@ -13,6 +13,9 @@
  *   (t, j, w_lo, w_hi); the uniform neighbour index is Lemire's unbiased multiply-shift with
  *   rejection (reading R4) over the word stream blk(w,t,0).x1..x3, blk(w,t,1).x0..x3, ...
  *   The PPR coin is x0 < T with T = floor(alpha * 2^32) (reading R5).
+ *   PageRank (reading R23): fixed length l; at each step the same coin x0 < T (T from
+ *   the restart probability p) sends the walk to a uniform vertex, Lemire over n on the same word
+ *   stream, instead of to a uniform neighbour.
  * Pins: tests/test_oracle_pins.py (Philox KATs, Lemire exhaustive counts, closed-form Markov and
  * PPR distributions, chi-square uniformity, geometric length, edge validity, brute force).
  */
@@ -22,6 +25,7 @@
 
 #define ORACLE_DEEPWALK 0
 #define ORACLE_PPR 1
+#define ORACLE_PAGERANK 2 /* random walk with restart; reading R23 */
 #define ORACLE_EMPTY 0xFFFFFFFFu
 
 void oracle_philox4x32_10(const uint32_t ctr[4], const uint32_t key[2], uint32_t out[4]);
@@ -44,6 +48,11 @@ uint64_t oracle_walks(uint32_t n, const uint64_t* row_ptr, const uint32_t* col, 
                       const uint64_t* ids, const uint32_t* starts, int app, uint32_t length,
                       uint32_t T, uint32_t lmax, uint64_t seed, uint32_t* paths, uint32_t stride,
                       uint32_t* lengths, uint64_t* truncated, int threads);
+
+/* Visit frequency: counts[v] += number of path entries equal to v, over the
+ * `count` rows of paths (row r has lengths[r] entries). */
+void oracle_visit_counts(uint64_t count, const uint32_t* paths, uint32_t stride, const uint32_t* lengths,
+                         uint64_t* counts);
 
 /* Lemire exhaustive check (pin P4): over all 2^32 words x, histogram of accepted residues. */
 void oracle_lemire_exhaustive(uint32_t d, uint64_t* hist, uint64_t* rejected, int threads);

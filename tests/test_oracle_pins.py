@@ -226,6 +226,41 @@ def test_p7_ppr_endpoint_is_textbook_ppr_vector(name):
     assert _chi2_against(np.bincount(ends, minlength=g.n), pi) > P_MIN
 
 
+@pytest.mark.parametrize("name", sorted(TINY))
+@pytest.mark.parametrize("t", [1, 4, 9])
+def test_p7_pagerank_endpoint_is_restart_chain_power(name, t):
+    """Random walk with restart: the position after t steps is e_s M^t with
+    M = (1-p) D^-1 A + p J/n (restart to a uniform vertex)."""
+    g = lt_inputs.small_graph(TINY[name])
+    p = 0.3
+    M = (1 - p) * _transition(g) + p * np.full((g.n, g.n), 1.0 / g.n)
+    s = 0
+    W = 200_000
+    paths, lengths, _, _ = O.walks(g.row_ptr, g.col, np.full(W, s, np.uint32), app=O.PAGERANK, length=t, alpha=p,
+                                   seed=300 + t)
+    assert np.all(lengths == t + 1)
+    expect = np.linalg.matrix_power(M, t)[s]
+    assert _chi2_against(np.bincount(paths[:, t], minlength=g.n), expect) > P_MIN
+
+
+def test_pagerank_restart_rate_and_visit_counts():
+    """On a path graph 0-1-...-9 a restart is visible as a non-neighbour jump with probability
+    (1 - deg/n) per restart; the observed rate of non-neighbour jumps pins the restart probability.
+    Visit counts are the histogram of the path entries."""
+    g = lt_inputs.small_graph([(k, k + 1) for k in range(9)])
+    p, W, L = 0.25, 20_000, 20
+    paths, lengths, _, _ = O.walks(g.row_ptr, g.col, lt_inputs.deepwalk_starts(W, g.n), app=O.PAGERANK, length=L,
+                                   alpha=p, seed=8)
+    a, b = paths[:, :-1].astype(np.int64), paths[:, 1:].astype(np.int64)
+    jump = np.abs(a - b) != 1
+    deg = np.diff(g.row_ptr.astype(np.int64))
+    expect = p * np.mean(1 - deg[a] / g.n)  # a restart lands on a non-neighbour w.p. 1 - deg/n
+    assert abs(jump.mean() - expect) < 4 * np.sqrt(expect * (1 - expect) / jump.size)
+    counts = O.visit_counts(paths, lengths, g.n)
+    np.testing.assert_array_equal(counts, np.bincount(paths.ravel(), minlength=g.n))
+    assert counts.sum() == W * (L + 1)
+
+
 # ---------------------------------------------------------------- P8: PPR length law
 def test_p8_ppr_length_is_geometric():
     g = lt_inputs.small_graph(TINY["k4"])
@@ -276,17 +311,18 @@ def _sync_simulator(g, starts, app, length, alpha, lmax, seed):
     """All walks advance together, one global step at a time (different loop structure from the
     per-walk oracle; same definition)."""
     W = len(starts)
-    stride = length + 1 if app == O.DEEPWALK else lmax + 1
+    stride = lmax + 1 if app == O.PPR else length + 1
     paths = np.full((W, stride), O.EMPTY, dtype=np.uint64)
     v = starts.astype(np.uint64)
     paths[:, 0] = v
     alive = np.ones(W, dtype=bool)
     t_len = np.ones(W, dtype=np.int64)
-    T = np.uint64(int(np.floor(alpha * 2.0 ** 32))) if app == O.PPR else None
+    T = np.uint64(int(np.floor(alpha * 2.0 ** 32))) if app in (O.PPR, O.PAGERANK) else None
+    n = np.uint64(g.n)
     rp = g.row_ptr.astype(np.uint64)
     wid = np.arange(W, dtype=np.uint64)
     for t in range(stride - 1 + 1):
-        if app == O.DEEPWALK and t == length:
+        if app in (O.DEEPWALK, O.PAGERANK) and t == length:
             break
         if app == O.PPR and t == lmax:
             break
@@ -300,10 +336,14 @@ def _sync_simulator(g, starts, app, length, alpha, lmax, seed):
             stop = b[0] < T
             alive[idx[stop]] = False
             idx, b = idx[~stop], tuple(x[~stop] for x in b)
-        d = rp[v[idx] + np.uint64(1)] - rp[v[idx]]
-        dead = d == 0
+        restart = np.zeros(len(idx), dtype=bool)
+        if app == O.PAGERANK:
+            restart = b[0] < T
+        # restarting walks pick a uniform vertex, Lemire over n on the same word stream
+        d = np.where(restart, n, rp[v[idx] + np.uint64(1)] - rp[v[idx]])
+        dead = (d == 0) & ~restart
         alive[idx[dead]] = False
-        idx, d, b = idx[~dead], d[~dead], tuple(x[~dead] for x in b)
+        idx, d, b, restart = idx[~dead], d[~dead], tuple(x[~dead] for x in b), restart[~dead]
         choice = np.zeros(len(idx), dtype=np.uint64)
         done = np.zeros(len(idx), dtype=bool)
         thr = (np.uint64(2 ** 32) % d)
@@ -320,17 +360,18 @@ def _sync_simulator(g, starts, app, length, alpha, lmax, seed):
             acc = (~done) & ((m & _MASK) >= thr)
             choice[acc] = m[acc] >> np.uint64(32)
             done |= acc
-        v[idx] = g.col[(rp[v[idx]] + choice).astype(np.int64)].astype(np.uint64)
+        moved = g.col[np.where(restart, 0, rp[v[idx]] + choice).astype(np.int64)].astype(np.uint64)
+        v[idx] = np.where(restart, choice, moved)
         paths[idx, t + 1] = v[idx]
         t_len[idx] = t + 2
     return paths.astype(np.uint32), t_len.astype(np.uint32)
 
 
-@pytest.mark.parametrize("app", [O.DEEPWALK, O.PPR])
+@pytest.mark.parametrize("app", [O.DEEPWALK, O.PPR, O.PAGERANK])
 def test_p10_brute_force_synchronous_equals_oracle(app):
     g = lt_inputs.rmat_cpu(10, 16 * 1024, seed=4)
     W = 3000
-    starts = lt_inputs.deepwalk_starts(W, g.n) if app == O.DEEPWALK else lt_inputs.ppr_starts(W, g.argmax_deg)
+    starts = lt_inputs.ppr_starts(W, g.argmax_deg) if app == O.PPR else lt_inputs.deepwalk_starts(W, g.n)
     kw = dict(app=app, length=12, alpha=0.3, lmax=20, seed=0x1234_5678_9ABC)
     po, lo, _, _ = O.walks(g.row_ptr, g.col, starts, **kw)
     ps, ls = _sync_simulator(g, starts, kw["app"], kw["length"], kw["alpha"], kw["lmax"], kw["seed"])
