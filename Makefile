@@ -45,7 +45,14 @@ $(CSRC)/%.o: $(CSRC)/%.cpp $(LT_H)
 $(PKG)/liblt.so: $(LT_CU:.cu=.o) $(LT_CPP:.cpp=.o)
 	$(NVCC) $(ARCH) -shared $^ -o $@
 
+# Experiment builds of liblt.so with compile-time switches (tools/variants/ is not shipped product):
+#   make variant VTAG=nohint VDEFS="-DLT_PATH_HINT=0 -DLT_VIS_HINT=0"; run with LT_LIBRARY=tools/variants/liblt_nohint.so
+variant: $(LT_CPP:.cpp=.o)
+	mkdir -p tools/variants
+	$(NVCC) $(NVFLAGS) $(VDEFS) -Iinclude -c $(CSRC)/lt_kernels.cu -o tools/variants/lt_kernels_$(VTAG).o
+	$(NVCC) $(ARCH) -shared tools/variants/lt_kernels_$(VTAG).o $(LT_CPP:.cpp=.o) -o tools/variants/liblt_$(VTAG).so
+
 clean:
 	rm -f tools/gather_bench lt_inputs/*.o lt_inputs/*.so oracle/*.so $(CSRC)/*.o $(CSRC)/*.ptxas.txt $(PKG)/*.so
 
-.PHONY: all inputs oracle lt tools clean
+.PHONY: all inputs oracle lt tools clean variant

@@ -73,6 +73,11 @@ def parse():
     ap.add_argument("--graph-pool-gb", type=float, default=0.0,
                     help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
     ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
+    ap.add_argument("--app", default="config", choices=["config", "deepwalk", "ppr", "pagerank"],
+                    help="override the config's application; pagerank = random walk with restart "
+                         "(PAPER.md:287, SURVEY.md 8(f) f2) of the config's length, with visit counting")
+    ap.add_argument("--restart-p", type=float, default=0.15, help="PageRank restart probability")
+    ap.add_argument("--visit-counts", type=int, default=-1, help="fused visit counting: -1 auto (on for pagerank)")
     ap.add_argument("--mode", default="replicas", choices=["replicas", "own"],
                     help="N>1: replicas (each rank its own |V| walks, no collective, weak scaling) or own "
                          "(range ownership: |V| walks in total, NCCL all-to-all of crossing walks per "
@@ -90,6 +95,13 @@ def workload(args):
     if args.tuples is not None:
         c["tuples"] = args.tuples
     c["partitions"] = args.partitions if args.partitions is not None else (c.get("partitions") or DEFAULT_P[args.config])
+    if args.app != "config" and args.app != c["app"]:
+        c["name"] = f"{args.app} on {c['name']}"
+        c["app"] = args.app
+        c.setdefault("length", 80)
+        c.setdefault("alpha", 0.15)
+    if c["app"] == "pagerank":
+        c["restart_p"] = args.restart_p
     return c
 
 
@@ -97,11 +109,23 @@ def app_param(c):
     import paper_conf_icde_xing0wxl23_b200 as LT
     if c["app"] == "deepwalk":
         return LT.DEEPWALK, float(c["length"])
+    if c["app"] == "pagerank":
+        return LT.PAGERANK, float(c["length"])
     return LT.PPR, float(c["alpha"])
 
 
+def init_walks(eng, c, starts, seed, first):
+    """lt_walks_init_ex, or lt_walks_init_pagerank for the random walk with restart."""
+    import paper_conf_icde_xing0wxl23_b200 as LT
+    app, param = app_param(c)
+    if app == LT.PAGERANK:
+        eng.walks_init_pagerank(starts, int(param), c["restart_p"], seed, first)
+    else:
+        eng.walks_init(starts, app, param, seed, first)
+
+
 def starts_for(c, g, W, first):
-    if c["app"] == "deepwalk":
+    if c["app"] in ("deepwalk", "pagerank"):
         return lt_inputs.deepwalk_starts(W, g.n, first_walk_id=first)
     return lt_inputs.ppr_starts(W, g.argmax_deg)
 
@@ -153,9 +177,9 @@ class Clocks:
 def oracle_sample(c, g_host, W, first, seconds, threads=0):
     """Time the oracle (as it stands) on a bounded prefix sample of the workload's walks."""
     import oracle as O
-    app = O.DEEPWALK if c["app"] == "deepwalk" else O.PPR
-    kw = dict(app=app, length=int(c.get("length", 0)), alpha=float(c.get("alpha", 0.15)), seed=c["seed"],
-              threads=threads)
+    app = {"deepwalk": O.DEEPWALK, "ppr": O.PPR, "pagerank": O.PAGERANK}[c["app"]]
+    alpha = float(c["restart_p"]) if c["app"] == "pagerank" else float(c.get("alpha", 0.15))
+    kw = dict(app=app, length=int(c.get("length", 0)), alpha=alpha, seed=c["seed"], threads=threads)
     # calibrate on a small prefix, then size the sample for ~`seconds` of work
     n0 = min(W, 200_000)
     st = starts_for(c, g_host, n0, first)
@@ -199,9 +223,11 @@ def cfg_json(c, g, W, extra):
     d = {"workload": f"{c['name']} (BASELINE.json configs[{c['idx'] - 1}])", "scale": c["scale"],
          "rmat_tuples": c["tuples"], "kronecker": bool(c["permute"]), "vertices": g.n, "csr_entries": g.m,
          "walks_per_gpu": W, "app": c["app"]}
-    if c["app"] == "deepwalk":
+    if c["app"] in ("deepwalk", "pagerank"):
         d["length"] = c["length"]
-    else:
+    if c["app"] == "pagerank":
+        d["restart_p"] = c["restart_p"]
+    if c["app"] == "ppr":
         d["alpha"] = c["alpha"]
     d.update(extra)
     return d
@@ -277,7 +303,8 @@ def main():
     starts_d = torch.from_numpy(starts_h.view(np.int32)).cuda(local)
 
     ooc = args.graph_pool_gb > 0
-    eng = LT.Engine(device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
+    vis = args.visit_counts == 1 or (args.visit_counts == -1 and c["app"] == "pagerank")
+    eng = LT.Engine(visit_counts=vis, device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill)
@@ -298,7 +325,7 @@ def main():
     superstep_counters = {}
 
     def one_step():
-        eng.walks_init(starts_d, app, param, args.seed, first)
+        init_walks(eng, c, starts_d, args.seed, first)
         if own:
             superstep_counters.update(ltdist.run_supersteps(eng, comm, f"cuda:{local}"))
         else:
@@ -336,7 +363,8 @@ def main():
     steps_k = steps_local
     finished = sum(s["num_walks"] for s in stats) if not own else len(stats) * W // world
     moves = max(0, visits - finished)  # a walk's final visit ends in termination, every other in a move
-    alg_bytes = steps_k * 104 + visits * 16 + moves * 16
+    # + one 32-B sector read-modify-write per path entry for the fused visit counts (when on)
+    alg_bytes = steps_k * (104 + (32 if vis else 0)) + visits * 16 + moves * 16
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
     if os.path.exists(peaks_path):
@@ -374,14 +402,14 @@ def main():
                        refill=args.refill) as e2:
             e2.graph_load(g.row_ptr, g.col, ps)
             for _ in range(2):
-                e2.walks_init(starts_d, app, param, args.seed, first)
+                init_walks(e2, c, starts_d, args.seed, first)
                 e2.run()
             torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record()
             sts = []
             for _ in range(3):
-                e2.walks_init(starts_d, app, param, args.seed, first)
+                init_walks(e2, c, starts_d, args.seed, first)
                 e2.run()
                 sts.append(e2.stats())
             b.record()
@@ -418,7 +446,26 @@ def main():
                      "hit_rate": last["pool_hits"] / max(1, last["iterations"])}
 
     e2e = None
-    if not args.no_e2e and args.e2e_steps > 0 and not own:
+    if not args.no_e2e and args.e2e_steps > 0 and not own and vis:
+        # the visit-frequency workload's result is the count vector: per step, pinned starts H2D
+        # (lt_walks_init_pagerank / _ex from host memory), the walk, and the u64[n] counts D2H
+        h_starts = torch.from_numpy(starts_h.view(np.int32)).pin_memory()
+        h_counts = torch.empty(g.n, dtype=torch.int64, pin_memory=True)
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        e_steps = 0
+        for _ in range(args.e2e_steps):
+            init_walks(eng, c, h_starts, args.seed, first)
+            eng.run()
+            eng.visit_counts(h_counts)
+            e_steps += eng.stats()["steps"]
+        b.record()
+        barrier()
+        e2e = {"value": e_steps / (a.elapsed_time(b) / 1000), "unit": "steps/s", "h2d_bytes_per_step": W * 4,
+               "d2h_bytes_per_step": g.n * 8, "pinned": True, "steps": args.e2e_steps,
+               "api": "lt_walks_init* (host starts) + lt_run + lt_get_visit_counts (host)"}
+    elif not args.no_e2e and args.e2e_steps > 0 and not own:
         S = int(c["length"]) + 1 if c["app"] == "deepwalk" else 128
         try:
             h_paths = torch.empty((W, S), dtype=torch.int32, pin_memory=True)
@@ -471,7 +518,7 @@ def main():
     cpu = None
     parity = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        eng.walks_init(starts_d, app, param, args.seed, first)
+        init_walks(eng, c, starts_d, args.seed, first)
         eng.run()
         gh = host_graph(g)
         r = oracle_sample(c, gh, W, first, args.cpu_seconds)
@@ -483,6 +530,13 @@ def main():
         ii = idx.astype(np.int64)
         mism = int(np.sum(np.any(gp != r["paths"][ii], axis=1) | (gl != r["lengths"][ii])))
         parity = {"sampled_walks": int(len(idx)), "mismatched_walks": mism, "vs": "oracle (bit-exact)"}
+        if vis:  # the counts are a global sum: check their total and one sampled property exactly
+            import oracle as O
+            cnt = eng.visit_counts().astype(np.int64)
+            parity["visit_counts_total"] = int(cnt.sum())
+            parity["visit_counts_total_ok"] = bool(cnt.sum() == eng.stats()["steps"] + W)
+            parity["visit_counts_of_sample_le_gpu"] = bool(np.all(
+                O.visit_counts(r["paths"], r["lengths"], g.n).astype(np.int64) <= cnt))
 
     last = stats[-1]
     if rank == 0:

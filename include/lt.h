@@ -52,7 +52,11 @@ typedef enum {
 
 typedef enum {
   LT_APP_DEEPWALK = 0, /* uniform sampling, fixed length l */
-  LT_APP_PPR = 1       /* personalized PageRank: stop with probability alpha per step */
+  LT_APP_PPR = 1,      /* personalized PageRank: stop with probability alpha per step */
+  LT_APP_PAGERANK = 2  /* PageRank / random walk with restart: fixed length l; at each step, with
+                          probability p, restart at a uniform random vertex instead of moving to a
+                          uniform neighbour (reading R23). Started with
+                          lt_walks_init_pagerank (it takes both l and p). */
 } lt_app;
 
 typedef enum {
@@ -109,7 +113,12 @@ typedef struct lt_config {
   uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
   uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P == 1, the measured
                                  best), 1 off, 2 on */
-  uint32_t reserved[1];
+  uint32_t visit_counts;      /* 1 -> count per-vertex visit frequency ("the visit
+                                 frequency of each vertex is recorded") into a u64[n] device array
+                                 reserved at lt_walks_init* and zeroed there: every path entry (start
+                                 included) adds 1 to its vertex. Read with lt_get_visit_counts*. The
+                                 kernels count in u32 while no count can reach 2^32 (W * stride <
+                                 2^32) and widen at the end of lt_run; 2 -> always count in u64. */
 } lt_config;
 
 typedef struct lt_stats {
@@ -178,6 +187,17 @@ lt_status lt_walks_init(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts,
 lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, int starts_on_device,
                            uint64_t first_walk_id, lt_app app, double length_or_alpha, uint64_t seed);
 
+/* PageRank / random walk with restart ("at each step, a walk has a probability p to
+ * restart at a random vertex, instead of uniformly selecting one of the neighbors"; reading R23):
+ * walk i (ID first_walk_id + i) starts at starts[i] and takes exactly `length` steps (l >= 0 integer;
+ * a dead end without a restart stops it early). At step t the PPR coin word x0 of blk(w,t,0) decides:
+ * x0 < floor(p 2^32) -> the next vertex is Lemire(n) over the step's word stream (a uniform vertex);
+ * otherwise a uniform neighbour as in DeepWalk. 0 < p < 1. Path stride l+1. Same ownership, errors and
+ * state rules as lt_walks_init_ex. Combine with lt_config.visit_counts for the visit-frequency
+ * estimate of PageRank (the paper's output for this application). */
+lt_status lt_walks_init_pagerank(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, int starts_on_device,
+                                 uint64_t first_walk_id, uint32_t length, double restart_p, uint64_t seed);
+
 /* Run the partition scheduler until every walk has terminated (a3-a7). Blocks the host. */
 lt_status lt_run(lt_ctx* ctx);
 
@@ -195,6 +215,13 @@ lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, u
 lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_lengths);
 
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out);
+
+/* Visit frequency (lt_config.visit_counts = 1): counts[v] = number of path entries equal
+ * to v over the walks of the last lt_walks_init* (on this rank: the starts it kept and the steps it
+ * took; the sum over ranks is the global count). counts is caller-owned u64[n], host (lt_get_visit_counts)
+ * or device (lt_get_visit_counts_device). LT_ERR_STATE before lt_run or when counting was off. */
+lt_status lt_get_visit_counts(lt_ctx* ctx, uint64_t* counts);
+lt_status lt_get_visit_counts_device(lt_ctx* ctx, uint64_t* d_counts);
 
 /* End-to-end sampling into HOST buffers with the copy-out overlapped: the same result as
  * lt_walks_init_ex(W, starts, host, first_walk_id, ...) + lt_run + lt_get_paths, computed in

@@ -56,6 +56,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
   if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
+  if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -121,6 +122,8 @@ void lt_destroy(lt_ctx* ctx) {
   }
   if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
   cudaFree(ctx->d_starts);
+  cudaFree(ctx->d_visits);
+  cudaFree(ctx->d_visits32);
   cudaFree(ctx->d_slots);
   cudaFree(ctx->d_ring);
   cudaFree(ctx->d_hc);
@@ -365,8 +368,23 @@ lt_status lt_walks_init(lt_ctx* ctx, uint64_t W, const uint32_t* starts, lt_app 
   return lt_walks_init_ex(ctx, W, starts, 0, 0, app, param, seed);
 }
 
+static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
+                                 uint64_t first_walk_id, lt_app app, double length_d, double alpha, uint64_t seed);
+
 lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device, uint64_t first_walk_id,
                            lt_app app, double param, uint64_t seed) {
+  if (app == LT_APP_PAGERANK) return fail(LT_ERR_INVALID, "PageRank takes a length and p: use lt_walks_init_pagerank");
+  if (app == LT_APP_DEEPWALK) return walks_init_impl(ctx, W, starts, on_device, first_walk_id, app, param, 0.0, seed);
+  return walks_init_impl(ctx, W, starts, on_device, first_walk_id, app, 0.0, param, seed);
+}
+
+lt_status lt_walks_init_pagerank(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
+                                 uint64_t first_walk_id, uint32_t length, double restart_p, uint64_t seed) {
+  return walks_init_impl(ctx, W, starts, on_device, first_walk_id, LT_APP_PAGERANK, (double)length, restart_p, seed);
+}
+
+static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
+                                 uint64_t first_walk_id, lt_app app, double length_d, double alpha, uint64_t seed) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_walks_init before lt_graph_load");
   if (W && !starts) return fail(LT_ERR_INVALID, "starts is NULL");
@@ -374,20 +392,23 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   CK(cudaSetDevice(ctx->cfg.device));
   uint32_t length = 0, T = 0, stride = 0;
   const uint32_t lmax = ctx->cfg.ppr_max_len;
-  if (app == LT_APP_DEEPWALK) {
-    if (!(param >= 0) || param != std::floor(param) || param > 1e6)
-      return fail(LT_ERR_INVALID, "DeepWalk length must be an integer in [0, 1e6]");
-    length = (uint32_t)param;
+  if (app == LT_APP_DEEPWALK || app == LT_APP_PAGERANK) {
+    if (!(length_d >= 0) || length_d != std::floor(length_d) || length_d > 1e6)
+      return fail(LT_ERR_INVALID, "walk length must be an integer in [0, 1e6]");
+    length = (uint32_t)length_d;
     stride = length + 1;
-  } else if (app == LT_APP_PPR) {
-    if (!(param > 0 && param < 1)) return fail(LT_ERR_INVALID, "PPR alpha must be in (0, 1)");
-    const double t = param * 4294967296.0;  // T = floor(alpha 2^32) (reading R5)
+  }
+  if (app == LT_APP_PPR || app == LT_APP_PAGERANK) {
+    if (!(alpha > 0 && alpha < 1))
+      return fail(LT_ERR_INVALID, "PPR alpha / PageRank restart probability must be in (0, 1)");
+    const double t = alpha * 4294967296.0;  // T = floor(alpha 2^32) (reading R5)
     T = (uint32_t)t;
-    stride = lmax + 1;
-  } else {
+    if (app == LT_APP_PPR) stride = lmax + 1;
+  } else if (app != LT_APP_DEEPWALK) {
     return fail(LT_ERR_INVALID, "unknown app");
   }
   ctx->walks_ready = false;
+  ctx->visits_ready = false;
   ctx->ran = false;
   ctx->stats.h2d_bytes = 0;
   ctx->stats.d2h_bytes = 0;
@@ -416,6 +437,10 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
   CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
   CK(ensure(ctx->d_free, ctx->free_cap, num_chunks));
+  // visit counters: u32 while no count can reach 2^32 (at most W * stride path entries in total)
+  const bool narrow = ctx->cfg.visit_counts == 1 && (uint64_t)W * stride < 0xFFFFFFFFull;
+  if (ctx->cfg.visit_counts) CK(ensure(ctx->d_visits, ctx->visits_cap, ctx->n));
+  if (narrow) CK(ensure(ctx->d_visits32, ctx->visits32_cap, ctx->n));
   if (on_device && W) {
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
     CK(lt::launch_check_starts(d_starts, W, ctx->n, ctx->d_small + 2, s));
@@ -444,6 +469,9 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   p.wk.length = length;
   p.wk.T = T;
   p.wk.lmax = lmax;
+  p.wk.n = ctx->n;
+  p.wk.visits = ctx->cfg.visit_counts ? ctx->d_visits : nullptr;
+  p.wk.visits32 = narrow ? ctx->d_visits32 : nullptr;
   p.pool.slots = ctx->d_slots;
   p.pool.C = (uint32_t)C;
   p.pool.c_shift = c_shift;
@@ -486,6 +514,8 @@ lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int 
   CK(lt::launch_pool_reset(p, s));
   ctx->stats.kernel_launches++;
   if (W) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
+  if (narrow) CK(cudaMemsetAsync(ctx->d_visits32, 0, (size_t)ctx->n * sizeof(uint32_t), s));
+  else if (ctx->cfg.visit_counts) CK(cudaMemsetAsync(ctx->d_visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
   if (W && ctx->world > 1) CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
@@ -529,6 +559,10 @@ lt_status lt_run(lt_ctx* ctx) {
     CK(lt::launch_finalize_paths(ctx->params, ctx->W, s));
     ctx->stats.kernel_launches++;
   }
+  if (ctx->params.wk.visits32) {  // the result is u64[n]
+    CK(lt::launch_widen(ctx->params.wk.visits32, ctx->params.wk.visits, ctx->n, s));
+    ctx->stats.kernel_launches++;
+  }
   CK(cudaEventRecord(ctx->ev_b, s));
   st = lt::snapshot(ctx);
   if (st != LT_OK) return st;
@@ -547,6 +581,7 @@ lt_status lt_run(lt_ctx* ctx) {
   ctx->stats.visits = ctx->h_ctr->visits;
   ctx->stats.truncated = ctx->h_ctr->truncated;
   ctx->ran = true;
+  ctx->visits_ready = ctx->cfg.visit_counts != 0;
   if (ctx->h_ctr->err & lt::kErrOOM) return fail(LT_ERR_CUDA, "walk pool exhausted on the device (invariant violated)");
   if (ctx->h_ctr->err) return fail(LT_ERR_CUDA, "device invariant violated (ring slot reinstalled)");
   return LT_OK;
@@ -705,6 +740,7 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
   if (ctx->world != 1) return fail(LT_ERR_INVALID, "lt_run_to_host needs a single-rank context");
   if (W && (!starts || !paths || !lengths)) return fail(LT_ERR_INVALID, "NULL argument");
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_run_to_host before lt_graph_load");
+  if (ctx->cfg.visit_counts) return fail(LT_ERR_INVALID, "lt_run_to_host does not accumulate visit counts; use lt_run");
   CK(cudaSetDevice(ctx->cfg.device));
   if (chunks == 0) chunks = 8;
   const uint64_t wc = std::max<uint64_t>((W + chunks - 1) / chunks, 1);
@@ -785,6 +821,23 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
   ctx->stats.h2d_bytes = h2d;
   ctx->stats.d2h_bytes = d2h;
   return LT_OK;
+}
+
+static lt_status copy_visits(lt_ctx* ctx, uint64_t* counts, cudaMemcpyKind kind) {
+  if (!ctx || !counts) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->cfg.visit_counts) return fail(LT_ERR_STATE, "visit counting is off (lt_config.visit_counts)");
+  if (!ctx->visits_ready) return fail(LT_ERR_STATE, "visit counts requested before lt_run");
+  CK(cudaSetDevice(ctx->cfg.device));
+  CK(cudaMemcpyAsync(counts, ctx->d_visits, (size_t)ctx->n * sizeof(uint64_t), kind, ctx->stream));
+  if (kind == cudaMemcpyDeviceToHost) ctx->stats.d2h_bytes += (uint64_t)ctx->n * 8;
+  CK(cudaStreamSynchronize(ctx->stream));
+  return LT_OK;
+}
+
+lt_status lt_get_visit_counts(lt_ctx* ctx, uint64_t* counts) { return copy_visits(ctx, counts, cudaMemcpyDeviceToHost); }
+
+lt_status lt_get_visit_counts_device(lt_ctx* ctx, uint64_t* d_counts) {
+  return copy_visits(ctx, d_counts, cudaMemcpyDeviceToDevice);
 }
 
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out) {

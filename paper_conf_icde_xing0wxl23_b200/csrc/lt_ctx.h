@@ -77,6 +77,11 @@ struct lt_ctx {
   size_t paths_cap = 0;
   uint32_t* d_lengths = nullptr;
   size_t lengths_cap = 0;
+  unsigned long long* d_visits = nullptr;  // [n] visit counts (cfg.visit_counts)
+  size_t visits_cap = 0;
+  uint32_t* d_visits32 = nullptr;          // [n] narrow counters (while counts fit in u32)
+  size_t visits32_cap = 0;
+  bool visits_ready = false;
   uint32_t* d_starts = nullptr;
   size_t starts_cap = 0;
   // pool

@@ -50,7 +50,11 @@ struct Walk {
   uint32_t* lengths;
   uint64_t first_walk_id;
   uint32_t seed_lo, seed_hi;
-  uint32_t app, length, T, lmax;
+  uint32_t app, length, T, lmax;  // app: 0 DeepWalk, 1 PPR, 2 PageRank (random walk with restart)
+  uint32_t n;                     // |V|: a PageRank restart draws its vertex from [0, n)
+  unsigned long long* visits;     // [n] per-vertex visit counts or nullptr (off)
+  uint32_t* visits32;             // [n] narrow counters used instead while every count fits in u32
+                                  // (W * stride < 2^32); widened into `visits` at the end of lt_run
 };
 
 struct Counters {
@@ -93,6 +97,7 @@ cudaError_t launch_compact_rows(const uint32_t* paths, uint64_t pitch, uint64_t 
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
+cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
                              cudaStream_t s);
 int update_kernel_occupancy(uint32_t block, uint32_t ilp);  // resident blocks per SM (update kernel)

@@ -216,6 +216,8 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
       have = dest >= p.own.own_lo && dest < p.own.own_hi;
       if (have) {
         wk.paths[i * wk.pitch] = v;
+        if (wk.visits32) atomicAdd(wk.visits32 + v, 1u);  // the start is the walk's first visit
+        else if (wk.visits) atomicAdd(wk.visits + v, 1ull);
         rec = make_uint4((uint32_t)i, v, 0u, 0u);
       }
     }
@@ -274,6 +276,25 @@ __device__ __forceinline__ Policies make_policies() {
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p.first));
   return p;
 }
+
+// Path-entry stores: every path sector is written once and never read back
+// by the walk; LT_PATH_HINT=1 sends it to L2 with the evict_first policy so it does not push out the
+// lines the step re-reads (row_ptr of hot vertices, bucket tails, visit counters). Off by default.
+#ifndef LT_PATH_HINT
+#define LT_PATH_HINT 0  // measured: evict_first path stores cost DeepWalk 2 % (67.4 vs 66.0 ms), gain PageRank < 1 %
+#endif
+__device__ __forceinline__ void st_sector(uint32_t* dst, const uint32_t* v, const Policies& pol) {
+#if LT_PATH_HINT
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;"
+               :: "l"(dst), "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "l"(pol.first) : "memory");
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;"
+               :: "l"(dst + 4), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "l"(pol.first) : "memory");
+#else
+  uint4* d = reinterpret_cast<uint4*>(dst);
+  d[0] = make_uint4(v[0], v[1], v[2], v[3]);
+  d[1] = make_uint4(v[4], v[5], v[6], v[7]);
+#endif
+}
 template <int GM>
 __device__ __forceinline__ uint32_t ld_col(const uint32_t* p, const Policies& pol) {
   if (GM == 0) return __ldg(p);
@@ -303,7 +324,36 @@ template <int ILP> struct MinBlocks { static constexpr int v = 4; };
 template <> struct MinBlocks<2> { static constexpr int v = 3; };
 template <> struct MinBlocks<4> { static constexpr int v = 2; };
 
-template <int APP, int GM, int ILP, int LAY>
+// VIS: fused per-vertex visit counting (lt_config.visit_counts) compiled out (0), with u64 counters
+// (1), or with u32 counters (2, while every count fits): the default kernels carry no trace of it.
+// The add is a fire-and-forget RED to the vertex's counter, resolved in L2.
+// The counters carry an L2 evict_last policy: they are the only lines of the step that are re-read
+// at random (visits are degree-skewed, so the hot counters stay resident).
+#ifndef LT_VIS_HINT
+#define LT_VIS_HINT 1
+#endif
+template <int VIS>
+__device__ __forceinline__ void count_visit(const Walk& wk, uint32_t v, uint64_t pol_last) {
+#if LT_VIS_HINT
+  if (VIS == 1)
+    asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u64 [%0], 1, %1;" :: "l"(wk.visits + v), "l"(pol_last)
+                 : "memory");
+  if (VIS == 2)
+    asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], 1, %1;" :: "l"(wk.visits32 + v), "l"(pol_last)
+                 : "memory");
+#else
+  (void)pol_last;
+  if (VIS == 1) atomicAdd(wk.visits + v, 1ull);
+  if (VIS == 2) atomicAdd(wk.visits32 + v, 1u);
+#endif
+}
+__device__ __forceinline__ uint64_t make_evict_last() {
+  uint64_t p = 0;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
+template <int APP, int GM, int ILP, int LAY, int VIS>
 __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
@@ -317,6 +367,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
   const Policies pol = make_policies();
+  const uint64_t pol_last = VIS ? make_evict_last() : 0;
   unsigned long long my_steps = 0, my_trunc = 0;
 
   for (unsigned long long base = head + ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * (32 * ILP);
@@ -360,7 +411,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
 #pragma unroll
       for (int s = 0; s < ILP; ++s) {
         if (alive[s]) {
-          if (APP == 0) {
+          if (APP != 1) {  // DeepWalk and PageRank: fixed length l
             if (rec[s].z == wk.length) alive[s] = false;
           } else if (rec[s].z == wk.lmax) {
             trunc[s] = true;
@@ -393,15 +444,23 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
       for (int s = 0; s < ILP; ++s) {
         nv[s] = 0;
         if (APP == 1 && alive[s] && b[s].x < wk.T) alive[s] = false;  // terminate before moving
-        if (alive[s] && d[s] == 0) alive[s] = false;                   // dead end
+        const bool restart = APP == 2 && alive[s] && b[s].x < wk.T;    // PageRank: jump to a uniform vertex
+        if (alive[s] && !restart && d[s] == 0) alive[s] = false;        // dead end
         if (alive[s]) {
-          const uint64_t m = (uint64_t)b[s].y * d[s];
+          const uint32_t dd = restart ? wk.n : d[s];  // the draw ranges over [0, n) on a restart
+          const uint64_t m = (uint64_t)b[s].y * dd;
           const uint64_t wid = wk.first_walk_id + rec[s].x;
-          const uint32_t idx = ((uint32_t)m < d[s])
-                                   ? lemire_slow(d[s], b[s], rec[s].z, (uint32_t)wid, (uint32_t)(wid >> 32),
+          const uint32_t idx = ((uint32_t)m < dd)
+                                   ? lemire_slow(dd, b[s], rec[s].z, (uint32_t)wid, (uint32_t)(wid >> 32),
                                                  wk.seed_lo, wk.seed_hi)
                                    : (uint32_t)(m >> 32);
-          if (LAY == 0) {
+          if (restart) {
+            nv[s] = idx;
+            if (LAY == 1 && idx - lo < span) {  // staying: the next step needs its offset and degree
+              off[s] = __ldg(wk.row_ptr + idx);
+              d[s] = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off[s]);
+            }
+          } else if (LAY == 0) {
             nv[s] = ld_col<GM>(wk.col + off[s] + idx, pol);
           } else {
             const uint4 e = ld_adj<GM>(wk.adj + off[s] + idx, pol);
@@ -416,6 +475,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
         if (alive[s]) {
           rec[s].y = nv[s];
           rec[s].z += 1;
+          count_visit<VIS>(wk, nv[s], pol_last);
           const uint32_t t = rec[s].z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -424,9 +484,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
             nb[s] += 1;
             if ((t & 7u) == 7u) {  // entry t closes sector [t-7, t]
               if (nb[s] == 8) {
-                uint4* dst = reinterpret_cast<uint4*>(prow[s] + (t - 7));
-                dst[0] = make_uint4(pb[s][0], pb[s][1], pb[s][2], pb[s][3]);
-                dst[1] = make_uint4(pb[s][4], pb[s][5], pb[s][6], pb[s][7]);
+                st_sector(prow[s] + (t - 7), pb[s], pol);
               } else {
 #pragma unroll
                 for (int q = 0; q < 8; ++q)
@@ -494,7 +552,7 @@ __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, c
   __syncwarp();
 }
 
-template <int APP, int GM, int LAY>
+template <int APP, int GM, int LAY, int VIS>
 __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
@@ -508,6 +566,7 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
   const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
   unsigned long long* claim = pl.claim + k;
   const Policies pol = make_policies();
+  const uint64_t pol_last = VIS ? make_evict_last() : 0;
   unsigned long long my_steps = 0, my_trunc = 0;
 
   bool has = false;
@@ -560,7 +619,7 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
     // ---- one step of every lane that holds a walk
     bool done = false, left = false, trunc = false;
     if (has) {
-      if (APP == 0 && rec.z == wk.length) {
+      if (APP != 1 && rec.z == wk.length) {
         done = true;
       } else if (APP == 1 && rec.z == wk.lmax) {
         done = true;
@@ -573,15 +632,23 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
         }
         const uint64_t wid = wk.first_walk_id + rec.x;
         const uint4 b = philox10(make_uint4(rec.z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
-        if ((APP == 1 && b.x < wk.T) || d == 0) {
+        const bool restart = APP == 2 && b.x < wk.T;  // PageRank: jump to a uniform vertex
+        if ((APP == 1 && b.x < wk.T) || (d == 0 && !restart)) {
           done = true;
         } else {
-          const uint64_t m = (uint64_t)b.y * d;
-          const uint32_t idx = ((uint32_t)m < d) ? lemire_slow(d, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
-                                                              wk.seed_lo, wk.seed_hi)
-                                                 : (uint32_t)(m >> 32);
+          const uint32_t dd = restart ? wk.n : d;
+          const uint64_t m = (uint64_t)b.y * dd;
+          const uint32_t idx = ((uint32_t)m < dd) ? lemire_slow(dd, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
+                                                               wk.seed_lo, wk.seed_hi)
+                                                  : (uint32_t)(m >> 32);
           uint32_t nv;
-          if (LAY == 0) {
+          if (restart) {
+            nv = idx;
+            if (LAY == 1 && idx - lo < span) {
+              off = __ldg(wk.row_ptr + idx);
+              d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
+            }
+          } else if (LAY == 0) {
             nv = ld_col<GM>(wk.col + off + idx, pol);
           } else {
             const uint4 e = ld_adj<GM>(wk.adj + off + idx, pol);
@@ -591,6 +658,7 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
           }
           rec.y = nv;
           rec.z += 1;
+          count_visit<VIS>(wk, nv, pol_last);
           const uint32_t t = rec.z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -599,9 +667,7 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
             nb += 1;
             if ((t & 7u) == 7u) {
               if (nb == 8) {
-                uint4* dst = reinterpret_cast<uint4*>(prow + (t - 7));
-                dst[0] = make_uint4(pb[0], pb[1], pb[2], pb[3]);
-                dst[1] = make_uint4(pb[4], pb[5], pb[6], pb[7]);
+                st_sector(prow + (t - 7), pb, pol);
               } else {
 #pragma unroll
                 for (int q = 0; q < 8; ++q)
@@ -752,9 +818,9 @@ uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 
 int update_kernel_occupancy(uint32_t block, uint32_t ilp) {
   int nb = 0;
-  if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1>, (int)block, 0);
-  else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1>, (int)block, 0);
-  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1>, (int)block, 0);
+  if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
+  else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1, 0>, (int)block, 0);
+  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1, 0>, (int)block, 0);
   return nb > 0 ? nb : 1;
 }
 
@@ -801,55 +867,64 @@ cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cud
   return cudaGetLastError();
 }
 
-template <int APP, int GM, int ILP, int LAY>
+template <int APP, int GM, int ILP, int LAY, int VIS>
 void launch_update_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_update<APP, GM, ILP, LAY>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_update<APP, GM, ILP, LAY, VIS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          kSmemBoundsCap * 4);
     attr = true;
   }
-  k_update<APP, GM, ILP, LAY><<<grid, block, bounds_smem(p), s>>>(p, k);
+  k_update<APP, GM, ILP, LAY, VIS><<<grid, block, bounds_smem(p), s>>>(p, k);
 }
 
-template <int APP, int GM, int LAY>
+template <int APP, int GM, int LAY, int VIS>
 void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_update_rf<APP, GM, LAY>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
+    cudaFuncSetAttribute(k_update_rf<APP, GM, LAY, VIS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         kSmemBoundsCap * 4);
     attr = true;
   }
-  k_update_rf<APP, GM, LAY><<<grid, block, bounds_smem(p), s>>>(p, k);
+  k_update_rf<APP, GM, LAY, VIS><<<grid, block, bounds_smem(p), s>>>(p, k);
 }
 
-template <int APP, int GM, int LAY>
+template <int APP, int GM, int LAY, int VIS>
 void launch_update_ilp(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   if (p.refill) {
-    launch_update_rf<APP, GM, LAY>(p, k, grid, block, s);
+    launch_update_rf<APP, GM, LAY, VIS>(p, k, grid, block, s);
     return;
   }
   switch (p.ilp) {
-    case 1: launch_update_t<APP, GM, 1, LAY>(p, k, grid, block, s); break;
-    case 4: launch_update_t<APP, GM, 4, LAY>(p, k, grid, block, s); break;
-    default: launch_update_t<APP, GM, 2, LAY>(p, k, grid, block, s); break;
+    case 1: launch_update_t<APP, GM, 1, LAY, VIS>(p, k, grid, block, s); break;
+    case 4: launch_update_t<APP, GM, 4, LAY, VIS>(p, k, grid, block, s); break;
+    default: launch_update_t<APP, GM, 2, LAY, VIS>(p, k, grid, block, s); break;
   }
 }
 
-template <int APP>
+template <int APP, int VIS>
 void launch_update_app(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   const bool adj = p.wk.adj != nullptr;
   if (p.gather_mode == 0) {
-    if (adj) launch_update_ilp<APP, 0, 1>(p, k, grid, block, s);
-    else launch_update_ilp<APP, 0, 0>(p, k, grid, block, s);
+    if (adj) launch_update_ilp<APP, 0, 1, VIS>(p, k, grid, block, s);
+    else launch_update_ilp<APP, 0, 0, VIS>(p, k, grid, block, s);
   } else {
-    if (adj) launch_update_ilp<APP, 3, 1>(p, k, grid, block, s);
-    else launch_update_ilp<APP, 3, 0>(p, k, grid, block, s);
+    if (adj) launch_update_ilp<APP, 3, 1, VIS>(p, k, grid, block, s);
+    else launch_update_ilp<APP, 3, 0, VIS>(p, k, grid, block, s);
   }
 }
 
+template <int VIS>
+void launch_update_vis(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  if (p.wk.app == 0) launch_update_app<0, VIS>(p, k, grid, block, s);
+  else if (p.wk.app == 1) launch_update_app<1, VIS>(p, k, grid, block, s);
+  else launch_update_app<2, VIS>(p, k, grid, block, s);
+}
+
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  if (p.wk.app == 0) launch_update_app<0>(p, k, grid, block, s);
-  else launch_update_app<1>(p, k, grid, block, s);
+  if (p.wk.visits32) launch_update_vis<2>(p, k, grid, block, s);
+  else if (p.wk.visits) launch_update_vis<1>(p, k, grid, block, s);
+  else launch_update_vis<0>(p, k, grid, block, s);
   return cudaGetLastError();
 }
 
@@ -890,6 +965,17 @@ cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s) {
   if (!W) return cudaSuccess;
   k_check_range<<<num_sms() * 4, 256, 0, s>>>(starts, W, n, bad);
+  return cudaGetLastError();
+}
+
+__global__ void k_widen(const uint32_t* __restrict__ src, unsigned long long* __restrict__ dst, uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    dst[i] = src[i];
+}
+
+cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_widen<<<num_sms() * 8, 256, 0, s>>>(src, dst, n);
   return cudaGetLastError();
 }
 

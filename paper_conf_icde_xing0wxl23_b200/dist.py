@@ -55,7 +55,8 @@ class TorchComm:
         return int(t.item())
 
     def allreduce_(self, t, op: str):
-        self.dist.all_reduce(t, op={"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX}[op], group=self.group)
+        ops = {"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM}
+        self.dist.all_reduce(t, op=ops[op], group=self.group)
 
 
 class ThreadComm:
@@ -102,7 +103,7 @@ class ThreadComm:
         acc = allv[0].to(t.device)
         for o in allv[1:]:
             o = o.to(t.device)
-            acc = (acc.minimum(o) if op == "min" else acc.maximum(o))
+            acc = acc.minimum(o) if op == "min" else acc.maximum(o) if op == "max" else acc + o
         t.copy_(acc)
 
 
@@ -147,3 +148,13 @@ def merge_paths(engine, comm):
     paths ^= SIGN
     comm.allreduce_(lengths, "max")
     return paths, lengths
+
+
+def merge_visit_counts(engine, comm, device):
+    """Global per-vertex visit frequency: each rank counted the starts it kept and the
+    steps it took, so the global count is the sum over ranks. Returns an int64 tensor [n] (u64 bits)."""
+    import torch
+    counts = torch.empty(engine.n, dtype=torch.int64, device=device)
+    engine.visit_counts(counts)
+    comm.allreduce_(counts, "sum")
+    return counts

@@ -22,7 +22,7 @@ if not os.path.exists(LIB_PATH):
 _lib = ctypes.CDLL(LIB_PATH)
 
 LT_OK, LT_ERR_INVALID, LT_ERR_STATE, LT_ERR_OOM, LT_ERR_CUDA, LT_ERR_NCCL = range(6)
-DEEPWALK, PPR = 0, 1
+DEEPWALK, PPR, PAGERANK = 0, 1, 2
 POLICY_SELECTIVE, POLICY_ROUND_ROBIN, POLICY_SELECTIVE_ONLY, POLICY_PREEMPTIVE_ONLY = 0, 1, 2, 3
 INSERT_WARP_AGGREGATED, INSERT_DIRECT = 0, 1
 LAYOUT_AUTO, LAYOUT_CSR, LAYOUT_ADJ = 0, 1, 2
@@ -32,7 +32,8 @@ EXPORTED = [
     "lt_config_default", "lt_create", "lt_destroy", "lt_last_error", "lt_partition_bounds", "lt_graph_load",
     "lt_graph_load_device", "lt_get_bounds", "lt_walks_init", "lt_walks_init_ex", "lt_run", "lt_path_stride",
     "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
-    "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host",
+    "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
+    "lt_get_visit_counts", "lt_get_visit_counts_device",
 ]
 
 
@@ -59,7 +60,7 @@ class Config(ctypes.Structure):
         ("rank", ctypes.c_uint32),
         ("world", ctypes.c_uint32),
         ("refill", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 1),
+        ("visit_counts", ctypes.c_uint32),
     ]
 
 
@@ -93,6 +94,9 @@ _lib.lt_graph_load_device.argtypes = [_vp, _u32, _u64, _vp, _vp, _u32]
 _lib.lt_get_bounds.argtypes = [_vp, _vp, ctypes.POINTER(_u32)]
 _lib.lt_walks_init.argtypes = [_vp, _u64, _vp, ctypes.c_int, ctypes.c_double, _u64]
 _lib.lt_walks_init_ex.argtypes = [_vp, _u64, _vp, ctypes.c_int, _u64, ctypes.c_int, ctypes.c_double, _u64]
+_lib.lt_walks_init_pagerank.argtypes = [_vp, _u64, _vp, ctypes.c_int, _u64, _u32, ctypes.c_double, _u64]
+_lib.lt_get_visit_counts.argtypes = [_vp, _vp]
+_lib.lt_get_visit_counts_device.argtypes = [_vp, _vp]
 _lib.lt_run.argtypes = [_vp]
 _lib.lt_path_stride.argtypes = [_vp, ctypes.POINTER(_u32)]
 _lib.lt_get_paths.argtypes = [_vp, _vp, _vp]
@@ -158,7 +162,8 @@ class Engine:
                  timing: bool = False, stream=None, blocks_per_sm: int = 0, l2_fetch_bytes: int = 0,
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
-                 zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0):
+                 zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
+                 visit_counts: bool = False):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -180,6 +185,7 @@ class Engine:
         cfg.rank = rank
         cfg.world = world
         cfg.refill = refill
+        cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device
         h = _vp()
@@ -234,6 +240,23 @@ class Engine:
         _check(_lib.lt_walks_init_ex(self._h, W, p, int(dev), first_walk_id, app, float(param), seed))
         self._starts_keep = keep
         self.num_walks = W
+
+    def walks_init_pagerank(self, starts, length: int, restart_p: float, seed: int = 1, first_walk_id: int = 0):
+        """PageRank / random walk with restart (lt_walks_init_pagerank)."""
+        p, dev, keep = _ptr(starts, np.uint32)
+        W = keep.numel() if _is_torch(keep) else len(keep)
+        _check(_lib.lt_walks_init_pagerank(self._h, W, p, int(dev), first_walk_id, int(length), float(restart_p), seed))
+        self._starts_keep = keep
+        self.num_walks = W
+
+    def visit_counts(self, out=None):
+        """Per-vertex visit frequency u64[n] (lt_get_visit_counts; needs visit_counts=True). `out` may be a
+        host array or a CUDA int64 tensor (device copy)."""
+        if out is None:
+            out = np.zeros(self.n, dtype=np.uint64)
+        p, dev, keep = _ptr(out, np.uint64)
+        _check((_lib.lt_get_visit_counts_device if dev else _lib.lt_get_visit_counts)(self._h, p))
+        return out
 
     def run(self):
         _check(_lib.lt_run(self._h))

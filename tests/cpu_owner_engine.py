@@ -31,10 +31,21 @@ class CpuOwnerEngine:
         return q if self.own_lo <= q < self.own_hi else self.P + int(self.owner[q])
 
     def walks_init(self, starts, app, param, seed, lmax=127):
-        W = len(starts)
         self.app, self.param, self.seed, self.lmax = app, param, seed, lmax
         self.T = O.ppr_threshold(param) if app == LT.PPR else 0
         self.stride = int(param) + 1 if app == LT.DEEPWALK else lmax + 1
+        self._init(starts)
+
+    def walks_init_pagerank(self, starts, length, restart_p, seed):
+        self.app, self.param, self.seed, self.lmax = LT.PAGERANK, length, seed, 127
+        self.T = O.ppr_threshold(restart_p)
+        self.stride = int(length) + 1
+        self._init(starts)
+
+    def _init(self, starts):
+        W = len(starts)
+        self.n = self.g.n
+        self.counts = np.zeros(self.g.n, dtype=np.uint64)
         self.num_walks = W
         self.paths = np.full((W, self.stride), EMPTY, dtype=np.uint32)
         self.lengths = np.zeros(W, dtype=np.uint32)
@@ -43,13 +54,14 @@ class CpuOwnerEngine:
             q = self._part(int(starts[w]))
             if self.own_lo <= q < self.own_hi:
                 self.paths[w, 0] = starts[w]
+                self.counts[int(starts[w])] += 1
                 self.buckets[q].append((w, int(starts[w]), 0))
 
     def _visit(self, rec, lo, hi):
         w, v, t = rec
         rp, col = self.g.row_ptr, self.g.col
         while True:
-            if self.app == LT.DEEPWALK and t == int(self.param):
+            if self.app in (LT.DEEPWALK, LT.PAGERANK) and t == int(self.param):
                 break
             if self.app == LT.PPR and t == self.lmax:
                 break
@@ -57,13 +69,21 @@ class CpuOwnerEngine:
                 x0 = O.philox4x32_10([t, 0, w & 0xFFFFFFFF, w >> 32], [self.seed & 0xFFFFFFFF, self.seed >> 32])[0]
                 if x0 < self.T:
                     break
+            restart = False
+            if self.app == LT.PAGERANK:
+                x0 = O.philox4x32_10([t, 0, w & 0xFFFFFFFF, w >> 32], [self.seed & 0xFFFFFFFF, self.seed >> 32])[0]
+                restart = x0 < self.T
             d = int(rp[v + 1] - rp[v])
-            if d == 0:
-                break
-            idx, _ = O.lemire(self.seed, w, t, d)
-            v = int(col[int(rp[v]) + idx])
+            if restart:
+                v, _ = O.lemire(self.seed, w, t, self.g.n)
+            else:
+                if d == 0:
+                    break
+                idx, _ = O.lemire(self.seed, w, t, d)
+                v = int(col[int(rp[v]) + idx])
             t += 1
             self.paths[w, t] = v
+            self.counts[v] += 1
             if not (lo <= v < hi):
                 return (w, v, t)
         self.lengths[w] = t + 1
@@ -104,6 +124,11 @@ class CpuOwnerEngine:
         arr = recv[:count].numpy().view(np.uint32)
         for w, v, t, _ in arr:
             self.buckets[self._bucket(self._part(int(v)))].append((int(w), int(v), int(t)))
+
+    def visit_counts(self, out):
+        import torch
+        out.copy_(torch.from_numpy(self.counts.view(np.int64)))
+        return out
 
     def partial_paths(self):
         import torch

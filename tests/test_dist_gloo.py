@@ -36,20 +36,25 @@ def _worker(rank, world, port, app, param, P, out_q):
     try:
         g = lt_inputs.rmat_cpu(9, 3000, seed=5)
         W = 700
-        starts = lt_inputs.deepwalk_starts(W, g.n) if app == LT.DEEPWALK else lt_inputs.ppr_starts(W, g.argmax_deg)
+        starts = lt_inputs.ppr_starts(W, g.argmax_deg) if app == LT.PPR else lt_inputs.deepwalk_starts(W, g.n)
         eng = CpuOwnerEngine(g, P, rank, world)
-        eng.walks_init(starts, app, param, 11)
+        if app == LT.PAGERANK:
+            eng.walks_init_pagerank(starts, 12, param, 11)
+        else:
+            eng.walks_init(starts, app, param, 11)
         comm = ltdist.TorchComm()
         counters = ltdist.run_supersteps(eng, comm, "cpu")
         paths, lengths = ltdist.merge_paths(eng, comm)
+        counts = ltdist.merge_visit_counts(eng, comm, "cpu")
         if rank == 0:
-            out_q.put((paths.numpy().view(np.uint32).copy(), lengths.numpy().view(np.uint32).copy(), counters))
+            out_q.put((paths.numpy().view(np.uint32).copy(), lengths.numpy().view(np.uint32).copy(), counters,
+                       counts.numpy().view(np.uint64).copy()))
     finally:
         dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("world", [2, 3])
-@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 12), (LT.PPR, 0.2)])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 12), (LT.PPR, 0.2), (LT.PAGERANK, 0.3)])
 def test_ownership_protocol_gloo(world, app, param):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -58,15 +63,17 @@ def test_ownership_protocol_gloo(world, app, param):
     procs = [ctx.Process(target=_worker, args=(r, world, port, app, param, P, q)) for r in range(world)]
     for p in procs:
         p.start()
-    paths, lengths, counters = q.get(timeout=300)
+    paths, lengths, counters, counts = q.get(timeout=300)
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
     g = lt_inputs.rmat_cpu(9, 3000, seed=5)
     W = 700
-    starts = lt_inputs.deepwalk_starts(W, g.n) if app == LT.DEEPWALK else lt_inputs.ppr_starts(W, g.argmax_deg)
-    kw = dict(app=O.DEEPWALK, length=12) if app == LT.DEEPWALK else dict(app=O.PPR, alpha=0.2)
+    starts = lt_inputs.ppr_starts(W, g.argmax_deg) if app == LT.PPR else lt_inputs.deepwalk_starts(W, g.n)
+    kw = {LT.DEEPWALK: dict(app=O.DEEPWALK, length=12), LT.PPR: dict(app=O.PPR, alpha=0.2),
+          LT.PAGERANK: dict(app=O.PAGERANK, length=12, alpha=0.3)}[app]
     op, ol, _, _ = O.walks(g.row_ptr, g.col, starts, seed=11, **kw)
     np.testing.assert_array_equal(lengths, ol)
     np.testing.assert_array_equal(paths, op)
+    np.testing.assert_array_equal(counts, O.visit_counts(op, ol, g.n))  # summed over ranks
     assert counters["supersteps"] >= 2 and counters["records_sent"] > 0

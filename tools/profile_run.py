@@ -30,6 +30,8 @@ def main():
     ap.add_argument("--layout", type=int, default=0)
     ap.add_argument("--path-mode", type=int, default=0)
     ap.add_argument("--refill", type=int, default=0)
+    ap.add_argument("--app", default="config", choices=["config", "pagerank"])
+    ap.add_argument("--restart-p", type=float, default=0.15)
     a = ap.parse_args()
     import torch
 
@@ -50,10 +52,13 @@ def main():
     with LT.Engine(chunk_walks=a.chunk_walks, l2_fetch_bytes=a.l2_fetch, timing=True,
                    gather_mode=a.gather_mode, ilp=a.ilp, blocks_per_sm=a.blocks_per_sm,
                    layout=a.layout, path_mode=a.path_mode,
-                   refill=a.refill) as e:
+                   refill=a.refill, visit_counts=a.app == "pagerank") as e:
         e.graph_load(g.row_ptr, g.col, a.partitions)
         for _ in range(a.steps):
-            e.walks_init(sd, app, prm, 1)
+            if a.app == "pagerank":  # random walk with restart + visit counts
+                e.walks_init_pagerank(sd, int(c.get("length", 80)), a.restart_p, 1)
+            else:
+                e.walks_init(sd, app, prm, 1)
             e.run()
         s = e.stats()
     torch.cuda.synchronize()
