@@ -174,8 +174,12 @@ class Clocks:
 
 
 # ------------------------------------------------------------------------------ CPU oracle legs
-def oracle_sample(c, g_host, W, first, seconds, threads=0):
-    """Time the oracle (as it stands) on a bounded prefix sample of the workload's walks."""
+def oracle_sample(c, g_host, W, first, seconds, threads=None):
+    """Time the oracle (as it stands) on a bounded prefix sample of the workload's walks, with one
+    OpenMP thread per host core this process may use (explicitly: torchrun exports
+    OMP_NUM_THREADS=1, which would otherwise leave the oracle on one core)."""
+    if threads is None:
+        threads = cores()
     import oracle as O
     app = {"deepwalk": O.DEEPWALK, "ppr": O.PPR, "pagerank": O.PAGERANK}[c["app"]]
     alpha = float(c["restart_p"]) if c["app"] == "pagerank" else float(c.get("alpha", 0.15))
@@ -264,7 +268,7 @@ def run_reference(args):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic", "config": cfg_json(c, g, W, {"partitions": None}),
             "cpu_baseline": {"value": value, "unit": "steps/s", "cores": cores(), "kind": "oracle",
-                             "sample": f"walks 0..{ns - 1} of the workload per step (oracle/ C + OpenMP)"},
+                             "sample": f"walks 0..{ns - 1} of the workload per step (oracle/ C + OpenMP, {cores()} threads)"},
             "e2e": {"value": value, "unit": "steps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -283,9 +287,17 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # LT_BENCH_SHARE_DEVICE=1 (tests of the multi-rank launch on a 1-GPU box only): every rank on
+    # cuda:0 with gloo for the barrier / max-over-ranks reductions. Never used for reported numbers.
+    share = os.environ.get("LT_BENCH_SHARE_DEVICE") == "1" and world > 1
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = workload(args)
     c["idx"] = args.config
     c["seed"] = args.seed
@@ -524,7 +536,7 @@ def main():
         r = oracle_sample(c, gh, W, first, args.cpu_seconds)
         cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "kind": "oracle",
                "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
-                         f"{r['seconds']:.1f} s; oracle/ C + OpenMP, nproc threads)"}
+                         f"{r['seconds']:.1f} s; oracle/ C + OpenMP, {cores()} threads)"}
         idx = np.linspace(0, r["walks"] - 1, num=min(r["walks"], 20000)).astype(np.uint64)
         gp, gl = eng.get_paths_rows(idx)
         ii = idx.astype(np.int64)
@@ -559,6 +571,8 @@ def main():
                              "update_launches": last["update_launches"], "run_ms": last["run_ms"],
                              "init_ms": last["init_ms"], "update_ms": last["update_ms"],
                              "chunks_total": last["chunks_total"], "chunks_free_min": last["chunks_free_min"]}}
+        if share:
+            line["config"]["shared_device_test"] = "all ranks on cuda:0 over gloo: launch test, not a measurement"
         if host_link:
             line["host_link"] = host_link
         if own:
