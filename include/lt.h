@@ -216,6 +216,15 @@ lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_length
 
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out);
 
+/* Ragged copy-out of all paths to HOST buffers: offsets[W+1] (u64; offsets[0] = 0 and
+ * offsets[w+1] - offsets[w] = length[w]) and vertices (u32; walk w's path vertices at
+ * [offsets[w], offsets[w+1])). vertices_capacity is in entries; *total receives offsets[W]. If it is
+ * short the offsets are still written and LT_ERR_INVALID is returned. Suited to PPR, whose rows are
+ * mostly padding (E[length] = 1/alpha of L_max+1 slots). Scratch device memory is reserved on the first
+ * call (never inside lt_run). */
+lt_status lt_get_paths_compact(lt_ctx* ctx, uint64_t* offsets, uint32_t* vertices, uint64_t vertices_capacity,
+                               uint64_t* total);
+
 /* Visit frequency (lt_config.visit_counts = 1): counts[v] = number of path entries equal
  * to v over the walks of the last lt_walks_init* (on this rank: the starts it kept and the steps it
  * took; the sum over ranks is the global count). counts is caller-owned u64[n], host (lt_get_visit_counts)
@@ -232,6 +241,13 @@ lt_status lt_get_visit_counts_device(lt_ctx* ctx, uint64_t* d_counts);
 lt_status lt_run_to_host(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, uint64_t first_walk_id,
                          lt_app app, double length_or_alpha, uint64_t seed, uint32_t* paths, uint32_t* lengths,
                          uint32_t chunks);
+
+/* lt_run_to_host with the ragged layout of lt_get_paths_compact: offsets[W+1] and vertices
+ * (capacity in entries; W * stride always suffices). Each walk range's offsets and packed vertices
+ * stream to the host while the next range walks. */
+lt_status lt_run_to_host_compact(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, uint64_t first_walk_id,
+                                 lt_app app, double length_or_alpha, uint64_t seed, uint64_t* offsets,
+                                 uint32_t* vertices, uint64_t vertices_capacity, uint32_t chunks);
 
 /* ---- Range ownership across GPUs (the north star's multi-GPU mode, not
  * in the paper). With cfg.world = R > 1, rank r owns partitions [floor(P r / R), floor(P (r+1) / R));

@@ -117,6 +117,8 @@ void lt_destroy(lt_ctx* ctx) {
     if (ctx->d_paths2[i] && ctx->d_paths2[i] != ctx->d_paths) cudaFree(ctx->d_paths2[i]);
     if (ctx->d_lengths2[i] && ctx->d_lengths2[i] != ctx->d_lengths) cudaFree(ctx->d_lengths2[i]);
     if (ctx->d_dense2[i]) cudaFree(ctx->d_dense2[i]);
+    if (ctx->d_off2[i]) cudaFree(ctx->d_off2[i]);
+    if (ctx->d_vert2[i]) cudaFree(ctx->d_vert2[i]);
     if (ctx->ev_computed[i]) cudaEventDestroy(ctx->ev_computed[i]);
     if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
   }
@@ -129,6 +131,8 @@ void lt_destroy(lt_ctx* ctx) {
   cudaFree(ctx->d_hc);
   cudaFree(ctx->d_free);
   cudaFree(ctx->d_small);
+  cudaFree(ctx->d_tiles);
+  if (ctx->h_total) cudaFreeHost(ctx->h_total);
   cudaFree(ctx->d_ctr);
   if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
   if (ctx->h_ctr) cudaFreeHost(ctx->h_ctr);
@@ -555,10 +559,9 @@ lt_status lt_run(lt_ctx* ctx) {
   CK(cudaEventRecord(ctx->ev_a, s));
   lt_status st = ctx->ooc.on ? lt::run_out_of_core(ctx) : lt::run_resident(ctx);
   if (st != LT_OK) return st;
-  if (ctx->world == 1) {  // with ownership the rows are pre-filled and merged by the caller
-    CK(lt::launch_finalize_paths(ctx->params, ctx->W, s));
-    ctx->stats.kernel_launches++;
-  }
+  // Path rows hold entries 0..length-1; the 0xFFFFFFFF padding of the rest is output formatting and is
+  // written lazily by the first copy-out (ensure_padded). With ownership the rows were pre-filled.
+  ctx->padded = ctx->world > 1;
   if (ctx->params.wk.visits32) {  // the result is u64[n]
     CK(lt::launch_widen(ctx->params.wk.visits32, ctx->params.wk.visits, ctx->n, s));
     ctx->stats.kernel_launches++;
@@ -597,6 +600,11 @@ lt_status lt_path_stride(lt_ctx* ctx, uint32_t* stride) {
 static lt_status need_ran(lt_ctx* ctx) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
+  CK(cudaSetDevice(ctx->cfg.device));
+  if (!ctx->padded) {  // pad unused path slots with 0xFFFFFFFF once, before the first copy-out
+    CK(lt::launch_finalize_paths(ctx->params, ctx->W, ctx->stream));
+    ctx->padded = true;
+  }
   return LT_OK;
 }
 
@@ -655,6 +663,49 @@ lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_length
                          ctx->stride * sizeof(uint32_t), ctx->W, cudaMemcpyDeviceToDevice, s));
   if (d_lengths && ctx->W)
     CK(cudaMemcpyAsync(d_lengths, ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+  CK(cudaStreamSynchronize(s));
+  return LT_OK;
+}
+
+// Pack rows [0, n) of (paths, lengths) into buffer b: offsets (n entries, base + exclusive prefix sum)
+// and vertices; returns the range's vertex total (synchronises the stream once, for the total).
+static lt_status pack_compact(lt_ctx* ctx, const uint32_t* d_paths, const uint32_t* d_lengths, uint64_t n, int b,
+                              unsigned long long base, uint64_t* total) {
+  cudaStream_t s = ctx->stream;
+  if (!ctx->h_total) CK(cudaHostAlloc((void**)&ctx->h_total, sizeof(unsigned long long), cudaHostAllocMapped));
+  unsigned long long* d_total = nullptr;
+  CK(cudaHostGetDevicePointer((void**)&d_total, ctx->h_total, 0));
+  CK(ensure(ctx->d_tiles, ctx->tiles_cap, std::max<uint64_t>(lt::paths_scan_tiles(n), 1)));
+  CK(ensure(ctx->d_off2[b], ctx->off2_cap[b], std::max<uint64_t>(n, 1)));
+  *ctx->h_total = 0;
+  CK(lt::launch_paths_scan(d_lengths, n, ctx->d_tiles, d_total, s));
+  CK(cudaStreamSynchronize(s));
+  const uint64_t tot = *(volatile unsigned long long*)ctx->h_total;
+  CK(ensure(ctx->d_vert2[b], ctx->vert2_cap[b], std::max<uint64_t>(tot, 1)));
+  CK(lt::launch_paths_pack(d_lengths, n, ctx->d_tiles, base, ctx->d_off2[b], d_paths, ctx->pitch, ctx->d_vert2[b], s));
+  *total = tot;
+  return LT_OK;
+}
+
+lt_status lt_get_paths_compact(lt_ctx* ctx, uint64_t* offsets, uint32_t* vertices, uint64_t vertices_capacity,
+                               uint64_t* total) {
+  if (!ctx || !offsets || !total) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
+  CK(cudaSetDevice(ctx->cfg.device));
+  uint64_t tot = 0;
+  lt_status st = pack_compact(ctx, ctx->d_paths, ctx->d_lengths, ctx->W, 0, 0, &tot);
+  if (st != LT_OK) return st;
+  cudaStream_t s = ctx->stream;
+  if (ctx->W) CK(cudaMemcpyAsync(offsets, ctx->d_off2[0], ctx->W * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  offsets[ctx->W] = tot;
+  *total = tot;
+  if (tot > vertices_capacity) {
+    CK(cudaStreamSynchronize(s));
+    return fail(LT_ERR_INVALID, "vertices buffer too small: need " + std::to_string(tot));
+  }
+  if (tot && !vertices) return fail(LT_ERR_INVALID, "NULL vertices");
+  if (tot) CK(cudaMemcpyAsync(vertices, ctx->d_vert2[0], tot * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+  ctx->stats.d2h_bytes += ctx->W * 8 + tot * 4;
   CK(cudaStreamSynchronize(s));
   return LT_OK;
 }
@@ -734,11 +785,16 @@ lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count) {
   return LT_OK;
 }
 
-lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64_t first_walk_id, lt_app app,
-                         double param, uint64_t seed, uint32_t* paths, uint32_t* lengths, uint32_t chunks) {
+// lt_run_to_host / lt_run_to_host_compact: dense rows (paths != NULL) or the ragged layout
+// (offsets != NULL: offsets[W+1] + vertices[<= vcap]).
+static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64_t first_walk_id, lt_app app,
+                                  double param, uint64_t seed, uint32_t* paths, uint32_t* lengths, uint64_t* offsets,
+                                  uint32_t* vertices, uint64_t vcap, uint32_t chunks) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (ctx->world != 1) return fail(LT_ERR_INVALID, "lt_run_to_host needs a single-rank context");
-  if (W && (!starts || !paths || !lengths)) return fail(LT_ERR_INVALID, "NULL argument");
+  const bool compact = offsets != nullptr;
+  if (W && (!starts || (!compact && (!paths || !lengths)))) return fail(LT_ERR_INVALID, "NULL argument");
+  if (compact && vcap && !vertices) return fail(LT_ERR_INVALID, "NULL vertices");
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_run_to_host before lt_graph_load");
   if (ctx->cfg.visit_counts) return fail(LT_ERR_INVALID, "lt_run_to_host does not accumulate visit counts; use lt_run");
   CK(cudaSetDevice(ctx->cfg.device));
@@ -760,6 +816,7 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
   uint64_t steps = 0, visits = 0, trunc = 0, launches = 0, upd = 0, sweeps = 0, h2d = 0, d2h = 0;
   double run_ms = 0, init_ms = 0, update_ms = 0;
   lt_status st = LT_OK;
+  uint64_t vbase = 0;  // compact: vertices written before this range
   for (uint64_t a = 0, c = 0; a < W || (W == 0 && c == 0); a += wc, ++c) {
     const uint64_t n = std::min<uint64_t>(wc, W - a);
     const int b = (int)(c & 1);
@@ -785,10 +842,28 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
     init_ms += ctx->stats.init_ms;
     update_ms += ctx->stats.update_ms;
     h2d += ctx->stats.h2d_bytes;
-    if (n) {  // stream chunk c out while chunk c+1 computes
+    if (n && compact) {  // ragged copy-out: offsets + packed vertices of this range
+      uint64_t tot = 0;
+      st = pack_compact(ctx, ctx->d_paths2[b], ctx->d_lengths2[b], n, b, vbase, &tot);
+      if (st != LT_OK) break;
+      if (vbase + tot > vcap) {
+        st = fail(LT_ERR_INVALID, "vertices buffer too small");
+        break;
+      }
+      CK(cudaEventRecord(ctx->ev_computed[b], ctx->stream));
+      CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_computed[b], 0));
+      CK(cudaMemcpyAsync(offsets + a, ctx->d_off2[b], n * sizeof(uint64_t), cudaMemcpyDeviceToHost, ctx->copy_stream));
+      if (tot)
+        CK(cudaMemcpyAsync(vertices + vbase, ctx->d_vert2[b], tot * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                           ctx->copy_stream));
+      CK(cudaEventRecord(ctx->ev_copied[b], ctx->copy_stream));
+      vbase += tot;
+      d2h += n * 8 + tot * 4;
+    } else if (n) {  // stream chunk c out while chunk c+1 computes
       // dense rows first (a 2-D copy of 324-B rows runs well below the link rate)
       CK(ensure(ctx->d_dense2[b], ctx->dense2_cap[b], n * ctx->stride));
-      CK(lt::launch_compact_rows(ctx->d_paths2[b], ctx->pitch, ctx->stride, n, ctx->d_dense2[b], ctx->stream));
+      CK(lt::launch_compact_rows(ctx->d_paths2[b], ctx->d_lengths2[b], ctx->pitch, ctx->stride, n, ctx->d_dense2[b],
+                                 ctx->stream));
       CK(cudaEventRecord(ctx->ev_computed[b], ctx->stream));
       CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_computed[b], 0));
       CK(cudaMemcpyAsync(paths + a * ctx->stride, ctx->d_dense2[b], n * ctx->stride * sizeof(uint32_t),
@@ -801,6 +876,7 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
     if (W == 0) break;
   }
   CK(cudaStreamSynchronize(ctx->copy_stream));
+  if (compact && st == LT_OK) offsets[W] = vbase;
   ctx->d_paths = save_p;
   ctx->paths_cap = save_pc;
   ctx->d_lengths = save_l;
@@ -821,6 +897,19 @@ lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64
   ctx->stats.h2d_bytes = h2d;
   ctx->stats.d2h_bytes = d2h;
   return LT_OK;
+}
+
+lt_status lt_run_to_host(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64_t first_walk_id, lt_app app,
+                         double param, uint64_t seed, uint32_t* paths, uint32_t* lengths, uint32_t chunks) {
+  return run_to_host_impl(ctx, W, starts, first_walk_id, app, param, seed, paths, lengths, nullptr, nullptr, 0, chunks);
+}
+
+lt_status lt_run_to_host_compact(lt_ctx* ctx, uint64_t W, const uint32_t* starts, uint64_t first_walk_id, lt_app app,
+                                 double param, uint64_t seed, uint64_t* offsets, uint32_t* vertices,
+                                 uint64_t vertices_capacity, uint32_t chunks) {
+  if (!offsets) return fail(LT_ERR_INVALID, "NULL offsets");
+  return run_to_host_impl(ctx, W, starts, first_walk_id, app, param, seed, nullptr, nullptr, offsets, vertices,
+                          vertices_capacity, chunks);
 }
 
 static lt_status copy_visits(lt_ctx* ctx, uint64_t* counts, cudaMemcpyKind kind) {

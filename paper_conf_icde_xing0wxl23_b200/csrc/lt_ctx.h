@@ -70,6 +70,7 @@ struct lt_ctx {
   // walks
   bool walks_ready = false;
   bool ran = false;
+  bool padded = false;  // path slots past each length hold 0xFFFFFFFF (done lazily, before a copy-out)
   uint64_t W = 0, first = 0, seed = 0;
   lt_app app = LT_APP_DEEPWALK;
   uint32_t length = 0, T = 0, lmax = 127, stride = 1, pitch = 8;
@@ -111,6 +112,14 @@ struct lt_ctx {
   size_t lengths2_cap[2] = {0, 0};
   uint32_t* d_dense2[2] = {nullptr, nullptr};  // dense (stride-pitched) staging for the flat D2H
   size_t dense2_cap[2] = {0, 0};
+  // compact (ragged) path output scratch: tile sums, total, offsets and packed vertices (x2 buffers)
+  unsigned long long* d_tiles = nullptr;
+  size_t tiles_cap = 0;
+  unsigned long long* h_total = nullptr;  // mapped pinned
+  unsigned long long* d_off2[2] = {nullptr, nullptr};
+  size_t off2_cap[2] = {0, 0};
+  uint32_t* d_vert2[2] = {nullptr, nullptr};
+  size_t vert2_cap[2] = {0, 0};
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_computed[2] = {nullptr, nullptr}, ev_copied[2] = {nullptr, nullptr};
   cudaEvent_t ev_a = nullptr, ev_b = nullptr;

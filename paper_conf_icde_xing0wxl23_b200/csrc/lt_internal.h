@@ -92,11 +92,19 @@ cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, 
                                uint32_t* out_paths, uint32_t* out_lengths, cudaStream_t s);
 cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Counters* ctr, const int* free_top,
                             unsigned long long* out_hc, Counters* out_ctr, int* out_free, cudaStream_t s);
-cudaError_t launch_compact_rows(const uint32_t* paths, uint64_t pitch, uint64_t stride, uint64_t n, uint32_t* out,
-                                cudaStream_t s);
+cudaError_t launch_compact_rows(const uint32_t* paths, const uint32_t* lengths, uint64_t pitch, uint64_t stride,
+                                uint64_t n, uint32_t* out, cudaStream_t s);
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
+// compact path output: (1) tile sums + their exclusive scan (total -> *total); (2) offsets[i] = base +
+// exclusive prefix of lengths for i < n, rows packed into vertices (indexed from 0 for this range)
+uint64_t paths_scan_tiles(uint64_t n);  // tile_sum entries launch_paths_scan needs
+cudaError_t launch_paths_scan(const uint32_t* lengths, uint64_t n, unsigned long long* tile_sum,
+                              unsigned long long* total, cudaStream_t s);
+cudaError_t launch_paths_pack(const uint32_t* lengths, uint64_t n, const unsigned long long* tile_off,
+                              unsigned long long base, unsigned long long* offsets, const uint32_t* paths,
+                              uint64_t pitch, uint32_t* vertices, cudaStream_t s);
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
                              cudaStream_t s);

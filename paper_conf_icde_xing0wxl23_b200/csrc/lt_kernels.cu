@@ -14,6 +14,9 @@
 // Written independently of oracle/ (which is never linked or included here).
 #include "lt_internal.h"
 
+#include <cub/block/block_reduce.cuh>
+#include <cub/block/block_scan.cuh>
+
 #include <algorithm>
 #include <cstdio>
 
@@ -770,13 +773,110 @@ __global__ void k_snapshot(const unsigned long long* __restrict__ hc, uint64_t n
   }
 }
 
-// Rows [0, n) of the pitched path matrix -> a dense n x stride buffer (one flat D2H afterwards).
-__global__ void k_compact_rows(const uint32_t* __restrict__ paths, uint64_t pitch, uint64_t stride, uint64_t n,
-                               uint32_t* __restrict__ out) {
+// Rows [0, n) of the pitched path matrix -> a dense n x stride buffer (one flat D2H afterwards), with
+// the entries past each row's length written as 0xFFFFFFFF (the padding lt_run leaves undone).
+__global__ void k_compact_rows(const uint32_t* __restrict__ paths, const uint32_t* __restrict__ lengths, uint64_t pitch,
+                               uint64_t stride, uint64_t n, uint32_t* __restrict__ out) {
   const uint64_t total = n * stride;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x)
-    out[i] = paths[(i / stride) * pitch + (i % stride)];
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t r = i / stride, t = i % stride;
+    out[i] = t < __ldg(lengths + r) ? paths[r * pitch + t] : kEmpty;
+  }
 }
+
+// ---- compact (ragged) path output: offsets = base + exclusive prefix sum of lengths, vertices packed.
+// Three passes over tiles of kScanTile lengths: tile sums; one block scans the tile sums (and writes
+// the total); each tile scans itself, writes its offsets and packs its rows (warp per row).
+constexpr uint32_t kScanTile = 4096;  // 256 threads x 16 lengths
+
+__global__ void __launch_bounds__(256) k_scan_tiles(const uint32_t* __restrict__ len, uint64_t n,
+                                                   unsigned long long* __restrict__ tile_sum) {
+  using Reduce = cub::BlockReduce<unsigned long long, 256>;
+  __shared__ typename Reduce::TempStorage tmp;
+  const uint64_t base = (uint64_t)blockIdx.x * kScanTile + threadIdx.x * 16;
+  unsigned long long x = 0;
+#pragma unroll
+  for (int j = 0; j < 16; ++j)
+    if (base + j < n) x += len[base + j];
+  const unsigned long long t = Reduce(tmp).Sum(x);
+  if (threadIdx.x == 0) tile_sum[blockIdx.x] = t;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_tile_sums(unsigned long long* __restrict__ tile_sum, uint64_t ntiles,
+                                                         unsigned long long* __restrict__ total) {
+  using Scan = cub::BlockScan<unsigned long long, 1024>;
+  __shared__ typename Scan::TempStorage tmp;
+  __shared__ unsigned long long carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (uint64_t b = 0; b < ntiles; b += 1024) {
+    const uint64_t i = b + threadIdx.x;
+    unsigned long long x = i < ntiles ? tile_sum[i] : 0, agg = 0;
+    Scan(tmp).ExclusiveSum(x, x, agg);
+    if (i < ntiles) tile_sum[i] = x + carry;
+    __syncthreads();
+    if (threadIdx.x == 0) carry += agg;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *total = carry;
+}
+
+__global__ void __launch_bounds__(256) k_scan_apply(const uint32_t* __restrict__ len, uint64_t n,
+                                                   const unsigned long long* __restrict__ tile_off,
+                                                   unsigned long long base, unsigned long long* __restrict__ offsets,
+                                                   const uint32_t* __restrict__ paths, uint64_t pitch,
+                                                   uint32_t* __restrict__ vertices) {
+  using Scan = cub::BlockScan<unsigned long long, 256>;
+  __shared__ typename Scan::TempStorage tmp;
+  __shared__ unsigned long long s_off[kScanTile];
+  const uint64_t t0 = (uint64_t)blockIdx.x * kScanTile;
+  const uint64_t mine = t0 + threadIdx.x * 16;
+  unsigned long long v[16], x = 0;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    v[j] = (mine + j < n) ? len[mine + j] : 0;
+    x += v[j];
+  }
+  Scan(tmp).ExclusiveSum(x, x);
+  const unsigned long long tb = tile_off[blockIdx.x];  // local (0-based) offset of this tile
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    s_off[threadIdx.x * 16 + j] = tb + x;
+    if (mine + j < n) offsets[mine + j] = base + tb + x;
+    x += v[j];
+  }
+  __syncthreads();
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t rows = (n - t0 < kScanTile) ? n - t0 : kScanTile;
+  for (uint64_t r = threadIdx.x >> 5; r < rows; r += blockDim.x >> 5) {
+    const uint32_t L = __ldg(len + t0 + r);
+    const uint32_t* src = paths + (t0 + r) * pitch;
+    uint32_t* dst = vertices + s_off[r];
+    for (uint32_t t = lane; t < L; t += 32) dst[t] = src[t];
+  }
+}
+
+}  // namespace
+
+uint64_t paths_scan_tiles(uint64_t n) { return (n + kScanTile - 1) / kScanTile; }
+
+cudaError_t launch_paths_scan(const uint32_t* lengths, uint64_t n, unsigned long long* tile_sum,
+                              unsigned long long* total, cudaStream_t s) {
+  const uint64_t nt = (n + kScanTile - 1) / kScanTile;
+  if (nt) k_scan_tiles<<<(uint32_t)nt, 256, 0, s>>>(lengths, n, tile_sum);
+  k_scan_tile_sums<<<1, 1024, 0, s>>>(tile_sum, nt, total);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_paths_pack(const uint32_t* lengths, uint64_t n, const unsigned long long* tile_off,
+                              unsigned long long base, unsigned long long* offsets, const uint32_t* paths,
+                              uint64_t pitch, uint32_t* vertices, cudaStream_t s) {
+  const uint64_t nt = (n + kScanTile - 1) / kScanTile;
+  if (nt) k_scan_apply<<<(uint32_t)nt, 256, 0, s>>>(lengths, n, tile_off, base, offsets, paths, pitch, vertices);
+  return cudaGetLastError();
+}
+
+namespace {
 
 __global__ void k_check_range(const uint32_t* a, uint64_t cnt, uint32_t n, uint32_t* bad) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += (uint64_t)gridDim.x * blockDim.x)
@@ -949,10 +1049,10 @@ cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Coun
   return cudaGetLastError();
 }
 
-cudaError_t launch_compact_rows(const uint32_t* paths, uint64_t pitch, uint64_t stride, uint64_t n, uint32_t* out,
-                                cudaStream_t s) {
+cudaError_t launch_compact_rows(const uint32_t* paths, const uint32_t* lengths, uint64_t pitch, uint64_t stride,
+                                uint64_t n, uint32_t* out, cudaStream_t s) {
   if (!n) return cudaSuccess;
-  k_compact_rows<<<num_sms() * 8, 256, 0, s>>>(paths, pitch, stride, n, out);
+  k_compact_rows<<<num_sms() * 8, 256, 0, s>>>(paths, lengths, pitch, stride, n, out);
   return cudaGetLastError();
 }
 

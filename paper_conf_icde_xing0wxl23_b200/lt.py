@@ -33,7 +33,7 @@ EXPORTED = [
     "lt_graph_load_device", "lt_get_bounds", "lt_walks_init", "lt_walks_init_ex", "lt_run", "lt_path_stride",
     "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
-    "lt_get_visit_counts", "lt_get_visit_counts_device",
+    "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
 ]
 
 
@@ -108,6 +108,8 @@ _lib.lt_pending.argtypes = [_vp, ctypes.POINTER(_u64), _vp]
 _lib.lt_exchange_pack.argtypes = [_vp, _vp, _u64, _vp]
 _lib.lt_exchange_insert.argtypes = [_vp, _vp, _u64]
 _lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
+_lib.lt_run_to_host_compact.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u64, _u32]
+_lib.lt_get_paths_compact.argtypes = [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]
 
 
 class LTError(RuntimeError):
@@ -280,6 +282,39 @@ class Engine:
             raise ValueError("run_to_host writes host buffers")
         _check(_lib.lt_run_to_host(self._h, W, ps, first_walk_id, app, float(param), seed, pp, pl, chunks))
         return paths, lengths
+
+    def run_to_host_compact(self, starts, app: int = DEEPWALK, param: float = 80, seed: int = 1,
+                            first_walk_id: int = 0, offsets=None, vertices=None, chunks: int = 0):
+        """lt_run_to_host with the ragged output: (offsets u64[W+1], vertices u32[offsets[W]]).
+        Preallocated host buffers (pinned torch tensors for overlapped copies) may be passed; vertices
+        needs room for W * stride entries in the worst case."""
+        ps, dev, keep = _ptr(starts, np.uint32)
+        if dev:
+            raise ValueError("run_to_host_compact takes host starts")
+        W = keep.numel() if _is_torch(keep) else len(keep)
+        S = (int(param) + 1) if app == DEEPWALK else self._lmax + 1
+        if offsets is None:
+            offsets = np.empty(W + 1, dtype=np.uint64)
+        if vertices is None:
+            vertices = np.empty(max(W * S, 1), dtype=np.uint32)
+        po, do, ko = _ptr(offsets, np.uint64)
+        pv, dv, kv = _ptr(vertices, np.uint32)
+        if do or dv:
+            raise ValueError("run_to_host_compact writes host buffers")
+        cap = kv.numel() if _is_torch(kv) else len(kv)
+        _check(_lib.lt_run_to_host_compact(self._h, W, ps, first_walk_id, app, float(param), seed, po, pv, cap, chunks))
+        total = int(offsets[W])
+        return offsets, vertices[:total]
+
+    def get_paths_compact(self):
+        """Ragged copy-out (lt_get_paths_compact): (offsets u64[W+1], vertices u32[offsets[W]])."""
+        W, S = self.num_walks, self.stride()
+        offsets = np.empty(W + 1, dtype=np.uint64)
+        vertices = np.empty(max(W * S, 1), dtype=np.uint32)
+        total = _u64()
+        _check(_lib.lt_get_paths_compact(self._h, offsets.ctypes.data, vertices.ctypes.data, len(vertices),
+                                         ctypes.byref(total)))
+        return offsets, vertices[: total.value]
 
     def stride(self) -> int:
         s = _u32()

@@ -276,3 +276,51 @@ def test_run_to_host_streamed(gpu, cfg1, chunks, app, param):
     np.testing.assert_array_equal(lengths.numpy().view(np.uint32), ol)
     np.testing.assert_array_equal(paths.numpy().view(np.uint32), op)
     assert st["steps"] == osteps and st["num_walks"] == W
+
+
+def _ragged_equals_rows(offsets, vertices, paths, lengths):
+    assert offsets[0] == 0 and np.array_equal(np.diff(offsets.astype(np.int64)), lengths.astype(np.int64))
+    assert len(vertices) == int(offsets[-1])
+    for w in range(len(lengths)):
+        np.testing.assert_array_equal(vertices[int(offsets[w]): int(offsets[w + 1])], paths[w, : lengths[w]])
+
+
+@pytest.mark.parametrize("app,param,W", [(LT.PPR, 0.15, 4096), (LT.PPR, 0.5, 9000), (LT.DEEPWALK, 9, 4097),
+                                         (LT.DEEPWALK, 3, 0)])
+@pytest.mark.parametrize("P", [1, 4])
+def test_compact_paths_equal_oracle(gpu, cfg1, app, param, W, P):
+    """lt_get_paths_compact: offsets = exclusive prefix sum of the oracle's lengths, vertices = the
+    oracle's rows concatenated (tiles of 4096 lengths: W = 9000 spans a ragged third tile)."""
+    starts = (lt_inputs.deepwalk_starts(W, cfg1.n) if app == LT.DEEPWALK else lt_inputs.ppr_starts(W, cfg1.argmax_deg))
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, app, param, 3)
+        e.run()
+        offsets, vertices = e.get_paths_compact()
+        paths, lengths = e.get_paths()  # lazy padding after a compact copy-out
+    op, ol, _, _ = run_oracle(cfg1, starts, app, param, 3)
+    np.testing.assert_array_equal(paths, op)
+    _ragged_equals_rows(offsets, vertices, op, ol)
+
+
+@pytest.mark.parametrize("chunks", [1, 3])
+@pytest.mark.parametrize("app,param", [(LT.PPR, 0.2), (LT.DEEPWALK, 11)])
+def test_run_to_host_compact(gpu, cfg1, chunks, app, param):
+    W = 10_000
+    starts = (lt_inputs.deepwalk_starts(W, cfg1.n) if app == LT.DEEPWALK else lt_inputs.ppr_starts(W, cfg1.argmax_deg))
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 1)
+        offsets, vertices = e.run_to_host_compact(starts, app, param, 9, 77, chunks=chunks)
+        st = e.stats()
+    op, ol, osteps, _ = run_oracle(cfg1, starts, app, param, 9, first=77)
+    _ragged_equals_rows(offsets, vertices, op, ol)
+    assert st["steps"] == osteps
+
+
+def test_compact_capacity_error(gpu, cfg1):
+    starts = lt_inputs.ppr_starts(2000, cfg1.argmax_deg)
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 1)
+        with pytest.raises(LT.LTError) as ei:
+            e.run_to_host_compact(starts, LT.PPR, 0.15, 1, vertices=np.empty(10, dtype=np.uint32))
+        assert ei.value.status == LT.lt.LT_ERR_INVALID

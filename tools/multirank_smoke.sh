@@ -1,0 +1,11 @@
+# Multi-rank launch of bench.py on a 1-GPU box (all ranks share cuda:0; gloo for the collectives).
+# Checks the driver's torchrun path end to end at small size; the numbers are not measurements.
+export LT_BENCH_SHARE_DEVICE=1
+for n in 2 4; do
+  python -m torch.distributed.run --nnodes=1 --nproc-per-node $n --master-addr 127.0.0.1 --master-port 29511 \
+    bench.py --gpus $n --steps 3 --warmup 3 --config 2 --no-cpu-baseline > gpurun_out/multirank_n$n.json 2> gpurun_out/multirank_n$n.err
+  echo "n=$n rc=$?"
+  python -m torch.distributed.run --nnodes=1 --nproc-per-node $n --master-addr 127.0.0.1 --master-port 29512 \
+    bench.py --impl reference --gpus $n --steps 2 --warmup 3 --config 2 > gpurun_out/multirank_ref_n$n.json 2> gpurun_out/multirank_ref_n$n.err
+  echo "ref n=$n rc=$?"
+done
