@@ -73,6 +73,8 @@ def parse():
     ap.add_argument("--graph-pool-gb", type=float, default=0.0,
                     help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
     ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
+    ap.add_argument("--continue-resident", type=int, default=1,
+                    help="out-of-core: walks keep stepping into partitions resident in the graph pool (f4)")
     ap.add_argument("--app", default="config", choices=["config", "deepwalk", "ppr", "pagerank"],
                     help="override the config's application; pagerank = random walk with restart "
                          "(PAPER.md:287, SURVEY.md 8(f) f2) of the config's length, with visit counting")
@@ -319,7 +321,8 @@ def main():
     eng = LT.Engine(visit_counts=vis, device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
-                    rank=rank if own else 0, world=world if own else 1, refill=args.refill)
+                    rank=rank if own else 0, world=world if own else 1, refill=args.refill,
+                    continue_resident=bool(args.continue_resident))
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
@@ -455,7 +458,9 @@ def main():
                      "iterations": last["iterations"], "explicit_copies": last["explicit_copies"],
                      "pool_hits": last["pool_hits"], "zero_copy_launches": last["zero_copy_launches"],
                      "preemptive_launches": last["preemptive_launches"],
-                     "hit_rate": last["pool_hits"] / max(1, last["iterations"])}
+                     "hit_rate": last["pool_hits"] / max(1, last["iterations"]),
+                     "continue_resident": bool(args.continue_resident),
+                     "visits_per_step": last["visits"] / max(1, last["steps"])}
 
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0 and not own and vis:

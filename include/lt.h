@@ -119,6 +119,11 @@ typedef struct lt_config {
                                  included) adds 1 to its vertex. Read with lt_get_visit_counts*. The
                                  kernels count in u32 while no count can reach 2^32 (W * stride <
                                  2^32) and widen at the end of lt_run; 2 -> always count in u64. */
+  uint32_t continue_resident; /* out-of-core: 1 -> a walk leaving the launched partition for another
+                                 partition resident in the graph pool keeps stepping there instead of
+                                 being appended to its bucket (parity-neutral);
+                                 uses the lane-refill kernel. Ignored when the graph is HBM-resident. */
+  uint32_t reserved[3];
 } lt_config;
 
 typedef struct lt_stats {

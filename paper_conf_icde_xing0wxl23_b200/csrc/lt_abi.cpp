@@ -97,6 +97,7 @@ static void free_ooc(lt_ctx* ctx) {
   for (auto e : o.ev_used) cudaEventDestroy(e);
   if (o.load_stream) cudaStreamDestroy(o.load_stream);
   if (o.d_gpool) cudaFree(o.d_gpool);
+  if (o.d_table) cudaFree(o.d_table);
   if (o.h_row_ptr) cudaFreeHost(o.h_row_ptr);
   if (o.h_col) cudaFreeHost(o.h_col);
   ctx->ooc = lt::OutOfCore();
@@ -294,6 +295,9 @@ static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     CK(cudaEventCreateWithFlags(&o.ev_used[q], cudaEventDisableTiming));
   }
   CK(cudaStreamCreateWithFlags(&o.load_stream, cudaStreamNonBlocking));
+  CK(cudaMalloc((void**)&o.d_table, (size_t)P * sizeof(uint32_t)));
+  CK(cudaMemset(o.d_table, 0xFF, (size_t)P * sizeof(uint32_t)));
+  o.table.assign(P, lt::kEmpty);
   o.on = true;
   ctx->stats.pool_blocks = o.m_g;
   ctx->stats.pool_block_bytes = o.block_bytes;
@@ -492,6 +496,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.pool.free_list = ctx->d_free;
   p.pool.free_top = (int*)ctx->d_small;
   p.ctr = ctx->d_ctr;
+  p.cont = lt::Cont{};
+  if (ctx->ooc.on && ctx->cfg.continue_resident)
+    p.cont = lt::Cont{ctx->ooc.d_table, ctx->ooc.d_gpool, ctx->ooc.block_bytes, ctx->ooc.rp_bytes};
   p.insert_mode = ctx->cfg.insert_mode;
   p.gather_mode = ctx->cfg.gather_mode;
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
@@ -499,8 +506,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
   // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
   p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
+  if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
-  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp);
+  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0);
 
   ctx->W = W;
   ctx->first = first_walk_id;

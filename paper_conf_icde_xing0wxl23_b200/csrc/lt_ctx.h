@@ -40,6 +40,10 @@ struct OutOfCore {
   std::vector<uint64_t> loaded_at;  // block -> load sequence number (FIFO eviction)
   std::vector<cudaEvent_t> ev_ready, ev_used;  // per block: load finished / last compute use
   cudaStream_t load_stream = nullptr;
+  // resident-neighbour continuation (f4): device table partition -> block (kEmpty if not usable) and
+  // its host mirror
+  uint32_t* d_table = nullptr;
+  std::vector<uint32_t> table;
 };
 
 }  // namespace lt

@@ -71,8 +71,19 @@ struct Owner {
   const uint16_t* owner;  // [P] rank of each partition (nullptr when world == 1)
 };
 
+// Resident-neighbour continuation (out-of-core mode): table[q] = graph-pool block
+// holding partition q, ready and safe to read for the whole launch, or kEmpty. A walk that leaves the
+// launched partition for a partition in the table keeps stepping through that block's view instead of
+// being appended to a bucket. table == nullptr: off.
+struct Cont {
+  const uint32_t* table;          // [P]
+  const char* gpool;              // block b at gpool + b * block_bytes: row_ptr slice, col slice at rp_bytes
+  uint64_t block_bytes, rp_bytes;
+};
+
 struct Params {
   Walk wk;
+  Cont cont;
   Pool pool;
   Counters* ctr;
   Owner own;
@@ -105,10 +116,13 @@ cudaError_t launch_paths_scan(const uint32_t* lengths, uint64_t n, unsigned long
 cudaError_t launch_paths_pack(const uint32_t* lengths, uint64_t n, const unsigned long long* tile_off,
                               unsigned long long base, unsigned long long* offsets, const uint32_t* paths,
                               uint64_t pitch, uint32_t* vertices, cudaStream_t s);
+cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_t* val, uint32_t count,
+                             cudaStream_t s);  // table[idx[i]] = val[i], count <= kTableSetMax
+constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
                              cudaStream_t s);
-int update_kernel_occupancy(uint32_t block, uint32_t ilp);  // resident blocks per SM (update kernel)
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill);  // resident blocks per SM (update kernel)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

@@ -544,6 +544,9 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
 // without refill most lanes of a warp idle most of the time. A warp claims kRefill positions of the
 // bucket at a time (one atomic per kRefill walks) and hands them to its idle lanes.
 constexpr uint32_t kRefill = 64;
+#ifndef LT_RF_MINB
+#define LT_RF_MINB 4  // resident 256-thread blocks per SM the register budget is cut for (64 regs)
+#endif
 
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
@@ -555,8 +558,13 @@ __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, c
   __syncwarp();
 }
 
-template <int APP, int GM, int LAY, int VIS>
-__global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
+// CONT (out-of-core, CSR layout only): resident-neighbour continuation (the
+// paper's preemptive idea taken inside the kernel). Each lane carries its own graph
+// view (row_ptr / col pointers pre-offset by the view's first vertex / first edge, and the range it
+// covers); a walk that leaves the view for a partition whose block is in p.cont.table switches to that
+// block's view and keeps stepping.
+template <int APP, int GM, int LAY, int VIS, int CONT>
+__global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
   const Pool& pl = p.pool;
@@ -575,6 +583,10 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
   bool has = false;
   uint4 rec = make_uint4(0, 0, 0, 0);  // .x = row, .y = v, .z = t
   uint32_t* prow = wk.paths;
+  // the lane's graph view (CONT): row_ptr indexed by the global vertex, col by the global offset
+  const unsigned long long* c_rp = wk.row_ptr - wk.vbase;
+  const uint32_t* c_col = wk.col - wk.ebase;
+  uint32_t c_lo = lo, c_span = span;
   uint32_t pb[8];
   uint32_t nb = 0;
   unsigned long long off = 0;
@@ -614,6 +626,12 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
           off = __ldg(wk.row_ptr + rec.y);
           d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
         }
+        if (CONT) {  // a walk from the bucket starts in the launched partition's view
+          c_rp = wk.row_ptr - wk.vbase;
+          c_col = wk.col - wk.ebase;
+          c_lo = lo;
+          c_span = span;
+        }
       }
       q_cur += (avail < (uint32_t)__popc(need)) ? avail : (uint32_t)__popc(need);
       need = __ballot_sync(kFull, !has);
@@ -629,9 +647,15 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
         trunc = true;
       } else {
         if (LAY == 0) {
-          const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
-          off = __ldg(rp) - wk.ebase;
-          d = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
+          if (CONT) {
+            const unsigned long long* rp = c_rp + rec.y;
+            off = __ldg(rp);
+            d = (uint32_t)(__ldg(rp + 1) - off);
+          } else {
+            const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
+            off = __ldg(rp) - wk.ebase;
+            d = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
+          }
         }
         const uint64_t wid = wk.first_walk_id + rec.x;
         const uint4 b = philox10(make_uint4(rec.z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
@@ -652,7 +676,7 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
               d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
             }
           } else if (LAY == 0) {
-            nv = ld_col<GM>(wk.col + off + idx, pol);
+            nv = ld_col<GM>((CONT ? c_col : wk.col) + off + idx, pol);
           } else {
             const uint4 e = ld_adj<GM>(wk.adj + off + idx, pol);
             nv = e.x;
@@ -681,7 +705,24 @@ __global__ void __launch_bounds__(256, 4) k_update_rf(Params p, uint32_t k) {
           } else if (wk.path_mode == 1) {
             prow[t] = nv;
           }
-          left = (nv - lo >= span);
+          if (CONT) {
+            left = (nv - c_lo >= c_span);
+            if (left) {  // into a resident partition: switch the view and keep stepping
+              const uint32_t q = find_partition(B, wk.P, nv);
+              const uint32_t blk = __ldg(p.cont.table + q);
+              if (blk != kEmpty) {
+                const char* base = p.cont.gpool + (uint64_t)blk * p.cont.block_bytes;
+                const unsigned long long* rp = reinterpret_cast<const unsigned long long*>(base);
+                c_lo = __ldg(wk.bounds + q);
+                c_span = __ldg(wk.bounds + q + 1) - c_lo;
+                c_rp = rp - c_lo;
+                c_col = reinterpret_cast<const uint32_t*>(base + p.cont.rp_bytes) - __ldg(rp);
+                left = false;
+              }
+            }
+          } else {
+            left = (nv - lo >= span);
+          }
         }
       }
     }
@@ -916,9 +957,10 @@ int num_sms() {
 
 uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 
-int update_kernel_occupancy(uint32_t block, uint32_t ilp) {
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill) {
   int nb = 0;
-  if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
+  if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
+  else if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
   else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1, 0>, (int)block, 0);
   else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1, 0>, (int)block, 0);
   return nb > 0 ? nb : 1;
@@ -978,15 +1020,26 @@ void launch_update_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block,
   k_update<APP, GM, ILP, LAY, VIS><<<grid, block, bounds_smem(p), s>>>(p, k);
 }
 
-template <int APP, int GM, int LAY, int VIS>
-void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+template <int APP, int GM, int LAY, int VIS, int CONT>
+void launch_update_rf_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(k_update_rf<APP, GM, LAY, VIS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaFuncSetAttribute(k_update_rf<APP, GM, LAY, VIS, CONT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          kSmemBoundsCap * 4);
     attr = true;
   }
-  k_update_rf<APP, GM, LAY, VIS><<<grid, block, bounds_smem(p), s>>>(p, k);
+  k_update_rf<APP, GM, LAY, VIS, CONT><<<grid, block, bounds_smem(p), s>>>(p, k);
+}
+
+template <int APP, int GM, int LAY, int VIS>
+void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  if constexpr (LAY == 0) {
+    if (p.cont.table) {
+      launch_update_rf_t<APP, GM, LAY, VIS, 1>(p, k, grid, block, s);
+      return;
+    }
+  }
+  launch_update_rf_t<APP, GM, LAY, VIS, 0>(p, k, grid, block, s);
 }
 
 template <int APP, int GM, int LAY, int VIS>
@@ -1068,9 +1121,29 @@ cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, 
   return cudaGetLastError();
 }
 
+struct TableSet {
+  uint32_t idx[kTableSetMax], val[kTableSetMax];
+};
+__global__ void k_table_set(uint32_t* table, TableSet ts, uint32_t count) {
+  if (threadIdx.x < count) table[ts.idx[threadIdx.x]] = ts.val[threadIdx.x];
+}
+
 __global__ void k_widen(const uint32_t* __restrict__ src, unsigned long long* __restrict__ dst, uint64_t n) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
     dst[i] = src[i];
+}
+
+cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_t* val, uint32_t count,
+                             cudaStream_t s) {
+  if (!count) return cudaSuccess;
+  if (count > kTableSetMax) return cudaErrorInvalidValue;
+  TableSet ts;
+  for (uint32_t i = 0; i < count; ++i) {
+    ts.idx[i] = idx[i];
+    ts.val[i] = val[i];
+  }
+  k_table_set<<<1, 32, 0, s>>>(table, ts, count);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s) {

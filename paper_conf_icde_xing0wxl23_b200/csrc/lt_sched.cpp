@@ -134,11 +134,48 @@ Params view_zero_copy(const lt_ctx* ctx) {
   return p;
 }
 
+// Continuation table (f4), kept on the compute stream: partition k's entry is published before a
+// launch that may read its block — for the launched partition itself (the stream already waits for
+// its load) and for every other resident partition whose load the host has seen complete — and
+// withdrawn before its block is reloaded. Every launch may read any published block, so a reload
+// waits for an event recorded on the compute stream after the withdrawal.
+lt_status table_publish(lt_ctx* ctx, int launched) {
+  OutOfCore& o = ctx->ooc;
+  if (!ctx->params.cont.table) return LT_OK;
+  uint32_t idx[kTableSetMax], val[kTableSetMax], cnt = 0;
+  for (uint32_t q = 0; q < o.m_g; ++q) {
+    const int k = o.part_in[q];
+    if (k < 0 || o.table[k] == q) continue;
+    if (k != launched && !event_done(o.ev_ready[q])) continue;
+    o.table[k] = q;
+    idx[cnt] = (uint32_t)k;
+    val[cnt] = q;
+    if (++cnt == kTableSetMax) {
+      CK(launch_table_set(o.d_table, idx, val, cnt, ctx->stream));
+      ctx->stats.kernel_launches++;
+      cnt = 0;
+    }
+  }
+  if (cnt) {
+    CK(launch_table_set(o.d_table, idx, val, cnt, ctx->stream));
+    ctx->stats.kernel_launches++;
+  }
+  return LT_OK;
+}
+
 lt_status load_partition(lt_ctx* ctx, uint32_t k, int b, uint64_t seq) {
   OutOfCore& o = ctx->ooc;
   const uint32_t v0 = ctx->h_bounds[k], v1 = ctx->h_bounds[k + 1];
   const uint64_t e0 = o.h_row_ptr[v0], e1 = o.h_row_ptr[v1];
   char* base = o.d_gpool + (size_t)b * o.block_bytes;
+  const int old = o.part_in[b];
+  if (ctx->params.cont.table && old >= 0 && o.table[old] != kEmpty) {  // withdraw the evicted partition
+    const uint32_t idx = (uint32_t)old, val = kEmpty;
+    CK(launch_table_set(o.d_table, &idx, &val, 1, ctx->stream));
+    ctx->stats.kernel_launches++;
+    o.table[old] = kEmpty;
+    CK(cudaEventRecord(o.ev_used[b], ctx->stream));  // after every launch that could read the block
+  }
   CK(cudaStreamWaitEvent(o.load_stream, o.ev_used[b], 0));  // the block's last reader is done
   CK(cudaMemcpyAsync(base, o.h_row_ptr + v0, 8ull * (v1 - v0 + 1), cudaMemcpyHostToDevice, o.load_stream));
   if (e1 > e0)
@@ -158,7 +195,9 @@ lt_status compute_block(lt_ctx* ctx, uint32_t k) {
   OutOfCore& o = ctx->ooc;
   const int b = o.block_of[k];
   CK(cudaStreamWaitEvent(ctx->stream, o.ev_ready[b], 0));
-  lt_status st = launch_update_timed(ctx, view_block(ctx, k, b), k, pending(ctx, k));
+  lt_status st = table_publish(ctx, (int)k);
+  if (st != LT_OK) return st;
+  st = launch_update_timed(ctx, view_block(ctx, k, b), k, pending(ctx, k));
   if (st != LT_OK) return st;
   CK(cudaEventRecord(o.ev_used[b], ctx->stream));
   return LT_OK;
@@ -206,6 +245,8 @@ lt_status run_out_of_core(lt_ctx* ctx) {
     // adaptive scheduling: zero copy when alpha * w < S_p (Alg. 2 l.3-4)
     if (ctx->cfg.zero_copy && alpha * pending(ctx, i) < partition_bytes(ctx, i)) {
       ctx->stats.zero_copy_launches++;
+      st = table_publish(ctx, -1);
+      if (st != LT_OK) return st;
       st = launch_update_timed(ctx, view_zero_copy(ctx), i, pending(ctx, i));
       if (st != LT_OK) return st;
       continue;

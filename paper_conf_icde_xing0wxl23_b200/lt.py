@@ -61,6 +61,8 @@ class Config(ctypes.Structure):
         ("world", ctypes.c_uint32),
         ("refill", ctypes.c_uint32),
         ("visit_counts", ctypes.c_uint32),
+        ("continue_resident", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 3),
     ]
 
 
@@ -165,7 +167,7 @@ class Engine:
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
-                 visit_counts: bool = False):
+                 visit_counts: bool = False, continue_resident: bool = False):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -187,6 +189,7 @@ class Engine:
         cfg.rank = rank
         cfg.world = world
         cfg.refill = refill
+        cfg.continue_resident = int(bool(continue_resident))
         cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device

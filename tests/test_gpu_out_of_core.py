@@ -110,3 +110,47 @@ def test_scheduling_counters_table3_shape(gpu):
         res[name] = (st["iterations"], st["explicit_copies"], round(hit, 3), st["preemptive_launches"])
     print("Table III shape (iterations, explicit copies, hit rate, preemptive launches):", res)
     assert res["PS"][3] > 0 and res["PS+SS"][3] > 0
+
+
+@pytest.mark.parametrize("policy", [LT.POLICY_SELECTIVE, LT.POLICY_ROUND_ROBIN])
+@pytest.mark.parametrize("blocks", [1, 3, 16])
+@pytest.mark.parametrize("zero_copy", [False, True])
+def test_continue_into_resident_partitions_exact(gpu, g14, policy, blocks, zero_copy):
+    """with continuation a walk that leaves the launched partition for another
+    partition resident in the graph pool keeps stepping there. Paths are unchanged (parity-neutral);
+    with more than one block resident, walks need fewer visits (bucket round trips)."""
+    P = 16
+    starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
+    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy,
+                             continue_resident=True)
+    op, ol, osteps, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)
+    assert st["steps"] == osteps
+    _, _, st0 = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy)
+    if blocks == P:  # everything resident after the first loads: most steps continue in-kernel
+        assert st["visits"] < st0["visits"] // 2
+    elif blocks > 1:
+        assert st["visits"] < st0["visits"]
+
+
+@pytest.mark.parametrize("app,param", [(LT.PPR, 0.15), (LT.PAGERANK, 0.2)])
+def test_continue_resident_ppr_and_pagerank(gpu, g14, app, param):
+    P, blocks = 32, 6
+    pool = block_bytes(g14, P) * blocks
+    starts = (lt_inputs.ppr_starts(20_000, g14.argmax_deg) if app == LT.PPR
+              else lt_inputs.deepwalk_starts(g14.n, g14.n))
+    with LT.Engine(graph_pool_bytes=pool, continue_resident=True, zero_copy=True, visit_counts=True) as e:
+        e.graph_load(g14.row_ptr, g14.col, P)
+        if app == LT.PAGERANK:
+            e.walks_init_pagerank(starts, 12, param, 5)
+        else:
+            e.walks_init(starts, app, param, 5)
+        e.run()
+        paths, lengths = e.get_paths()
+        counts = e.visit_counts()
+    kw = dict(app=O.PPR, alpha=param) if app == LT.PPR else dict(app=O.PAGERANK, length=12, alpha=param)
+    op, ol, _, _ = O.walks(g14.row_ptr, g14.col, starts, seed=5, **kw)
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)
+    np.testing.assert_array_equal(counts, O.visit_counts(op, ol, g14.n))

@@ -78,10 +78,13 @@ def test_ownership_ppr_exact(gpu, g13, world):
         np.testing.assert_array_equal(paths, op)
 
 
-def test_ownership_out_of_core_ranks(gpu, g13):
-    """Each rank running its owned range out of core (graph pool of 2 blocks)."""
+@pytest.mark.parametrize("cont", [False, True])
+def test_ownership_out_of_core_ranks(gpu, g13, cont):
+    """Each rank running its owned range out of core (graph pool of 2 blocks), with and without
+    continuation into resident partitions (f4)."""
     starts = lt_inputs.deepwalk_starts(g13.n, g13.n)
-    res = run_owned(g13, starts, LT.DEEPWALK, 10, 4, 8, 2, graph_pool_bytes=8 << 20, zero_copy=True)
+    res = run_owned(g13, starts, LT.DEEPWALK, 10, 4, 8, 2, graph_pool_bytes=8 << 20, zero_copy=True,
+                    continue_resident=cont)
     op, ol, _, _ = oracle_of(g13, starts, LT.DEEPWALK, 10, 4)
     for paths, lengths, _, st in res:
         np.testing.assert_array_equal(paths, op)
