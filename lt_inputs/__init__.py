@@ -46,6 +46,13 @@ def _lib():
                                        ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32)]
         lib.ltgen_rmat_gpu.restype = ctypes.c_int
         lib.ltgen_gpu_free.argtypes = [ctypes.c_void_p]
+        lib.ltgen_rmat_gpu_count.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int,
+                                             ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_uint64)]
+        lib.ltgen_rmat_gpu_into.argtypes = [ctypes.c_uint32, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int,
+                                            ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                            ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint64),
+                                            ctypes.POINTER(ctypes.c_uint32), ctypes.POINTER(ctypes.c_uint32),
+                                            ctypes.POINTER(ctypes.c_uint32)]
         lib.ltgen_gpu_last_error.restype = ctypes.c_char_p
         lib.ltgen_gpu_memcpy.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
         lib.ltgen_gpu_memcpy.restype = ctypes.c_int
@@ -93,12 +100,45 @@ def rmat_cpu(scale: int, tuples: int, seed: int = 1, permute: bool = False, thre
     return Graph(int(g.n), int(g.m), row_ptr, col, int(g.max_deg), int(g.argmax_deg))
 
 
-def rmat_gpu(scale: int, tuples: int, seed: int = 1, permute: bool = False, device: int = 0) -> Graph:
-    """Same graph as rmat_cpu, generated on the GPU; row_ptr/col are torch CUDA tensors."""
+def rmat_gpu_ranged(scale: int, tuples: int, seed: int = 1, permute: bool = False, device: int = 0,
+                    max_pass_keys: int | None = None) -> Graph:
+    """Same graph as rmat_cpu, generated on the GPU one source-vertex range at a time (for graphs whose
+    key arrays exceed device memory, e.g. BASELINE configs[4]); row_ptr/col are torch CUDA tensors
+    (col is a view of an allocation sized for every key before deduplication)."""
     import torch
 
     lib = _lib()
     torch.cuda.set_device(device)
+    total, mx = ctypes.c_uint64(), ctypes.c_uint64()
+    if lib.ltgen_rmat_gpu_count(scale, tuples, seed, int(permute), ctypes.byref(total), ctypes.byref(mx)) != 0:
+        raise RuntimeError("ltgen_rmat_gpu_count failed: " + lib.ltgen_gpu_last_error().decode())
+    row_ptr = torch.empty((1 << scale) + 1, dtype=torch.int64, device="cuda")
+    col = torch.empty(max(total.value, 1), dtype=torch.int32, device="cuda")
+    if max_pass_keys is None:  # pass buffers: 2 x 8 B keys + 1 B flag + sort scratch per key
+        free, _ = torch.cuda.mem_get_info()
+        max_pass_keys = max(int(mx.value), int(0.6 * free / 20))
+    n, m, md, am, passes = (ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32(),
+                            ctypes.c_uint32())
+    rc = lib.ltgen_rmat_gpu_into(scale, tuples, seed, int(permute), int(max_pass_keys), row_ptr.data_ptr(),
+                                 col.data_ptr(), total.value, ctypes.byref(n), ctypes.byref(m), ctypes.byref(md),
+                                 ctypes.byref(am), ctypes.byref(passes))
+    if rc != 0:
+        raise RuntimeError("ltgen_rmat_gpu_into failed: " + lib.ltgen_gpu_last_error().decode())
+    g = Graph(int(n.value), int(m.value), row_ptr[: n.value + 1], col[: m.value], int(md.value), int(am.value))
+    g.passes = int(passes.value)
+    return g
+
+
+def rmat_gpu(scale: int, tuples: int, seed: int = 1, permute: bool = False, device: int = 0) -> Graph:
+    """Same graph as rmat_cpu, generated on the GPU; row_ptr/col are torch CUDA tensors. Falls back to
+    the ranged build when the one-shot key arrays (about 40 B per tuple) do not fit."""
+    import torch
+
+    lib = _lib()
+    torch.cuda.set_device(device)
+    free, _ = torch.cuda.mem_get_info(device)
+    if 44 * tuples > 0.8 * free:
+        return rmat_gpu_ranged(scale, tuples, seed, permute, device)
     n = ctypes.c_uint32()
     m = ctypes.c_uint64()
     drp = ctypes.c_void_p()

@@ -1,6 +1,7 @@
 // lt_kernels.cu — sm_100a kernels of the partition-centric walk-update path.
 //
-//   k_init      a2: write path[w][0], bin each new walk into its start partition's bucket (a5)
+//   k_init      a2: bin each new walk into its start partition's bucket (a5); path[w][0] is written by the
+//               update kernel's first sector store (or here, in the per-step path mode)
 //   k_update    a3+a4+a5: Alg. 1 re-designed for B200. A warp takes 32 records of
 //               partition k's bucket (one coalesced 512-B read of 16-B records); each lane steps its
 //               walk (Philox4x32-10 + Lemire; gathers of row_ptr[v], row_ptr[v+1], col[...]; path
@@ -218,7 +219,9 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
       dest = find_partition(B, wk.P, v);
       have = dest >= p.own.own_lo && dest < p.own.own_hi;
       if (have) {
-        wk.paths[i * wk.pitch] = v;
+        // path[w][0]: with buffered path stores (path_mode 0) the update kernel writes the walk's first
+        // sector, entry 0 included, on the walk's first visit, so only the per-step mode stores it here
+        if (wk.path_mode == 1) wk.paths[i * wk.pitch] = v;
         if (wk.visits32) atomicAdd(wk.visits32 + v, 1u);  // the start is the walk's first visit
         else if (wk.visits) atomicAdd(wk.visits + v, 1ull);
         rec = make_uint4((uint32_t)i, v, 0u, 0u);
@@ -298,6 +301,31 @@ __device__ __forceinline__ void st_sector(uint32_t* dst, const uint32_t* v, cons
   d[1] = make_uint4(v[4], v[5], v[6], v[7]);
 #endif
 }
+// The per-step row_ptr pair of the CSR layout (LT_RP_HINT=1: L2 evict_last, so the offsets of hot
+// vertices survive the streaming col gathers and path stores).
+#ifndef LT_RP_HINT
+#define LT_RP_HINT 0
+#endif
+__device__ __forceinline__ unsigned long long ld_rp(const unsigned long long* p) {
+#if LT_RP_HINT == 1
+  unsigned long long v;
+  asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+               "ld.global.nc.L2::cache_hint.u64 %0, [%1], pol;\n\t}" : "=l"(v) : "l"(p));
+  return v;
+#elif LT_RP_HINT == 2  // 64-B DRAM fills instead of 128-B lines on a miss
+  unsigned long long v;
+  asm volatile("ld.global.nc.L2::64B.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+#elif LT_RP_HINT == 3
+  unsigned long long v;
+  asm volatile("{\n\t.reg .b64 pol;\n\tcreatepolicy.fractional.L2::evict_last.b64 pol, 1.0;\n\t"
+               "ld.global.nc.L2::cache_hint.L2::64B.u64 %0, [%1], pol;\n\t}" : "=l"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
+
 template <int GM>
 __device__ __forceinline__ uint32_t ld_col(const uint32_t* p, const Policies& pol) {
   if (GM == 0) return __ldg(p);
@@ -431,8 +459,9 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
             // the loaded graph may be one partition's slice (out-of-core pool block or a zero-copy
             // host view): row_ptr is indexed from vbase and col from ebase
             const unsigned long long* rp = wk.row_ptr + (rec[s].y - wk.vbase);
-            off[s] = __ldg(rp) - wk.ebase;
-            d[s] = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
+            const unsigned long long r0 = ld_rp(rp), r1 = ld_rp(rp + 1);
+            off[s] = r0 - wk.ebase;
+            d[s] = (uint32_t)(r1 - r0);
           }
         }
       }
@@ -649,12 +678,13 @@ __global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_
         if (LAY == 0) {
           if (CONT) {
             const unsigned long long* rp = c_rp + rec.y;
-            off = __ldg(rp);
-            d = (uint32_t)(__ldg(rp + 1) - off);
+            off = ld_rp(rp);
+            d = (uint32_t)(ld_rp(rp + 1) - off);
           } else {
             const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
-            off = __ldg(rp) - wk.ebase;
-            d = (uint32_t)(__ldg(rp + 1) - __ldg(rp));
+            const unsigned long long r0 = ld_rp(rp), r1 = ld_rp(rp + 1);
+            off = r0 - wk.ebase;
+            d = (uint32_t)(r1 - r0);
           }
         }
         const uint64_t wid = wk.first_walk_id + rec.x;

@@ -83,3 +83,21 @@ def test_gpu_generator_equals_cpu(gpu, scale, tuples, permute):
     assert (g.n, g.m, g.max_deg, g.argmax_deg) == (c.n, c.m, c.max_deg, c.argmax_deg)
     np.testing.assert_array_equal(g.row_ptr.cpu().numpy().view(np.uint64), c.row_ptr)
     np.testing.assert_array_equal(g.col.cpu().numpy().view(np.uint32), c.col)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("scale,tuples,permute,max_pass", [(12, 65536, False, 40_000), (15, 300_000, True, 70_000),
+                                                          (16, 16 * 65536, False, 10 ** 9), (14, 200_000, True, 400)])
+def test_ranged_gpu_generator_equals_cpu(gpu, scale, tuples, permute, max_pass):
+    """The ranged build (one source range per pass; configs[4] at scale 28) produces the same CSR as the
+    CPU build, with one pass or many (max_pass keys per pass), R-MAT and Kronecker."""
+    c = lt_inputs.rmat_cpu(scale, tuples, seed=1, permute=permute)
+    if max_pass == 400:  # smaller than the fullest source bin: refused, not truncated
+        with pytest.raises(RuntimeError):
+            lt_inputs.rmat_gpu_ranged(scale, tuples, seed=1, permute=permute, max_pass_keys=max_pass)
+        return
+    g = lt_inputs.rmat_gpu_ranged(scale, tuples, seed=1, permute=permute, max_pass_keys=max_pass)
+    assert (g.n, g.m, g.max_deg, g.argmax_deg) == (c.n, c.m, c.max_deg, c.argmax_deg)
+    assert (g.passes > 1) == (max_pass < 2 * tuples)
+    np.testing.assert_array_equal(g.row_ptr.cpu().numpy().view(np.uint64), c.row_ptr)
+    np.testing.assert_array_equal(g.col.cpu().numpy().view(np.uint32), c.col)
