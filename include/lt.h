@@ -123,7 +123,15 @@ typedef struct lt_config {
                                  partition resident in the graph pool keeps stepping there instead of
                                  being appended to its bucket (parity-neutral);
                                  uses the lane-refill kernel. Ignored when the graph is HBM-resident. */
-  uint32_t reserved[3];
+  uint32_t reserved0;
+  uint64_t walk_pool_walks;   /* m_w, the walk pool's capacity in walks (D4; SURVEY.md
+                                 8(f) f3): 0 -> sized for all W walks. When W > m_w the walks are
+                                 admitted in index order as the pool drains: lt_walks_init creates the
+                                 first m_w, and the scheduler admits more whenever walks have ended, so
+                                 at most m_w walks are ever live and the pool holds 2 m_w records
+                                 (+ per-bucket slack) however large W is. Single-rank contexts only.
+                                 Paths are unchanged. */
+  uint32_t reserved[2];
 } lt_config;
 
 typedef struct lt_stats {
@@ -153,6 +161,8 @@ typedef struct lt_stats {
   uint64_t graph_h2d_bytes;    /* CSR bytes copied host -> device by the scheduler */
   uint64_t pool_blocks;        /* m_g */
   uint64_t pool_block_bytes;
+  uint64_t admissions;         /* walk admissions (lt_walks_init's included) in the last init + run */
+  uint64_t peak_live;          /* most live walks seen at a scheduler step */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

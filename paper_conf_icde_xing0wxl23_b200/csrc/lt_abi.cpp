@@ -415,6 +415,8 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   } else if (app != LT_APP_DEEPWALK) {
     return fail(LT_ERR_INVALID, "unknown app");
   }
+  if (ctx->cfg.walk_pool_walks && ctx->world != 1)
+    return fail(LT_ERR_INVALID, "walk_pool_walks (walk admission) needs a single-rank context");
   ctx->walks_ready = false;
   ctx->visits_ready = false;
   ctx->ran = false;
@@ -435,12 +437,15 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const uint64_t C = ctx->cfg.chunk_walks;
   uint32_t c_shift = 0;
   while ((1ull << c_shift) < C) ++c_shift;
-  const uint64_t wc = (W + C - 1) / C;
+  // walk pool: sized for the walks that can be live at once
+  const uint64_t cap = (ctx->cfg.walk_pool_walks && ctx->cfg.walk_pool_walks < W) ? ctx->cfg.walk_pool_walks : W;
+  const uint64_t wc = (cap + C - 1) / C;
   const uint64_t ring_len = wc + 2;
   const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
   const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
-  CK(ensure(ctx->d_paths, ctx->paths_cap, std::max<uint64_t>(W, 1) * pitch));
+  // path_mode 2 stores no path entries (the paper's accounting): no path matrix
+  CK(ensure(ctx->d_paths, ctx->paths_cap, ctx->cfg.path_mode == 2 ? 8 : std::max<uint64_t>(W, 1) * pitch));
   CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
   CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
   CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
@@ -531,9 +536,15 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
   if (W && ctx->world > 1) CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
-  if (W) {
-    CK(lt::launch_init(p, d_starts, W, s));
+  ctx->adm_starts = d_starts;
+  ctx->cap_walks = cap;
+  ctx->admitted = cap;
+  ctx->stats.admissions = 0;
+  ctx->stats.peak_live = cap;
+  if (cap) {
+    CK(lt::launch_init(p, d_starts, cap, 0, s));
     ctx->stats.kernel_launches++;
+    ctx->stats.admissions = 1;
   }
   CK(cudaEventRecord(ctx->ev_b, s));
   ctx->walks_ready = true;
@@ -609,16 +620,22 @@ static lt_status need_ran(lt_ctx* ctx) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
   CK(cudaSetDevice(ctx->cfg.device));
-  if (!ctx->padded) {  // pad unused path slots with 0xFFFFFFFF once, before the first copy-out
+  if (!ctx->padded && ctx->cfg.path_mode != 2) {  // pad unused path slots with 0xFFFFFFFF once, before the first copy-out
     CK(lt::launch_finalize_paths(ctx->params, ctx->W, ctx->stream));
     ctx->padded = true;
   }
   return LT_OK;
 }
 
+static lt_status need_paths(lt_ctx* ctx) {
+  if (ctx->cfg.path_mode == 2) return fail(LT_ERR_STATE, "paths are not stored (path_mode 2)");
+  return LT_OK;
+}
+
 lt_status lt_get_paths(lt_ctx* ctx, uint32_t* paths, uint32_t* lengths) {
   lt_status st = need_ran(ctx);
   if (st != LT_OK) return st;
+  if (paths && (st = need_paths(ctx)) != LT_OK) return st;
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
   if (paths && ctx->W) {
@@ -637,6 +654,7 @@ lt_status lt_get_paths(lt_ctx* ctx, uint32_t* paths, uint32_t* lengths) {
 lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, uint32_t* paths, uint32_t* lengths) {
   lt_status st = need_ran(ctx);
   if (st != LT_OK) return st;
+  if ((st = need_paths(ctx)) != LT_OK) return st;
   if (count && (!rows || !paths || !lengths)) return fail(LT_ERR_INVALID, "NULL argument");
   for (uint64_t i = 0; i < count; ++i)
     if (rows[i] >= ctx->W) return fail(LT_ERR_INVALID, "row index >= W");
@@ -664,6 +682,7 @@ lt_status lt_get_paths_rows(lt_ctx* ctx, const uint64_t* rows, uint64_t count, u
 lt_status lt_get_paths_device(lt_ctx* ctx, uint32_t* d_paths, uint32_t* d_lengths) {
   lt_status st = need_ran(ctx);
   if (st != LT_OK) return st;
+  if (d_paths && (st = need_paths(ctx)) != LT_OK) return st;
   CK(cudaSetDevice(ctx->cfg.device));
   cudaStream_t s = ctx->stream;
   if (d_paths && ctx->W)
@@ -699,6 +718,7 @@ lt_status lt_get_paths_compact(lt_ctx* ctx, uint64_t* offsets, uint32_t* vertice
                                uint64_t* total) {
   if (!ctx || !offsets || !total) return fail(LT_ERR_INVALID, "NULL argument");
   if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
+  if (need_paths(ctx) != LT_OK) return LT_ERR_STATE;
   CK(cudaSetDevice(ctx->cfg.device));
   uint64_t tot = 0;
   lt_status st = pack_compact(ctx, ctx->d_paths, ctx->d_lengths, ctx->W, 0, 0, &tot);
@@ -805,6 +825,7 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
   if (compact && vcap && !vertices) return fail(LT_ERR_INVALID, "NULL vertices");
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_run_to_host before lt_graph_load");
   if (ctx->cfg.visit_counts) return fail(LT_ERR_INVALID, "lt_run_to_host does not accumulate visit counts; use lt_run");
+  if (ctx->cfg.path_mode == 2) return fail(LT_ERR_INVALID, "lt_run_to_host needs stored paths (path_mode 0 or 1)");
   CK(cudaSetDevice(ctx->cfg.device));
   if (chunks == 0) chunks = 8;
   const uint64_t wc = std::max<uint64_t>((W + chunks - 1) / chunks, 1);

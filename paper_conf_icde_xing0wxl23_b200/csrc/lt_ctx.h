@@ -89,6 +89,10 @@ struct lt_ctx {
   bool visits_ready = false;
   uint32_t* d_starts = nullptr;
   size_t starts_cap = 0;
+  // walk admission (lt_config.walk_pool_walks): walks [0, admitted) have been created; at most
+  // cap_walks are live; the rest are admitted from adm_starts as walks end
+  const uint32_t* adm_starts = nullptr;
+  uint64_t admitted = 0, cap_walks = 0;
   // pool
   uint4* d_slots = nullptr;
   size_t slots_cap = 0;
@@ -142,4 +146,6 @@ lt_status snapshot(lt_ctx* ctx);  // h_hc / h_ctr / h_free <- device, then sync 
 lt_status run_resident(lt_ctx* ctx);
 lt_status run_out_of_core(lt_ctx* ctx);
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound);
+// admit walks while live < cap_walks (returns true in *did if any were admitted)
+lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did);
 }  // namespace lt

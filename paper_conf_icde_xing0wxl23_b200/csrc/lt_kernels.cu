@@ -202,7 +202,8 @@ __device__ __forceinline__ uint32_t bucket_of(const Params& p, uint32_t q) {
 // ------------------------------------------------------------------------------------------ a2
 // Walk init: path[w][0] and insertion into the start partition's bucket. With range ownership
 // (world > 1) every rank sees every start and keeps the walks whose start partition it owns.
-__global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restrict__ starts, uint64_t W) {
+__global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restrict__ starts, uint64_t W,
+                                              uint64_t first_row) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
   const uint32_t* B = stage_bounds(wk, s_bounds);
@@ -210,12 +211,13 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
   const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
   for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; base < W;
        base += nwarps * 32) {
-    const uint64_t i = base + lane;
-    bool have = i < W;
+    const uint64_t j = base + lane;  // walk j of this admission = row first_row + j
+    const uint64_t i = first_row + j;
+    bool have = j < W;
     uint4 rec = make_uint4(0, 0, 0, 0);
     uint32_t dest = 0;
     if (have) {
-      const uint32_t v = starts[i];
+      const uint32_t v = starts[j];
       dest = find_partition(B, wk.P, v);
       have = dest >= p.own.own_lo && dest < p.own.own_hi;
       if (have) {
@@ -1031,11 +1033,11 @@ cudaError_t launch_pack(const Params& p, uint32_t bucket, uint4* out, uint64_t c
   return cudaGetLastError();
 }
 
-cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, cudaStream_t s) {
+cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, uint64_t first_row, cudaStream_t s) {
   uint64_t want = (W + 255) / 256;
   uint32_t grid = (uint32_t)std::min<uint64_t>(want ? want : 1, (uint64_t)num_sms() * 8);
   cudaFuncSetAttribute(k_init, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-  k_init<<<grid, 256, bounds_smem(p), s>>>(p, starts, W);
+  k_init<<<grid, 256, bounds_smem(p), s>>>(p, starts, W, first_row);
   return cudaGetLastError();
 }
 

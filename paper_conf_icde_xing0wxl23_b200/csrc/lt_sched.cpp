@@ -51,6 +51,23 @@ lt_status snapshot(lt_ctx* ctx) {
   return LT_OK;
 }
 
+// Walk admission (f3; lt_config.walk_pool_walks): create the next walks in index order once at least a
+// quarter of the pool (or everything still to come) has room, so live walks never exceed cap_walks.
+lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did) {
+  *did = false;
+  ctx->stats.peak_live = std::max<uint64_t>(ctx->stats.peak_live, live);
+  if (ctx->admitted >= ctx->W || live >= ctx->cap_walks) return LT_OK;
+  const uint64_t room = ctx->cap_walks - live, rest = ctx->W - ctx->admitted;
+  if (room < std::min<uint64_t>(rest, std::max<uint64_t>(ctx->cap_walks / 4, 1))) return LT_OK;
+  const uint64_t n = std::min(room, rest);
+  CK(launch_init(ctx->params, ctx->adm_starts + ctx->admitted, n, ctx->admitted, ctx->stream));
+  ctx->admitted += n;
+  ctx->stats.admissions++;
+  ctx->stats.kernel_launches++;
+  *did = true;
+  return LT_OK;
+}
+
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
   cudaStream_t s = ctx->stream;
   const uint64_t max_grid = (uint64_t)ctx->num_sms * ctx->occ;
@@ -75,9 +92,10 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
 }
 
 lt_status run_resident(lt_ctx* ctx) {
-  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
+  const uint64_t max_len = (ctx->app == LT_APP_PPR) ? ctx->lmax : ctx->length;
   std::vector<uint32_t> order;
   order.reserve(ctx->P);
+  uint64_t since_admission = 0;
   for (;;) {
     lt_status st = read_counts(ctx);  // one small D2H + sync per sweep
     if (st != LT_OK) return st;
@@ -86,9 +104,16 @@ lt_status run_resident(lt_ctx* ctx) {
     uint64_t total = 0;
     for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k)  // owned partitions (all when world == 1)
       if (pending(ctx, k)) { order.push_back(k); total += pending(ctx, k); }
+    bool admitted = false;
+    st = admit_walks(ctx, total, &admitted);
+    if (st != LT_OK) return st;
+    if (admitted) {  // recount with the new walks in their buckets
+      since_admission = 0;
+      continue;
+    }
     if (total == 0) return LT_OK;
-    // every live walk advances >= 1 step per sweep, so sweeps <= max_len + 1
-    if (ctx->stats.sweeps > max_len + 2) return fail(LT_ERR_CUDA, "scheduler did not converge");
+    // every live walk advances >= 1 step per sweep, so sweeps <= max_len + 1 between admissions
+    if (++since_admission > max_len + 3) return fail(LT_ERR_CUDA, "scheduler did not converge");
     if (ctx->cfg.policy == LT_POLICY_SELECTIVE || ctx->cfg.policy == LT_POLICY_SELECTIVE_ONLY)
       std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return pending(ctx, a) > pending(ctx, b); });
     uint64_t earlier = 0;
@@ -212,7 +237,7 @@ lt_status run_out_of_core(lt_ctx* ctx) {
   const bool selective = pol == LT_POLICY_SELECTIVE || pol == LT_POLICY_SELECTIVE_ONLY;
   const bool preemptive = pol == LT_POLICY_SELECTIVE || pol == LT_POLICY_PREEMPTIVE_ONLY;
   const uint64_t alpha = ctx->cfg.zc_alpha_bytes ? ctx->cfg.zc_alpha_bytes : 256;
-  const uint64_t max_len = (ctx->app == LT_APP_DEEPWALK) ? ctx->length : ctx->lmax;
+  const uint64_t max_len = (ctx->app == LT_APP_PPR) ? ctx->lmax : ctx->length;
   // each iteration consumes >= 1 visit and a walk makes <= max_len + 1 visits
   const uint64_t max_iters = ctx->W * (max_len + 1) + P + 64;
   uint64_t seq = 0;
@@ -224,6 +249,10 @@ lt_status run_out_of_core(lt_ctx* ctx) {
     if (ctx->h_ctr->err) return LT_OK;
     uint64_t total = 0;
     for (uint32_t k = lo; k < hi; ++k) total += pending(ctx, k);
+    bool admitted = false;
+    st = admit_walks(ctx, total, &admitted);
+    if (st != LT_OK) return st;
+    if (admitted) continue;
     if (total == 0) return LT_OK;
     if (ctx->stats.iterations > max_iters) return fail(LT_ERR_CUDA, "out-of-core scheduler did not converge");
     // scheduler.iteration(): select partition i
