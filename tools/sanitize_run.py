@@ -1,7 +1,8 @@
 #!/usr/bin/env python3
 """Small runs of every kernel path for compute-sanitizer (memcheck / racecheck / synccheck /
 initcheck): resident P=1 (refill), P=4 (batch kernel, CSR and ADJ), PPR, out-of-core with zero copy,
-two-rank ownership, streamed run_to_host."""
+two-rank ownership, streamed run_to_host (dense and ragged), ragged copy-out, PageRank with u32 / u64
+visit counters, out-of-core continuation, walk admission, paths off."""
 import os
 import sys
 import threading
@@ -33,6 +34,31 @@ with LT.Engine(graph_pool_bytes=1 << 20, zero_copy=True, chunk_walks=256) as e:
 with LT.Engine() as e:
     e.graph_load(g.row_ptr, g.col, 1)
     e.run_to_host(starts, LT.DEEPWALK, 10, 1, chunks=3)
+    e.run_to_host_compact(pstarts, LT.PPR, 0.15, 1, chunks=3)
+    e.walks_init(pstarts, LT.PPR, 0.15, 2)
+    e.run()
+    e.get_paths_compact()
+# PageRank with fused visit counters (u32 and u64), the CSR and ADJ layouts, P = 1 and P = 4
+for kw in [dict(P=1, visit_counts=1), dict(P=4, visit_counts=2, layout=LT.LAYOUT_CSR), dict(P=4, visit_counts=1)]:
+    P = kw.pop("P")
+    with LT.Engine(chunk_walks=256, **kw) as e:
+        e.graph_load(g.row_ptr, g.col, P)
+        e.walks_init_pagerank(starts, 10, 0.2, 1)
+        e.run()
+        e.get_paths()
+        e.visit_counts()
+# out of core with continuation into resident partitions, and walk admission under a pool cap
+with LT.Engine(graph_pool_bytes=1 << 20, zero_copy=True, continue_resident=True, chunk_walks=256,
+               walk_pool_walks=1000) as e:
+    e.graph_load(g.row_ptr, g.col, 8)
+    e.walks_init(starts, LT.DEEPWALK, 10, 1)
+    e.run()
+    e.get_paths()
+with LT.Engine(path_mode=2, walk_pool_walks=500, chunk_walks=64, visit_counts=True) as e:
+    e.graph_load(g.row_ptr, g.col, 3)
+    e.walks_init_pagerank(starts, 10, 0.2, 1)
+    e.run()
+    e.get_paths(paths=False)
 hub = ltdist.ThreadComm.Hub(2)
 
 
