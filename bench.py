@@ -67,6 +67,8 @@ def parse():
     ap.add_argument("--ilp", type=int, default=0)
     ap.add_argument("--path-mode", type=int, default=0)
     ap.add_argument("--refill", type=int, default=0)
+    ap.add_argument("--direct-start", type=int, default=1,
+                    help="1: with P == 1 the update kernel takes new walks straight from starts (no records)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--sweep", default="", help="comma list of P values to time (extra key)")
@@ -322,7 +324,7 @@ def main():
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill,
-                    continue_resident=bool(args.continue_resident))
+                    continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start))
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
@@ -603,6 +605,7 @@ def main():
                 "per_step": {"steps": last["steps"], "visits": last["visits"], "sweeps": last["sweeps"],
                              "update_launches": last["update_launches"], "run_ms": last["run_ms"],
                              "init_ms": last["init_ms"], "update_ms": last["update_ms"],
+                             "direct_start": bool(last["direct_start"]),
                              "chunks_total": last["chunks_total"], "chunks_free_min": last["chunks_free_min"]}}
         if share:
             line["config"]["shared_device_test"] = "all ranks on cuda:0 over gloo: launch test, not a measurement"

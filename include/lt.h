@@ -131,7 +131,12 @@ typedef struct lt_config {
                                  at most m_w walks are ever live and the pool holds 2 m_w records
                                  (+ per-bucket slack) however large W is. Single-rank contexts only.
                                  Paths are unchanged. */
-  uint32_t reserved[2];
+  uint32_t direct_start;      /* 0 auto: with one partition, one rank, an HBM-resident graph and no walk
+                                 pool cap, lt_walks_init writes no walk records: the update kernel
+                                 takes walk j straight from starts[j] (device starts must then stay
+                                 valid until lt_run returns, as with walk admission); 1 -> off (records
+                                 always built by the init kernel). Parity-neutral. */
+  uint32_t reserved1;
 } lt_config;
 
 typedef struct lt_stats {
@@ -163,6 +168,7 @@ typedef struct lt_stats {
   uint64_t pool_block_bytes;
   uint64_t admissions;         /* walk admissions (lt_walks_init's included) in the last init + run */
   uint64_t peak_live;          /* most live walks seen at a scheduler step */
+  uint64_t direct_start;       /* 1 if the last lt_walks_init* used the direct start (no walk records) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,
@@ -196,7 +202,9 @@ lt_status lt_get_bounds(lt_ctx* ctx, uint32_t* bounds, uint32_t* P);
 /* Create W walks (a2): walk i has ID first_walk_id + i (the Philox key counter), starts at
  * starts[i] < n, and is appended to the bucket of its start's partition. length_or_alpha is the
  * DeepWalk length l (a non-negative integer) or the PPR alpha in (0, 1). starts is host memory
- * (lt_walks_init) or device memory (lt_walks_init_device). W < 2^32 - 1. */
+ * (lt_walks_init; copied before the call returns) or device memory (lt_walks_init_ex with
+ * starts_on_device = 1; borrowed: it must stay valid and unchanged until lt_run returns, because walk
+ * admission and the direct start read it during the run). W < 2^32 - 1. */
 lt_status lt_walks_init(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, lt_app app,
                         double length_or_alpha, uint64_t seed);
 lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t num_walks, const uint32_t* starts, int starts_on_device,

@@ -57,6 +57,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
   if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
   if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
+  if (c.direct_start > 1) return fail(LT_ERR_INVALID, "direct_start must be 0 (auto) or 1 (off)");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -439,7 +440,13 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   while ((1ull << c_shift) < C) ++c_shift;
   // walk pool: sized for the walks that can be live at once
   const uint64_t cap = (ctx->cfg.walk_pool_walks && ctx->cfg.walk_pool_walks < W) ? ctx->cfg.walk_pool_walks : W;
-  const uint64_t wc = (cap + C - 1) / C;
+  // direct start (lt_config.direct_start): with one partition every new walk belongs to bucket 0, so
+  // the lane-refill kernel (the P == 1 default) takes walk j straight from starts[j]: k_init (16-B
+  // record write + read back + one bucket cursor atomic per warp) is skipped and, since a walk never
+  // leaves the only partition, no record is ever appended: the pool keeps only its per-bucket slack
+  const bool direct = ctx->cfg.direct_start == 0 && (ctx->cfg.refill == 0 || ctx->cfg.refill == 2) && ctx->P == 1 &&
+                      ctx->world == 1 && !ctx->ooc.on && cap == W;
+  const uint64_t wc = direct ? 0 : (cap + C - 1) / C;
   const uint64_t ring_len = wc + 2;
   const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
@@ -514,6 +521,8 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0);
+  p.direct = direct ? lt::Direct{d_starts, W} : lt::Direct{nullptr, 0};
+  ctx->stats.direct_start = direct ? 1 : 0;
 
   ctx->W = W;
   ctx->first = first_walk_id;
@@ -542,8 +551,10 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.admissions = 0;
   ctx->stats.peak_live = cap;
   if (cap) {
-    CK(lt::launch_init(p, d_starts, cap, 0, s));
-    ctx->stats.kernel_launches++;
+    if (!direct) {
+      CK(lt::launch_init(p, d_starts, cap, 0, s));
+      ctx->stats.kernel_launches++;
+    }
     ctx->stats.admissions = 1;
   }
   CK(cudaEventRecord(ctx->ev_b, s));

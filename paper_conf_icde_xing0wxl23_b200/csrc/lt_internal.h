@@ -81,12 +81,22 @@ struct Cont {
   uint64_t block_bytes, rp_bytes;
 };
 
+// Direct start (one partition, one rank, every walk admitted at once): bucket 0 holds the W new walks
+// as VIRTUAL positions [0, W) — no record is written by k_init; the lane-refill kernel builds the
+// record of position j in registers as {j, starts[j], 0, 0}. Positions past W (none with one
+// partition: a walk never leaves it) would be real slots. starts == nullptr: off.
+struct Direct {
+  const uint32_t* starts;
+  unsigned long long count;
+};
+
 struct Params {
   Walk wk;
   Cont cont;
   Pool pool;
   Counters* ctr;
   Owner own;
+  Direct direct;
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;

@@ -168,8 +168,9 @@ __device__ void last_cta_retire(const Params& p, int k, unsigned long long head,
       uint32_t* slot = pl.ring + (uint64_t)k * pl.ring_len + (ci % pl.ring_len);
       const uint32_t c = *(volatile uint32_t*)slot;
       *(volatile uint32_t*)slot = kEmpty;
+      if (c >= pl.num_chunks) continue;  // a direct-start bucket's virtual chunk (or the trash chunk)
       const int idx = atomicAdd(pl.free_top, 1);
-      if (idx >= 0 && c < pl.num_chunks) pl.free_list[idx] = c;
+      if (idx >= 0) pl.free_list[idx] = c;
     }
   }
   __syncthreads();
@@ -647,8 +648,14 @@ __global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_
       const uint32_t r = __popc(need & lanemask_lt());
       if (!has && r < avail) {
         const unsigned long long pos = q_cur + r;
-        const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
-        rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
+        if (pos < p.direct.count) {  // direct start: the new walk's record, built in registers (a2)
+          rec = make_uint4((uint32_t)pos, __ldg(p.direct.starts + pos), 0u, 0u);
+          if (wk.path_mode == 1) wk.paths[pos * wk.pitch] = rec.y;
+          count_visit<VIS>(wk, rec.y, pol_last);  // the start is the walk's first visit
+        } else {
+          const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
+          rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
+        }
         has = true;
         prow = wk.paths + (uint64_t)rec.x * wk.pitch;
         pb[7] = rec.y;
@@ -963,7 +970,11 @@ __global__ void k_pool_reset(Params p) {
   for (uint64_t i = tid; i < pl.num_chunks; i += stride) pl.free_list[i] = (uint32_t)i;
   const uint64_t nring = (uint64_t)pl.nbuckets * pl.ring_len;
   for (uint64_t i = tid; i < nring; i += stride) pl.ring[i] = kEmpty;
-  for (uint64_t i = tid; i < pl.nbuckets; i += stride) { pl.head[i] = 0; pl.cursor[i] = 0; pl.claim[i] = 0; }
+  for (uint64_t i = tid; i < pl.nbuckets; i += stride) {
+    pl.head[i] = 0;
+    pl.cursor[i] = (i == 0 && p.direct.starts) ? p.direct.count : 0;  // direct start: W virtual positions
+    pl.claim[i] = 0;
+  }
   if (tid == 0) {
     *pl.free_top = (int)pl.num_chunks;
     p.ctr->steps = 0; p.ctr->visits = 0; p.ctr->truncated = 0; p.ctr->err = 0; p.ctr->done_ctas = 0;

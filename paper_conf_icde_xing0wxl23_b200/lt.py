@@ -64,7 +64,8 @@ class Config(ctypes.Structure):
         ("continue_resident", ctypes.c_uint32),
         ("reserved0", ctypes.c_uint32),
         ("walk_pool_walks", ctypes.c_uint64),
-        ("reserved", ctypes.c_uint32 * 2),
+        ("direct_start", ctypes.c_uint32),
+        ("reserved1", ctypes.c_uint32),
     ]
 
 
@@ -76,7 +77,7 @@ class Stats(ctypes.Structure):
         ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
-            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live")]
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start")]
 
 
 class PoolState(ctypes.Structure):
@@ -169,7 +170,8 @@ class Engine:
                  gather_mode: int = 3, ilp: int = 0, layout: int = LAYOUT_AUTO,
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
-                 visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0):
+                 visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
+                 direct_start: bool = True):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -193,6 +195,7 @@ class Engine:
         cfg.refill = refill
         cfg.continue_resident = int(bool(continue_resident))
         cfg.walk_pool_walks = int(walk_pool_walks)
+        cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
         cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device

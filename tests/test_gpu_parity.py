@@ -27,7 +27,8 @@ def run_gpu(g, starts, app, param, seed, P, first=0, device_inputs=False, **cfg)
             e.graph_load(g.row_ptr, g.col, P)
             e.walks_init(starts, app, param, seed, first)
         e.run()
-        paths, lengths = e.get_paths()
+        # path_mode 2 stores no path matrix: only the lengths can be read back
+        paths, lengths = e.get_paths(paths=False if cfg.get("path_mode") == 2 else None)
         return paths, lengths, e.stats(), e.bounds()
 
 
@@ -256,6 +257,44 @@ def test_path_mode_off_keeps_lengths(gpu, cfg1):
     _, ol, osteps, _ = run_oracle(cfg1, starts, LT.PPR, 0.15, 4)
     np.testing.assert_array_equal(lengths, ol)
     assert st["steps"] == osteps
+
+
+@pytest.mark.parametrize("direct", [True, False])
+@pytest.mark.parametrize("path_mode", [0, 1])
+@pytest.mark.parametrize("device_inputs", [False, True])
+def test_direct_start(gpu, cfg1, direct, path_mode, device_inputs):
+    """Direct start (lt_config.direct_start; P == 1): no walk records are written at init, the update
+    kernel builds walk j's record from starts[j]. Paths, lengths, steps, visits and the pool invariants
+    are those of the record path; the stats say which path ran."""
+    W = 5003  # several refill claims of 64 and a ragged tail
+    for app, param, starts in ((LT.DEEPWALK, 17, lt_inputs.deepwalk_starts(W, cfg1.n)),
+                               (LT.PPR, 0.15, lt_inputs.ppr_starts(W, cfg1.argmax_deg))):
+        st = assert_parity(cfg1, starts, app, param, 9, P=1, first=123, path_mode=path_mode,
+                           device_inputs=device_inputs, direct_start=direct)
+        assert st["direct_start"] == (1 if direct else 0)
+        assert st["visits"] == W and st["admissions"] == 1
+    # never with several partitions, a walk-pool cap or the per-walk kernel without refill
+    st = assert_parity(cfg1, lt_inputs.deepwalk_starts(W, cfg1.n), LT.DEEPWALK, 5, 9, P=2, direct_start=direct)
+    assert st["direct_start"] == 0
+    st = assert_parity(cfg1, lt_inputs.deepwalk_starts(W, cfg1.n), LT.DEEPWALK, 5, 9, P=1, refill=1,
+                       direct_start=direct)
+    assert st["direct_start"] == 0
+    with LT.Engine(direct_start=direct, chunk_walks=64) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 1)
+        e.walks_init(lt_inputs.deepwalk_starts(W, cfg1.n), LT.DEEPWALK, 6, 2)
+        s0 = e.pool_state()
+        assert s0["pending"] == W and s0["device_err"] == 0, s0
+        assert s0["free_chunks"] + s0["ring_chunks"] == s0["total_chunks"], s0
+        e.run()
+        s1 = e.pool_state()
+        assert s1["pending"] == 0 and s1["device_err"] == 0, s1
+        assert s1["free_chunks"] + s1["ring_chunks"] == s1["total_chunks"], s1
+        assert s1["ring_chunks"] == (0 if direct else 1), s1  # direct: no chunk was ever installed
+        # a second epoch on the same context (the pool is reset by lt_walks_init)
+        e.walks_init(lt_inputs.deepwalk_starts(W, cfg1.n), LT.DEEPWALK, 6, 3)
+        e.run()
+        _, l2 = e.get_paths(paths=False)
+        assert np.all(l2 == 7)
 
 
 @pytest.mark.parametrize("chunks", [1, 3, 8])
