@@ -63,8 +63,12 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--e2e-chunks", type=int, default=16, help="lt_run_to_host walk ranges (copy-out overlap)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="oracle sample budget")
-    ap.add_argument("--layout", type=int, default=0, help="0 auto, 1 CSR, 2 ADJ (lt_layout)")
+    ap.add_argument("--layout", type=int, default=0, help="0 auto, 1 CSR, 2 ADJ, 3 ADJ12 (lt_layout)")
+    ap.add_argument("--release-col", type=int, default=1,
+                    help="1: once an augmented layout is built, keep a host copy of the CSR for the oracle legs "
+                         "and free the device col (the steps never read it): room for the path matrix")
     ap.add_argument("--ilp", type=int, default=0)
+    ap.add_argument("--gather-mode", type=int, default=3, help="lt_config.gather_mode: 3 L2 hints (default), 0 none")
     ap.add_argument("--path-mode", type=int, default=0)
     ap.add_argument("--refill", type=int, default=0)
     ap.add_argument("--direct-start", type=int, default=1,
@@ -320,14 +324,23 @@ def main():
 
     ooc = args.graph_pool_gb > 0
     vis = args.visit_counts == 1 or (args.visit_counts == -1 and c["app"] == "pagerank")
-    eng = LT.Engine(visit_counts=vis, device=local, chunk_walks=args.chunk_walks, policy=args.policy, insert_mode=args.insert_mode,
+    eng = LT.Engine(visit_counts=vis, device=local, chunk_walks=args.chunk_walks, policy=args.policy,
+                    insert_mode=args.insert_mode, gather_mode=args.gather_mode,
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill,
                     continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start))
+    torch.cuda.empty_cache()  # generator scratch back to the device before the library reserves its graph
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
+    g_host = None
+    if args.release_col and not ooc and eng.stats()["layout"] != LT.LAYOUT_CSR and not isinstance(g.col, np.ndarray) \
+            and not args.sweep:
+        if rank == 0 and world == 1 and not args.no_cpu_baseline:
+            g_host = host_graph(g)
+        g = lt_inputs.Graph(g.n, g.m, g.row_ptr, None, g.max_deg, g.argmax_deg)
+        torch.cuda.empty_cache()
 
     def barrier():
         torch.cuda.synchronize()
@@ -396,7 +409,8 @@ def main():
     layout = stats[-1]["layout"]
     # DRAM-missing random gathers issued by the update kernel: one per step (ADJ: adj entry;
     # CSR: col entry) + the row_ptr line per step (CSR) or per visit (ADJ)
-    gathers = steps_k * (1 if layout == LT.LAYOUT_ADJ else 2) + (visits if layout == LT.LAYOUT_ADJ else 0)
+    aug = layout in (LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12)
+    gathers = steps_k * (1 if aug else 2) + (visits if aug else 0)
     gather = None
     gc_path = os.path.join(ROOT, "profiles", "gather_ceiling.json")
     if upd_ms > 0:
@@ -567,7 +581,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         init_walks(eng, c, starts_d, args.seed, first)
         eng.run()
-        gh = host_graph(g)
+        gh = g_host if g_host is not None else host_graph(g)
         r = oracle_sample(c, gh, W, first, args.cpu_seconds)
         cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "kind": "oracle",
                "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
@@ -597,7 +611,7 @@ def main():
                                              "mode": "out_of_core" if ooc else "hbm_resident",
                                              "graph_pool_gb": args.graph_pool_gb if ooc else None,
                                              "l2": "inputs larger than L2 (CSR >> 126 MB); no flush",
-                                             "layout": "adj" if layout == LT.LAYOUT_ADJ else "csr",
+                                             "layout": {LT.LAYOUT_ADJ: "adj", LT.LAYOUT_ADJ12: "adj12"}.get(layout, "csr"),
                                              "graph_gen_s": round(gen_s, 2), "graph_load_s": round(load_s, 2),
                                              "graph_prep_ms": stats[-1]["graph_prep_ms"]}),
                 "clocks": ck, "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),

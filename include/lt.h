@@ -77,9 +77,16 @@ typedef enum {
 } lt_insert_mode;
 
 typedef enum {
-  LT_LAYOUT_AUTO = 0, /* ADJ when 16 B x m fits in half of the free device memory, else CSR */
+  LT_LAYOUT_AUTO = 0, /* ADJ when 16 B x m fits in half of the free device memory and in the 64 GiB
+                         a random gather can span at full rate on B200 (address-translation reach,
+                         measured), else ADJ12 under the same two limits (when it applies), else CSR */
   LT_LAYOUT_CSR = 1,  /* steps gather row_ptr[v], row_ptr[v+1] and col[row_ptr[v] + i] */
-  LT_LAYOUT_ADJ = 2   /* steps gather adj[row_ptr[v] + i] = {u, deg(u), row_ptr[u]}: one access per step */
+  LT_LAYOUT_ADJ = 2,  /* steps gather adj[row_ptr[v] + i] = {u, deg(u), row_ptr[u]}: one access per step */
+  LT_LAYOUT_ADJ12 = 3 /* the same in 12 B per entry {u, row_ptr[u] (40 bits), deg(u) (24 bits)}: needs
+                         m < 2^40 and every degree < 2^24 (else LT_ERR_INVALID at load)
+                         With ADJ / ADJ12 the steps never read col: a col the library copied is freed
+                         at load, and a borrowed device col is not read after lt_graph_load_device
+                         returns (the caller may free it). */
 } lt_layout;
 
 typedef struct lt_config {
@@ -169,6 +176,10 @@ typedef struct lt_stats {
   uint64_t admissions;         /* walk admissions (lt_walks_init's included) in the last init + run */
   uint64_t peak_live;          /* most live walks seen at a scheduler step */
   uint64_t direct_start;       /* 1 if the last lt_walks_init* used the direct start (no walk records) */
+  uint64_t graph_device_bytes; /* device bytes of the graph the steps gather from: row_ptr + the CSR
+                                  (layout CSR) or augmented (ADJ / ADJ12) entries of the owned
+                                  vertices (all vertices when world == 1);
+                                  0 out of core (see pool_blocks x pool_block_bytes) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

@@ -51,7 +51,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.block_threads != 256) return fail(LT_ERR_INVALID, "block_threads must be 256 in this build");
   if (c.policy > 3 || c.insert_mode > 1 || c.gather_mode > 3 || c.zero_copy > 1)
     return fail(LT_ERR_INVALID, "bad policy / insert_mode / gather_mode");
-  if (c.layout > 2) return fail(LT_ERR_INVALID, "bad layout");
+  if (c.layout > 3) return fail(LT_ERR_INVALID, "bad layout");
   if (c.world == 0) c.world = 1;
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
@@ -111,6 +111,7 @@ void lt_destroy(lt_ctx* ctx) {
   free_ooc(ctx);
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   cudaFree(ctx->d_adj);
+  cudaFree(ctx->d_adj12);
   cudaFree(ctx->d_bounds);
   cudaFree(ctx->d_owner);
   cudaFree(ctx->d_paths);
@@ -179,25 +180,83 @@ static lt_status validate_row_ptr(uint32_t n, uint64_t m, const uint64_t* row_pt
   return LT_OK;
 }
 
+// Slice-only graph with range ownership ("each rank holds only its CSR slice"): the CSR
+// entries of the vertices rank r owns, [row_ptr[b[own_lo]], row_ptr[b[own_hi]]). A step only ever
+// gathers from the adjacency of an owned vertex: a walk that reaches another rank's vertex is sent
+// there before its next step. The whole row_ptr stays (8 B per vertex): the ADJ build needs deg(u) and
+// row_ptr[u] of every neighbour u, owned or not.
+static lt_status owned_edges(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* h_row_ptr, uint32_t P, uint64_t* e_lo,
+                             uint64_t* e_hi) {
+  *e_lo = 0;
+  *e_hi = m;
+  const uint32_t R = ctx->world;
+  if (R <= 1) return LT_OK;
+  if (R > P) return fail(LT_ERR_INVALID, "need num_partitions >= world");
+  std::vector<uint32_t> b(P + 1);
+  lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
+  if (s != LT_OK) return s;
+  *e_lo = h_row_ptr[b[(uint64_t)P * ctx->rank / R]];
+  *e_hi = h_row_ptr[b[(uint64_t)P * (ctx->rank + 1) / R]];
+  return LT_OK;
+}
+
 static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* h_row_ptr, uint32_t P) {
   CK(cudaEventRecord(ctx->ev_a, ctx->stream));
   // Layout: the augmented adjacency costs 16 B per CSR entry and saves one
   // random DRAM access per step; auto-select it when it fits in half of the free device memory.
-  bool use_adj = ctx->cfg.layout == LT_LAYOUT_ADJ && !ctx->ooc.on;
-  if (ctx->cfg.layout == LT_LAYOUT_AUTO && !ctx->ooc.on) {
-    size_t fr = 0, tot = 0;
-    CK(cudaMemGetInfo(&fr, &tot));
-    use_adj = m > 0 && (double)m * 16.0 <= 0.5 * (double)fr;
+  // (with ownership only the owned slice [e_lo, e_hi) is built)
+  // The compact 12-B form (LT_LAYOUT_ADJ12) packs row_ptr[u] into 40 bits and deg(u) into 24: it is
+  // taken when asked for, or by auto when only 12 B per entry fit.
+  const uint64_t ml = ctx->ooc.on ? m : ctx->e_hi - ctx->e_lo;
+  uint64_t dmax = 0;
+  for (uint32_t v = 0; v < n; ++v) dmax = std::max<uint64_t>(dmax, h_row_ptr[v + 1] - h_row_ptr[v]);
+  const bool fits12 = m < (1ull << 40) && dmax < (1ull << 24);
+  int lay = LT_LAYOUT_CSR;
+  if (!ctx->ooc.on && ml) {
+    if (ctx->cfg.layout == LT_LAYOUT_ADJ) lay = LT_LAYOUT_ADJ;
+    if (ctx->cfg.layout == LT_LAYOUT_ADJ12) {
+      if (!fits12) return fail(LT_ERR_INVALID, "LT_LAYOUT_ADJ12 needs m < 2^40 and every degree < 2^24");
+      lay = LT_LAYOUT_ADJ12;
+    }
+    if (ctx->cfg.layout == LT_LAYOUT_AUTO) {
+      // Measured on B200 (profiles/r01_gather_tlb_reach.json): random gathers run at the full access
+      // rate over up to 64 GiB and fall off beyond it (72 GiB 0.87x, 80 GiB 0.62x, 128 GiB 0.27x), the
+      // reach of the GPU's address translation. An augmented array past that reach loses more than the
+      // row_ptr access it saves, so it is only chosen within it.
+      constexpr double kGatherReach = 64.0 * (1ull << 30);
+      size_t fr = 0, tot = 0;
+      CK(cudaMemGetInfo(&fr, &tot));
+      const double a16 = (double)ml * 16.0, a12 = (double)ml * 12.0;
+      if (a16 <= 0.5 * (double)fr && a16 <= kGatherReach) lay = LT_LAYOUT_ADJ;
+      else if (fits12 && a12 <= 0.5 * (double)fr && a12 <= kGatherReach) lay = LT_LAYOUT_ADJ12;
+    }
   }
-  if (use_adj && m) {
-    CK(ensure(ctx->d_adj, ctx->adj_cap, m));
-    CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, m, ctx->d_adj, ctx->stream));
+  if (lay == LT_LAYOUT_ADJ) {
+    CK(ensure(ctx->d_adj, ctx->adj_cap, ml));
+    CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj, ctx->stream));
   } else if (ctx->d_adj) {
     cudaFree(ctx->d_adj);
     ctx->d_adj = nullptr;
     ctx->adj_cap = 0;
   }
-  ctx->stats.layout = (use_adj && m) ? LT_LAYOUT_ADJ : LT_LAYOUT_CSR;
+  if (lay == LT_LAYOUT_ADJ12) {
+    CK(ensure(ctx->d_adj12, ctx->adj12_cap, 3 * ml));
+    CK(lt::launch_build_adj12(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj12, ctx->stream));
+  } else if (ctx->d_adj12) {
+    cudaFree(ctx->d_adj12);
+    ctx->d_adj12 = nullptr;
+    ctx->adj12_cap = 0;
+  }
+  // the steps of an augmented layout never read col: a col the library owns is released (a borrowed
+  // one may be released by the caller, include/lt.h)
+  if (lay != LT_LAYOUT_CSR && ctx->own_graph && ctx->d_col) {
+    CK(cudaStreamSynchronize(ctx->stream));
+    cudaFree(ctx->d_col);
+    ctx->d_col = nullptr;
+  }
+  ctx->stats.layout = (uint32_t)lay;
+  ctx->stats.graph_device_bytes = ctx->ooc.on ? 0
+      : ((uint64_t)n + 1) * 8 + ml * (lay == LT_LAYOUT_ADJ ? 16 : lay == LT_LAYOUT_ADJ12 ? 12 : 4);
   ctx->stats.out_of_core = ctx->ooc.on ? 1 : 0;
   std::vector<uint32_t> b(P + 1);
   lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
@@ -321,16 +380,23 @@ lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row
   free_ooc(ctx);
   if (ctx->cfg.graph_pool_bytes) {
     ctx->own_graph = false;
+    ctx->e_lo = 0;
+    ctx->e_hi = m;
     lt_status so = setup_out_of_core(ctx, n, m, row_ptr, col, false, P);
     if (so != LT_OK) return so;
     return finish_graph_load(ctx, n, m, row_ptr, P);
   }
+  uint64_t e_lo = 0, e_hi = m;
+  s = owned_edges(ctx, n, m, row_ptr, P, &e_lo, &e_hi);
+  if (s != LT_OK) return s;
   ctx->own_graph = true;
   CK(cudaMalloc((void**)&ctx->d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t)));
-  CK(cudaMalloc((void**)&ctx->d_col, std::max<uint64_t>(m, 1) * sizeof(uint32_t)));
+  CK(cudaMalloc((void**)&ctx->d_col, std::max<uint64_t>(e_hi - e_lo, 1) * sizeof(uint32_t)));
   CK(cudaMemcpy(ctx->d_row_ptr, row_ptr, ((size_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
-  if (m) CK(cudaMemcpy(ctx->d_col, col, m * sizeof(uint32_t), cudaMemcpyHostToDevice));
-  ctx->stats.h2d_bytes += ((uint64_t)n + 1) * 8 + m * 4;
+  if (e_hi > e_lo) CK(cudaMemcpy(ctx->d_col, col + e_lo, (e_hi - e_lo) * sizeof(uint32_t), cudaMemcpyHostToDevice));
+  ctx->e_lo = e_lo;
+  ctx->e_hi = e_hi;
+  ctx->stats.h2d_bytes += ((uint64_t)n + 1) * 8 + (e_hi - e_lo) * 4;
   return finish_graph_load(ctx, n, m, row_ptr, P);
 }
 
@@ -356,12 +422,19 @@ lt_status lt_graph_load_device(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64
   if (ctx->cfg.graph_pool_bytes) {  // host-resident copy of the caller's device CSR
     ctx->d_row_ptr = nullptr;
     ctx->d_col = nullptr;
+    ctx->e_lo = 0;
+    ctx->e_hi = m;
     lt_status so = setup_out_of_core(ctx, n, m, d_row_ptr, d_col, true, P);
     if (so != LT_OK) return so;
     return finish_graph_load(ctx, n, m, h.data(), P);
   }
+  uint64_t e_lo = 0, e_hi = m;
+  s = owned_edges(ctx, n, m, h.data(), P, &e_lo, &e_hi);
+  if (s != LT_OK) return s;
   ctx->d_row_ptr = (unsigned long long*)d_row_ptr;
-  ctx->d_col = (uint32_t*)d_col;
+  ctx->d_col = (uint32_t*)d_col + e_lo;  // a view of the owned slice of the caller's array
+  ctx->e_lo = e_lo;
+  ctx->e_hi = e_hi;
   return finish_graph_load(ctx, n, m, h.data(), P);
 }
 
@@ -473,8 +546,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.wk.row_ptr = ctx->d_row_ptr;
   p.wk.col = ctx->d_col;
   p.wk.vbase = 0;
-  p.wk.ebase = 0;
+  p.wk.ebase = ctx->ooc.on ? 0 : ctx->e_lo;  // col / adj hold the CSR entries from e_lo on (ownership slice)
   p.wk.adj = ctx->ooc.on ? nullptr : ctx->d_adj;
+  p.wk.adj12 = ctx->ooc.on ? nullptr : ctx->d_adj12;
   p.wk.bounds = ctx->d_bounds;
   p.wk.P = ctx->P;
   p.wk.paths = ctx->d_paths;
@@ -514,7 +588,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.insert_mode = ctx->cfg.insert_mode;
   p.gather_mode = ctx->cfg.gather_mode;
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
-  p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : (ctx->d_adj ? 1u : 2u);
+  p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : ((p.wk.adj || p.wk.adj12) ? 1u : 2u);
   // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
   // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
   p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;

@@ -62,11 +62,14 @@ struct lt_ctx {
   uint32_t nb = 0;             // buckets: P + (world > 1 ? world : 0)
   uint32_t rank = 0, world = 1, own_lo = 0, own_hi = 0;
   uint16_t* d_owner = nullptr;  // [P] owner rank per partition (world > 1)
-  unsigned long long* d_row_ptr = nullptr;
-  uint32_t* d_col = nullptr;
+  unsigned long long* d_row_ptr = nullptr;  // [n+1], the whole row_ptr (global offsets)
+  uint32_t* d_col = nullptr;                // CSR entries [e_lo, e_hi): d_col[0] is entry e_lo
+  uint64_t e_lo = 0, e_hi = 0;              // edges of the vertices this rank owns ([0, m) when world == 1)
   bool own_graph = false;
   uint4* d_adj = nullptr;  // augmented adjacency (layout ADJ), owned
   size_t adj_cap = 0;
+  uint32_t* d_adj12 = nullptr;  // compact augmented adjacency (layout ADJ12, 3 words per entry), owned
+  size_t adj12_cap = 0;
   std::vector<uint32_t> h_bounds;
   uint32_t* d_bounds = nullptr;
   size_t bounds_cap = 0;

@@ -40,7 +40,8 @@ struct Walk {
   const uint32_t* col;
   uint32_t vbase;
   unsigned long long ebase;
-  const uint4* adj;               // [m] augmented adjacency {u, deg(u), row_ptr[u]} or nullptr (CSR)
+  const uint4* adj;               // [m] augmented adjacency {u, deg(u), row_ptr[u]} or nullptr
+  const uint32_t* adj12;          // [3m] compact augmented adjacency (12 B per entry) or nullptr
   const uint32_t* bounds;         // [P+1]
   uint32_t P;
   uint32_t* paths;
@@ -133,6 +134,8 @@ constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
                              cudaStream_t s);
+cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
+                               cudaStream_t s);
 int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill);  // resident blocks per SM (update kernel)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 

@@ -346,6 +346,67 @@ __device__ __forceinline__ uint4 ld_adj(const uint4* p, const Policies& pol) {
   return v;
 }
 
+// Compact augmented adjacency (LAY 2): entry j is 12 bytes = 3 words {u, off lo32, off hi8 | deg << 8}
+// (row_ptr[u] < 2^40, deg(u) < 2^24). Two aligned 8-B loads cover the entry wherever it starts (byte
+// 12j is 8-aligned for even j, 4 past an 8-B boundary for odd j); they fall in one 64-B block unless the
+// entry itself straddles one (2 of every 16 entries), so a step is still ONE random DRAM access.
+struct Adj { uint32_t u, deg; unsigned long long off; };
+#ifndef LT_ADJ12_LOAD
+#define LT_ADJ12_LOAD 0  // 0: two 8-B loads; 1: three 4-B loads; 2: 16-B load + a second one when needed
+#endif
+#ifndef LT_ADJ12_POL
+#define LT_ADJ12_POL 0   // 0: evict_first + L2::64B (GM 3); 1: L2::64B only
+#endif
+template <int GM>
+__device__ __forceinline__ uint2 ld2_hint(const uint2* q, const Policies& pol) {
+  uint2 v;
+  if (GM == 0) return __ldg(q);
+#if LT_ADJ12_POL == 0
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.v2.u32 {%0, %1}, [%2], %3;" : "=r"(v.x), "=r"(v.y) : "l"(q), "l"(pol.first));
+#else
+  asm volatile("ld.global.nc.L2::64B.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(q));
+#endif
+  return v;
+}
+template <int GM>
+__device__ __forceinline__ uint32_t ld1_hint(const uint32_t* q, const Policies& pol) {
+  uint32_t v;
+  if (GM == 0) return __ldg(q);
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u32 %0, [%1], %2;" : "=r"(v) : "l"(q), "l"(pol.first));
+  return v;
+}
+template <int GM>
+__device__ __forceinline__ Adj ld_adj12(const uint32_t* a12, unsigned long long j, const Policies& pol) {
+  const unsigned long long w = 3 * j;  // word index of the entry
+  uint32_t w0, w1, w2;
+#if LT_ADJ12_LOAD == 1
+  w0 = ld1_hint<GM>(a12 + w, pol);
+  w1 = ld1_hint<GM>(a12 + w + 1, pol);
+  w2 = ld1_hint<GM>(a12 + w + 2, pol);
+#elif LT_ADJ12_LOAD == 2
+  const uint4* q4 = reinterpret_cast<const uint4*>(a12 + (w & ~3ull));
+  const uint4 A = ld_adj<GM>(q4, pol);
+  const uint32_t r = (uint32_t)(w & 3ull);
+  uint4 B = make_uint4(0, 0, 0, 0);
+  if (r >= 2) B = ld_adj<GM>(q4 + 1, pol);
+  w0 = r == 0 ? A.x : r == 1 ? A.y : r == 2 ? A.z : A.w;
+  w1 = r == 0 ? A.y : r == 1 ? A.z : r == 2 ? A.w : B.x;
+  w2 = r == 0 ? A.z : r == 1 ? A.w : r == 2 ? B.x : B.y;
+#else
+  const uint2* q = reinterpret_cast<const uint2*>(a12 + (w & ~1ull));
+  const uint2 lo = ld2_hint<GM>(q, pol), hi = ld2_hint<GM>(q + 1, pol);
+  const bool odd = (w & 1ull) != 0;
+  w0 = odd ? lo.y : lo.x;
+  w1 = odd ? hi.x : lo.y;
+  w2 = odd ? hi.y : hi.x;
+#endif
+  Adj e;
+  e.u = w0;
+  e.deg = w2 >> 8;
+  e.off = (unsigned long long)w1 | ((unsigned long long)(w2 & 0xFFu) << 32);
+  return e;
+}
+
 // ------------------------------------------------------------------------------- a3 + a4 + a5
 // ILP walks per lane: a warp takes 32*ILP consecutive records; each lane advances its ILP walks in
 // lockstep so their dependent gathers are in flight together (memory-level parallelism is what
@@ -354,6 +415,8 @@ __device__ __forceinline__ uint4 ld_adj(const uint4* p, const Policies& pol) {
 //   0 (CSR): per step row_ptr[v], row_ptr[v+1] (one line) then col[off + i] (one line);
 //   1 (ADJ): per step ONE 16-B gather adj[off + i] = {u, deg(u), row_ptr[u]} that carries the next
 //            vertex's degree and offset, so only a visit's first step reads row_ptr.
+// Offsets are global CSR positions; col / adj hold the entries from wk.ebase on (an out-of-core
+// block's slice, or the owned slice with range ownership), so every gather subtracts ebase.
 template <int ILP> struct MinBlocks { static constexpr int v = 4; };
 template <> struct MinBlocks<2> { static constexpr int v = 3; };
 template <> struct MinBlocks<4> { static constexpr int v = 2; };
@@ -435,7 +498,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
       for (int q = 0; q < 8; ++q) pb[s][q] = 0;
       pb[s][7] = rec[s].y;
       nb[s] = (alive[s] && (rec[s].z & 7u) == 0) ? 1u : 0u;  // entry t0 opens its sector: rewrite it too
-      if (LAY == 1 && alive[s]) {  // the visit's first vertex: its offset and degree from row_ptr
+      if (LAY != 0 && alive[s]) {  // the visit's first vertex: its offset and degree from row_ptr
         off[s] = __ldg(wk.row_ptr + rec[s].y);
         d[s] = (uint32_t)(__ldg(wk.row_ptr + rec[s].y + 1) - off[s]);
       }
@@ -491,17 +554,22 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
                                    : (uint32_t)(m >> 32);
           if (restart) {
             nv[s] = idx;
-            if (LAY == 1 && idx - lo < span) {  // staying: the next step needs its offset and degree
+            if (LAY != 0 && idx - lo < span) {  // staying: the next step needs its offset and degree
               off[s] = __ldg(wk.row_ptr + idx);
               d[s] = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off[s]);
             }
           } else if (LAY == 0) {
             nv[s] = ld_col<GM>(wk.col + off[s] + idx, pol);
-          } else {
-            const uint4 e = ld_adj<GM>(wk.adj + off[s] + idx, pol);
+          } else if (LAY == 1) {
+            const uint4 e = ld_adj<GM>(wk.adj + (off[s] - wk.ebase) + idx, pol);
             nv[s] = e.x;
             d[s] = e.y;
             off[s] = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+          } else {
+            const Adj e = ld_adj12<GM>(wk.adj12, off[s] - wk.ebase + idx, pol);
+            nv[s] = e.u;
+            d[s] = e.deg;
+            off[s] = e.off;
           }
         }
       }
@@ -660,7 +728,7 @@ __global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_
         prow = wk.paths + (uint64_t)rec.x * wk.pitch;
         pb[7] = rec.y;
         nb = ((rec.z & 7u) == 0) ? 1u : 0u;
-        if (LAY == 1) {
+        if (LAY != 0) {
           off = __ldg(wk.row_ptr + rec.y);
           d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
         }
@@ -710,17 +778,22 @@ __global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_
           uint32_t nv;
           if (restart) {
             nv = idx;
-            if (LAY == 1 && idx - lo < span) {
+            if (LAY != 0 && idx - lo < span) {
               off = __ldg(wk.row_ptr + idx);
               d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
             }
           } else if (LAY == 0) {
             nv = ld_col<GM>((CONT ? c_col : wk.col) + off + idx, pol);
-          } else {
-            const uint4 e = ld_adj<GM>(wk.adj + off + idx, pol);
+          } else if (LAY == 1) {
+            const uint4 e = ld_adj<GM>(wk.adj + (off - wk.ebase) + idx, pol);
             nv = e.x;
             d = e.y;
             off = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+          } else {
+            const Adj e = ld_adj12<GM>(wk.adj12, off - wk.ebase + idx, pol);
+            nv = e.u;
+            d = e.deg;
+            off = e.off;
           }
           rec.y = nv;
           rec.z += 1;
@@ -1027,6 +1100,27 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
   return cudaGetLastError();
 }
 
+// Compact augmented adjacency (LAY 2): words 3i..3i+2 = {u, row_ptr[u] lo32, row_ptr[u] hi8 | deg(u) << 8}
+// for u = col[i] (the host checked row_ptr[n] < 2^40 and every degree < 2^24).
+__global__ void k_build_adj12(const unsigned long long* __restrict__ row_ptr, const uint32_t* __restrict__ col,
+                              uint64_t m, uint32_t* __restrict__ a12) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t u = col[i];
+    const unsigned long long o = __ldg(row_ptr + u);
+    const uint32_t dg = (uint32_t)(__ldg(row_ptr + u + 1) - o);
+    a12[3 * i] = u;
+    a12[3 * i + 1] = (uint32_t)o;
+    a12[3 * i + 2] = (uint32_t)(o >> 32) | (dg << 8);
+  }
+}
+
+cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
+                               cudaStream_t s) {
+  if (!m) return cudaSuccess;
+  k_build_adj12<<<num_sms() * 8, 256, 0, s>>>(row_ptr, col, m, a12);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_insert_records(const Params& p, const uint4* recs, uint64_t count, cudaStream_t s) {
   if (!count) return cudaSuccess;
   uint64_t want = (count + 255) / 256;
@@ -1100,12 +1194,14 @@ void launch_update_ilp(const Params& p, uint32_t k, uint32_t grid, uint32_t bloc
 
 template <int APP, int VIS>
 void launch_update_app(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  const bool adj = p.wk.adj != nullptr;
+  const bool adj = p.wk.adj != nullptr, adj12 = p.wk.adj12 != nullptr;
   if (p.gather_mode == 0) {
     if (adj) launch_update_ilp<APP, 0, 1, VIS>(p, k, grid, block, s);
+    else if (adj12) launch_update_ilp<APP, 0, 2, VIS>(p, k, grid, block, s);
     else launch_update_ilp<APP, 0, 0, VIS>(p, k, grid, block, s);
   } else {
     if (adj) launch_update_ilp<APP, 3, 1, VIS>(p, k, grid, block, s);
+    else if (adj12) launch_update_ilp<APP, 3, 2, VIS>(p, k, grid, block, s);
     else launch_update_ilp<APP, 3, 0, VIS>(p, k, grid, block, s);
   }
 }

@@ -25,7 +25,7 @@ LT_OK, LT_ERR_INVALID, LT_ERR_STATE, LT_ERR_OOM, LT_ERR_CUDA, LT_ERR_NCCL = rang
 DEEPWALK, PPR, PAGERANK = 0, 1, 2
 POLICY_SELECTIVE, POLICY_ROUND_ROBIN, POLICY_SELECTIVE_ONLY, POLICY_PREEMPTIVE_ONLY = 0, 1, 2, 3
 INSERT_WARP_AGGREGATED, INSERT_DIRECT = 0, 1
-LAYOUT_AUTO, LAYOUT_CSR, LAYOUT_ADJ = 0, 1, 2
+LAYOUT_AUTO, LAYOUT_CSR, LAYOUT_ADJ, LAYOUT_ADJ12 = 0, 1, 2, 3
 EMPTY = 0xFFFFFFFF
 
 EXPORTED = [
@@ -77,7 +77,7 @@ class Stats(ctypes.Structure):
         ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
-            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start")]
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes")]
 
 
 class PoolState(ctypes.Structure):
@@ -232,7 +232,8 @@ class Engine:
         m = len(kcol) if not _is_torch(kcol) else kcol.numel()
         if dev_r:
             _check(_lib.lt_graph_load_device(self._h, n, m, prp, pcol, num_partitions))
-            self._graph_keep = (krp, kcol)  # borrowed device memory stays alive
+            # borrowed device memory stays alive; col only while the steps read it (CSR layout)
+            self._graph_keep = (krp, kcol) if self.stats()["layout"] == LAYOUT_CSR else (krp,)
         else:
             _check(_lib.lt_graph_load(self._h, n, m, prp, pcol, num_partitions))
             self._graph_keep = None

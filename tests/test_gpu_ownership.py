@@ -56,7 +56,7 @@ def g13():
 
 
 @pytest.mark.parametrize("world", [2, 3, 4])
-@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
 def test_ownership_deepwalk_exact(gpu, g13, world, layout):
     starts = lt_inputs.deepwalk_starts(3 * g13.n, g13.n)
     res = run_owned(g13, starts, LT.DEEPWALK, 16, 2, 12, world, layout=layout, chunk_walks=512)
@@ -66,6 +66,30 @@ def test_ownership_deepwalk_exact(gpu, g13, world, layout):
         np.testing.assert_array_equal(paths, op)
     assert sum(r[3]["steps"] for r in res) == osteps  # each step is taken on exactly one rank
     assert res[0][2]["records_sent"] > 0
+    # slice-only graph: a rank holds row_ptr plus the CSR (and ADJ) entries of the
+    # vertices it owns; the slices partition the m entries
+    per_entry = {LT.LAYOUT_CSR: 4, LT.LAYOUT_ADJ: 16, LT.LAYOUT_ADJ12: 12}[layout]
+    slices = [(st["graph_device_bytes"] - (g13.n + 1) * 8) / per_entry for _, _, _, st in res]
+    assert all(x == int(x) and 0 < x < g13.m for x in slices), slices
+    assert sum(slices) == g13.m
+    assert all(st["layout"] == layout for _, _, _, st in res)
+
+
+def test_ownership_device_graph_slice(gpu, g13):
+    """lt_graph_load_device with ownership: the caller's whole device CSR is borrowed, each rank gathers
+    only from (and builds ADJ only for) its owned slice."""
+    import torch
+    world = 3
+    starts = lt_inputs.deepwalk_starts(2 * g13.n, g13.n)
+    rp = torch.from_numpy(g13.row_ptr.view(np.int64)).cuda()
+    col = torch.from_numpy(g13.col.view(np.int32)).cuda()
+    g_dev = type("G", (), {"row_ptr": rp, "col": col})
+    res = run_owned(g_dev, starts, LT.DEEPWALK, 9, 8, 9, world, layout=LT.LAYOUT_ADJ, chunk_walks=256)
+    op, ol, _, _ = oracle_of(g13, starts, LT.DEEPWALK, 9, 8)
+    for paths, lengths, _, st in res:
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+    assert sum((st["graph_device_bytes"] - (g13.n + 1) * 8) // 16 for _, _, _, st in res) == g13.m
 
 
 @pytest.mark.parametrize("world", [2, 4])

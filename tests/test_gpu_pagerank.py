@@ -59,7 +59,7 @@ def test_pagerank_exact(gpu, cfg1, p, P):
         assert st["visits"] > 4096
 
 
-@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
 @pytest.mark.parametrize("ilp,refill", [(1, 1), (2, 1), (4, 1), (1, 2)])
 @pytest.mark.parametrize("P", [1, 8])
 @pytest.mark.parametrize("width", [1, 2])  # u32 counters (auto) / forced u64 counters

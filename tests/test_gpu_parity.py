@@ -226,7 +226,7 @@ def test_pool_invariants(gpu, cfg1, P, chunk):
         assert s1["free_chunks"] + s1["ring_chunks"] == s1["total_chunks"], s1
 
 
-@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
 @pytest.mark.parametrize("ilp,refill", [(1, 1), (2, 1), (4, 1), (1, 2)])
 @pytest.mark.parametrize("gather_mode", [0, 3])
 @pytest.mark.parametrize("P", [1, 8])
@@ -238,6 +238,50 @@ def test_kernel_variants_exact(gpu, cfg1, layout, ilp, refill, gather_mode, P):
     assert_parity(cfg1, lt_inputs.ppr_starts(3000, cfg1.argmax_deg), LT.PPR, 0.2, 7, P=P, **kw)
     g = lt_inputs.small_graph([(0, 1), (1, 3), (3, 4)], n=6)
     assert_parity(g, np.array([0, 2, 5, 4, 1, 2], dtype=np.uint32), LT.DEEPWALK, 9, 1, P=min(P, 6), **kw)
+
+
+def test_layouts_memory_and_limits(gpu, cfg1):
+    """Graph bytes per layout (col is released once an augmented layout is built from a host graph; a
+    borrowed device col is no longer referenced), and ADJ12's 24-bit degree limit."""
+    import torch
+    n, m = cfg1.n, cfg1.m
+    expect = {LT.LAYOUT_CSR: (n + 1) * 8 + 4 * m, LT.LAYOUT_ADJ: (n + 1) * 8 + 16 * m,
+              LT.LAYOUT_ADJ12: (n + 1) * 8 + 12 * m}
+    for lay, b in expect.items():
+        with LT.Engine(layout=lay) as e:
+            e.graph_load(cfg1.row_ptr, cfg1.col, 2)
+            st = e.stats()
+            assert st["layout"] == lay and st["graph_device_bytes"] == b, (lay, st["graph_device_bytes"], b)
+            # borrowed device graph: col is kept referenced only for CSR
+            rp = torch.from_numpy(cfg1.row_ptr.view(np.int64)).cuda()
+            col = torch.from_numpy(cfg1.col.view(np.int32)).cuda()
+            e.graph_load(rp, col, 2)
+            assert len(e._graph_keep) == (2 if lay == LT.LAYOUT_CSR else 1)
+            del col
+            torch.cuda.empty_cache()
+            starts = lt_inputs.deepwalk_starts(3000, n)
+            e.walks_init(starts, LT.DEEPWALK, 9, 4)
+            e.run()
+            p_, l_ = e.get_paths()
+        op, ol, _, _ = run_oracle(cfg1, starts, LT.DEEPWALK, 9, 4)
+        np.testing.assert_array_equal(p_, op)
+    # a star whose hub has 2^24 neighbours: too wide for ADJ12's 24-bit degree field
+    leaves = 1 << 24
+    src = np.concatenate([np.zeros(leaves, np.uint32), np.arange(1, leaves + 1, dtype=np.uint32)])
+    row_ptr = np.concatenate([[0, leaves], leaves + np.arange(1, leaves + 1)]).astype(np.uint64)
+    col = np.concatenate([np.arange(1, leaves + 1, dtype=np.uint32), np.zeros(leaves, np.uint32)])
+    assert len(src) == len(col) == row_ptr[-1]
+    with LT.Engine(layout=LT.LAYOUT_ADJ12) as e:
+        with pytest.raises(LT.LTError, match="2\\^24"):
+            e.graph_load(row_ptr, col, 1)
+    with LT.Engine() as e:  # auto falls back to a layout that holds it
+        e.graph_load(row_ptr, col, 1)
+        assert e.stats()["layout"] in (LT.LAYOUT_ADJ, LT.LAYOUT_CSR)
+        e.walks_init(np.array([0, 5, 1 << 24], np.uint32), LT.DEEPWALK, 6, 1)
+        e.run()
+        p_, l_ = e.get_paths()
+    op, ol, _, _ = O.walks(row_ptr, col, np.array([0, 5, 1 << 24], np.uint32), app=O.DEEPWALK, length=6, seed=1)
+    np.testing.assert_array_equal(p_, op)
 
 
 @pytest.mark.parametrize("path_mode", [0, 1])
