@@ -294,13 +294,17 @@ lt_status lt_run_to_host_compact(lt_ctx* ctx, uint64_t num_walks, const uint32_t
  * Path rows then hold only the entries this rank wrote (others 0xFFFFFFFF) and lengths only the
  * walks that ended here (others 0): the merged result is the element-wise min of the paths and the
  * max of the lengths over ranks. Walk records carry walk indices, identical on every rank. */
-/* Walks waiting in owned buckets (*local) and in the send bucket of each rank (outgoing[world]). */
+/* Walks waiting in owned buckets (*local) and in the send bucket of each rank (outgoing[world]).
+ * Reuses the counts lt_run read last when no walk has moved since (no device round trip), else
+ * reads them (one small D2H + stream synchronisation). */
 lt_status lt_pending(lt_ctx* ctx, uint64_t* local, uint64_t* outgoing);
 /* Move every send bucket into d_send (device, 16-B records, grouped by destination rank in rank
  * order); counts[world] (host) receives the number of records per destination (0 for this rank).
- * LT_ERR_INVALID if capacity (records) is too small. */
+ * LT_ERR_INVALID if capacity (records) is too small. Asynchronous: d_send is complete in the order
+ * of the context's stream (a collective enqueued after this call on that stream sees it). */
 lt_status lt_exchange_pack(lt_ctx* ctx, void* d_send, uint64_t capacity, uint64_t* counts);
-/* Insert `count` received records (device memory) into the owned buckets. */
+/* Insert `count` received records (device memory, read in stream order; the caller keeps it alive
+ * until the next synchronising call, e.g. lt_run) into the owned buckets. Asynchronous. */
 lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count);
 
 /* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:

@@ -611,6 +611,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.chunks_total = num_chunks;
   ctx->stats.kernel_launches = 0;
   CK(cudaEventRecord(ctx->ev_a, s));
+  ctx->snap_valid = false;
   CK(lt::launch_pool_reset(p, s));
   ctx->stats.kernel_launches++;
   if (W) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
@@ -671,8 +672,9 @@ lt_status lt_run(lt_ctx* ctx) {
     ctx->stats.kernel_launches++;
   }
   CK(cudaEventRecord(ctx->ev_b, s));
-  st = lt::snapshot(ctx);
+  st = lt::snapshot_cached(ctx);  // the scheduler's last count read (nothing moved since) or a fresh one
   if (st != LT_OK) return st;
+  CK(cudaEventSynchronize(ctx->ev_b));
   {
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
@@ -855,7 +857,7 @@ lt_status lt_pending(lt_ctx* ctx, uint64_t* local, uint64_t* outgoing) {
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
   CK(cudaSetDevice(ctx->cfg.device));
   const size_t nb = ctx->nb;
-  lt_status sn = lt::snapshot(ctx);
+  lt_status sn = lt::snapshot_cached(ctx);
   if (sn != LT_OK) return sn;
   uint64_t loc = 0;
   for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k) loc += ctx->h_hc[nb + k] - ctx->h_hc[k];
@@ -880,11 +882,13 @@ lt_status lt_exchange_pack(lt_ctx* ctx, void* d_send, uint64_t capacity, uint64_
   for (uint32_t r = 0; r < ctx->world; ++r) {
     counts[r] = out[r];
     if (!out[r]) continue;
+    ctx->snap_valid = false;
     CK(lt::launch_pack(ctx->params, ctx->P + r, (uint4*)d_send + off, out[r], ctx->stream));
     ctx->stats.kernel_launches++;
     off += out[r];
   }
-  CK(cudaStreamSynchronize(ctx->stream));
+  // no host synchronisation: the buffer is complete in stream order, which is what the collective that
+  // sends it (enqueued after this call on the same stream) needs
   return LT_OK;
 }
 
@@ -892,10 +896,10 @@ lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
   if (count && !d_recv) return fail(LT_ERR_INVALID, "NULL receive buffer");
+  if (count) ctx->snap_valid = false;
   CK(lt::launch_insert_records(ctx->params, (const uint4*)d_recv, count, ctx->stream));
   if (count) ctx->stats.kernel_launches++;
-  CK(cudaStreamSynchronize(ctx->stream));
-  return LT_OK;
+  return LT_OK;  // stream-ordered: the next lt_run's first count read synchronises
 }
 
 // lt_run_to_host / lt_run_to_host_compact: dense rows (paths != NULL) or the ragged layout

@@ -78,6 +78,7 @@ struct lt_ctx {
   bool walks_ready = false;
   bool ran = false;
   bool padded = false;  // path slots past each length hold 0xFFFFFFFF (done lazily, before a copy-out)
+  bool snap_valid = false;  // h_hc / h_ctr / h_free mirror the device (no pool-changing launch since)
   uint64_t W = 0, first = 0, seed = 0;
   lt_app app = LT_APP_DEEPWALK;
   uint32_t length = 0, T = 0, lmax = 127, stride = 1, pitch = 8;
@@ -146,6 +147,7 @@ struct lt_ctx {
 
 namespace lt {
 lt_status snapshot(lt_ctx* ctx);  // h_hc / h_ctr / h_free <- device, then sync the stream
+lt_status snapshot_cached(lt_ctx* ctx);  // snapshot() unless the mirror is still valid
 lt_status run_resident(lt_ctx* ctx);
 lt_status run_out_of_core(lt_ctx* ctx);
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound);

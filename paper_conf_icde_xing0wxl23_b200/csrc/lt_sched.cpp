@@ -48,8 +48,14 @@ lt_status snapshot(lt_ctx* ctx) {
   CK(launch_snapshot(ctx->d_hc, 2 * (uint64_t)ctx->nb, ctx->d_ctr, (const int*)ctx->d_small, dh, dc, df, ctx->stream));
   ctx->stats.kernel_launches++;
   CK(cudaStreamSynchronize(ctx->stream));
+  ctx->snap_valid = true;
   return LT_OK;
 }
+
+// Every launch that moves walks between buckets (update, init, insert, pack) clears snap_valid; the
+// ABI calls that only need the counts (lt_pending, lt_exchange_pack, the end of lt_run) then reuse the
+// mirror instead of another D2H + stream synchronisation.
+lt_status snapshot_cached(lt_ctx* ctx) { return ctx->snap_valid ? LT_OK : snapshot(ctx); }
 
 // Walk admission (f3; lt_config.walk_pool_walks): create the next walks in index order once at least a
 // quarter of the pool (or everything still to come) has room, so live walks never exceed cap_walks.
@@ -60,6 +66,7 @@ lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did) {
   const uint64_t room = ctx->cap_walks - live, rest = ctx->W - ctx->admitted;
   if (room < std::min<uint64_t>(rest, std::max<uint64_t>(ctx->cap_walks / 4, 1))) return LT_OK;
   const uint64_t n = std::min(room, rest);
+  ctx->snap_valid = false;
   CK(launch_init(ctx->params, ctx->adm_starts + ctx->admitted, n, ctx->admitted, ctx->stream));
   ctx->admitted += n;
   ctx->stats.admissions++;
@@ -81,6 +88,7 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
     }
     CK(cudaEventRecord(ctx->events[ctx->nev], s));
   }
+  ctx->snap_valid = false;
   CK(launch_update(p, k, (uint32_t)grid, ctx->block, s));
   if (ctx->cfg.timing) {
     CK(cudaEventRecord(ctx->events[ctx->nev + 1], s));

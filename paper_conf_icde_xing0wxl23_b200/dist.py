@@ -4,13 +4,19 @@ the paper): the superstep exchange around the C ABI.
 Rank r owns a contiguous range of partitions (lt_config.rank/world). Each superstep:
   1. lt_run            advance every walk in the owned buckets until it ends or leaves the range
                        (walks for rank q collect in send bucket q);
-  2. lt_exchange_pack  move the send buckets into one device buffer, grouped by destination;
-  3. all-to-all        of the per-rank counts, then of the 16-B walk records (NCCL over NVLink via
-                       torch.distributed; gloo on CPU in the tests);
-  4. lt_exchange_insert the received walks into the owned buckets (warp-aggregated insertion);
+  2. lt_exchange_pack  move the send buckets into one device buffer, grouped by destination (the
+                       counts come from lt_run's last count read: no extra device round trip);
+  3. all-gather        of every rank's per-destination counts (R x R): each rank reads what it will
+                       receive and the global number of crossing walks (the termination test) from
+                       the same matrix, in ONE small collective;
+  4. all-to-all        of the 16-B walk records (NCCL over NVLink via torch.distributed; gloo on CPU
+                       in the tests), stream-ordered after the pack;
+  5. lt_exchange_insert the received walks into the owned buckets (warp-aggregated insertion),
+                       stream-ordered, no host synchronisation;
 until no walk crossed ranks in a superstep (every live walk is then in some owned bucket, and lt_run
-ended them all). Paths are merged once at the end: element-wise unsigned min of the path rows
-(unwritten entries are 0xFFFFFFFF) and max of the lengths.
+ended them all). Host round trips per superstep: lt_run's count reads and the count all-gather.
+Paths are merged once at the end: element-wise unsigned min of the path rows (unwritten entries are
+0xFFFFFFFF) and max of the lengths.
 
 The exchange is the only data-path collective; this module only sequences ABI calls and
 collectives (plumbing), every walk step runs in the CUDA kernels behind the ABI.
@@ -38,6 +44,15 @@ class TorchComm:
         out = torch.empty_like(t)
         self.dist.all_to_all_single(out, t, group=self.group)
         return [int(x) for x in out.tolist()]
+
+    def allgather_counts(self, counts, device):
+        """Every rank's count vector: returns the R x R matrix M (M[r][q] = records r sends to q)."""
+        import torch
+        t = torch.tensor(counts, dtype=torch.int64, device=device)
+        parts = [torch.empty_like(t) for _ in range(self.world)]
+        self.dist.all_gather(parts, t, group=self.group)
+        m = torch.stack(parts).tolist()
+        return [[int(x) for x in row] for row in m]
 
     def alltoallv(self, send, send_counts, recv_counts):
         """send: int32 [sum(send_counts), 4]; returns int32 [sum(recv_counts), 4]."""
@@ -85,6 +100,9 @@ class ThreadComm:
         allc = self._gather(list(counts))
         return [allc[r][self.rank] for r in range(self.world)]
 
+    def allgather_counts(self, counts, device):
+        return [list(c) for c in self._gather(list(counts))]
+
     def alltoallv(self, send, send_counts, recv_counts):
         import torch
         offs = [0]
@@ -127,14 +145,15 @@ def run_supersteps(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
         engine.run()
         buf = send_buffer(engine, device, cache)
         counts = engine.exchange_pack(buf)
-        recv_counts = comm.alltoall_counts(counts, device)
-        recv = comm.alltoallv(buf, counts, recv_counts)
-        engine.exchange_insert(recv, sum(recv_counts))
-        crossed = comm.allreduce_sum(sum(recv_counts), device)
+        mat = comm.allgather_counts(counts, device)  # mat[r][q]: records rank r sends to rank q
+        crossed = sum(sum(row) for row in mat)
         supersteps += 1
         moved += sum(counts)
         if crossed == 0:
             return {"supersteps": supersteps, "records_sent": moved}
+        recv_counts = [mat[r][comm.rank] for r in range(comm.world)]
+        recv = comm.alltoallv(buf, counts, recv_counts)
+        engine.exchange_insert(recv, sum(recv_counts))
         if supersteps >= max_supersteps:
             raise RuntimeError("ownership supersteps did not converge")
 

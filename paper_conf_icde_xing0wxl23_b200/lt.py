@@ -385,6 +385,7 @@ class Engine:
         if d_recv is not None and count and not dev:
             raise ValueError("exchange_insert needs a CUDA tensor")
         _check(_lib.lt_exchange_insert(self._h, pp, count))
+        self._recv_keep = d_recv  # read asynchronously by the insert kernel (stream-ordered)
 
     def partial_paths(self):
         """This rank's share of paths (CUDA int32 tensors [W, stride], [W]) for the cross-rank merge."""

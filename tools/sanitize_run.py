@@ -2,7 +2,9 @@
 """Small runs of every kernel path for compute-sanitizer (memcheck / racecheck / synccheck /
 initcheck): resident P=1 (refill), P=4 (batch kernel, CSR and ADJ), PPR, out-of-core with zero copy,
 two-rank ownership, streamed run_to_host (dense and ragged), ragged copy-out, PageRank with u32 / u64
-visit counters, out-of-core continuation, walk admission, paths off."""
+visit counters, out-of-core continuation, walk admission, paths off, the direct start (P = 1, both
+path modes, device starts), the compact ADJ12 layout, slice-only ownership (CSR / ADJ / ADJ12, host and
+borrowed device graphs)."""
 import os
 import sys
 import threading
@@ -18,7 +20,9 @@ from paper_conf_icde_xing0wxl23_b200 import dist as ltdist  # noqa: E402
 g = lt_inputs.rmat_cpu(12, 65_536, seed=1)
 starts = lt_inputs.deepwalk_starts(4096, g.n)
 pstarts = lt_inputs.ppr_starts(4096, g.argmax_deg)
-for kw in [dict(P=1), dict(P=4, layout=LT.LAYOUT_CSR), dict(P=4, layout=LT.LAYOUT_ADJ), dict(P=4, refill=2)]:
+for kw in [dict(P=1), dict(P=4, layout=LT.LAYOUT_CSR), dict(P=4, layout=LT.LAYOUT_ADJ), dict(P=4, refill=2),
+           dict(P=1, layout=LT.LAYOUT_ADJ12), dict(P=4, layout=LT.LAYOUT_ADJ12), dict(P=1, path_mode=1),
+           dict(P=1, direct_start=False)]:
     P = kw.pop("P")
     with LT.Engine(chunk_walks=256, **kw) as e:
         e.graph_load(g.row_ptr, g.col, P)
@@ -59,21 +63,33 @@ with LT.Engine(path_mode=2, walk_pool_walks=500, chunk_walks=64, visit_counts=Tr
     e.walks_init_pagerank(starts, 10, 0.2, 1)
     e.run()
     e.get_paths(paths=False)
-hub = ltdist.ThreadComm.Hub(2)
+import torch  # noqa: E402
 
+with LT.Engine() as e:  # direct start from device starts
+    e.graph_load(g.row_ptr, g.col, 1)
+    e.walks_init(torch.from_numpy(starts.view(np.int32)).cuda(), LT.DEEPWALK, 10, 1)
+    e.run()
+    e.get_paths()
+d_rp = torch.from_numpy(g.row_ptr.view(np.int64)).cuda()
+d_col = torch.from_numpy(g.col.view(np.int32)).cuda()
+for layout, device_graph in [(LT.LAYOUT_AUTO, False), (LT.LAYOUT_CSR, False), (LT.LAYOUT_ADJ12, False),
+                             (LT.LAYOUT_ADJ, True), (LT.LAYOUT_CSR, True)]:
+    hub = ltdist.ThreadComm.Hub(2)
 
-def rank(r):
-    with LT.Engine(rank=r, world=2, chunk_walks=256) as e:
-        e.graph_load(g.row_ptr, g.col, 4)
-        e.walks_init(starts, LT.DEEPWALK, 10, 1)
-        comm = ltdist.ThreadComm(hub, r)
-        ltdist.run_supersteps(e, comm, "cuda")
-        ltdist.merge_paths(e, comm)
+    def rank(r):
+        with LT.Engine(rank=r, world=2, chunk_walks=256, layout=layout) as e:
+            if device_graph:
+                e.graph_load(d_rp, d_col, 4)
+            else:
+                e.graph_load(g.row_ptr, g.col, 4)
+            e.walks_init(starts, LT.DEEPWALK, 10, 1)
+            comm = ltdist.ThreadComm(hub, r)
+            ltdist.run_supersteps(e, comm, "cuda")
+            ltdist.merge_paths(e, comm)
 
-
-th = [threading.Thread(target=rank, args=(r,)) for r in range(2)]
-for t in th:
-    t.start()
-for t in th:
-    t.join()
+    th = [threading.Thread(target=rank, args=(r,)) for r in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
 print("sanitize_run done")
