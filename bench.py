@@ -69,6 +69,7 @@ def parse():
                          "and free the device col (the steps never read it): room for the path matrix")
     ap.add_argument("--ilp", type=int, default=0)
     ap.add_argument("--gather-mode", type=int, default=3, help="lt_config.gather_mode: 3 L2 hints (default), 0 none")
+    ap.add_argument("--l2-persist", type=int, default=0, help="lt_config.l2_persist: 1 = L2 set-aside for evict_last lines")
     ap.add_argument("--path-mode", type=int, default=0)
     ap.add_argument("--refill", type=int, default=0)
     ap.add_argument("--direct-start", type=int, default=1,
@@ -329,7 +330,8 @@ def main():
                     timing=True, layout=args.layout, ilp=args.ilp, path_mode=args.path_mode,
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill,
-                    continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start))
+                    continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start),
+                    l2_persist=args.l2_persist)
     torch.cuda.empty_cache()  # generator scratch back to the device before the library reserves its graph
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)

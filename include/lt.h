@@ -143,7 +143,9 @@ typedef struct lt_config {
                                  takes walk j straight from starts[j] (device starts must then stay
                                  valid until lt_run returns, as with walk admission); 1 -> off (records
                                  always built by the init kernel). Parity-neutral. */
-  uint32_t reserved1;
+  uint32_t l2_persist;        /* L2 set-aside for the lines the kernels tag evict_last (visit counters,
+                                 row_ptr): 0 -> leave cudaLimitPersistingL2CacheSize as it is; 1 -> set
+                                 it to the device maximum at lt_create (process-wide device state) */
 } lt_config;
 
 typedef struct lt_stats {
@@ -180,6 +182,7 @@ typedef struct lt_stats {
                                   (layout CSR) or augmented (ADJ / ADJ12) entries of the owned
                                   vertices (all vertices when world == 1);
                                   0 out of core (see pool_blocks x pool_block_bytes) */
+  uint64_t l2_persist_bytes;   /* cudaLimitPersistingL2CacheSize set at lt_create (lt_config.l2_persist) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

@@ -77,7 +77,20 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
     size_t g = c.l2_fetch_bytes ? c.l2_fetch_bytes : 32;
     CK(cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, g));
   }
-  cudaError_t e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
+  if (c.l2_persist > 1) {
+    lt_destroy(ctx);
+    return fail(LT_ERR_INVALID, "l2_persist must be 0 or 1");
+  }
+  cudaError_t e = cudaSuccess;
+  if (c.l2_persist == 1) {  // evict_last lines (visit counters, row_ptr) get an L2 set-aside to stay in
+    int mx = 0;
+    size_t got = 0;
+    e = cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, c.device);
+    if (e == cudaSuccess && mx > 0) e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)mx);
+    if (e == cudaSuccess) e = cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize);
+    ctx->stats.l2_persist_bytes = got;
+  }
+  if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
   if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_ctr, sizeof(lt::Counters));
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_ctr, sizeof(lt::Counters), cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_free, sizeof(int), cudaHostAllocMapped);

@@ -65,7 +65,7 @@ class Config(ctypes.Structure):
         ("reserved0", ctypes.c_uint32),
         ("walk_pool_walks", ctypes.c_uint64),
         ("direct_start", ctypes.c_uint32),
-        ("reserved1", ctypes.c_uint32),
+        ("l2_persist", ctypes.c_uint32),
     ]
 
 
@@ -77,7 +77,7 @@ class Stats(ctypes.Structure):
         ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
-            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes")]
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes")]
 
 
 class PoolState(ctypes.Structure):
@@ -171,7 +171,7 @@ class Engine:
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
                  visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
-                 direct_start: bool = True):
+                 direct_start: bool = True, l2_persist: int = 0):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -196,6 +196,7 @@ class Engine:
         cfg.continue_resident = int(bool(continue_resident))
         cfg.walk_pool_walks = int(walk_pool_walks)
         cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
+        cfg.l2_persist = int(l2_persist)
         cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device

@@ -42,6 +42,7 @@ def main():
     ap.add_argument("--partitions", type=int, default=0, help="0: one per rank")
     ap.add_argument("--legacy", action="store_true")
     ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--refill", type=int, default=0, help="lt_config.refill: 0 auto, 1 off, 2 on")
     a = ap.parse_args()
     import torch
 
@@ -54,7 +55,7 @@ def main():
     out = {}
 
     def rank_main(r, hub, res):
-        with LT.Engine(rank=r, world=a.world, timing=True) as e:
+        with LT.Engine(rank=r, world=a.world, timing=True, refill=a.refill) as e:
             e.graph_load(g.row_ptr, g.col, P)
             comm = ltdist.ThreadComm(hub, r)
             for rep in range(a.reps + 1):
@@ -81,7 +82,8 @@ def main():
         t.join()
     wall = min(max(res[r][i][0] for r in range(a.world)) for i in range(a.reps))
     ss = res[0][-1][1]
-    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "wall_ms": wall * 1e3,
+    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "refill": a.refill,
+           "wall_ms": wall * 1e3,
            "supersteps": ss, "ms_per_superstep": wall * 1e3 / ss, "n": g.n,
            "library": os.environ.get("LT_LIBRARY", "liblt.so")}
     print(json.dumps(out), flush=True)
