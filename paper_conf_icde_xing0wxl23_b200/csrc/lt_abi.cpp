@@ -140,6 +140,7 @@ void lt_destroy(lt_ctx* ctx) {
   }
   if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
   cudaFree(ctx->d_starts);
+  cudaFree(ctx->d_starts_all);
   cudaFree(ctx->d_visits);
   cudaFree(ctx->d_visits32);
   cudaFree(ctx->d_slots);
@@ -469,13 +470,15 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
 lt_status lt_walks_init_ex(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device, uint64_t first_walk_id,
                            lt_app app, double param, uint64_t seed) {
   if (app == LT_APP_PAGERANK) return fail(LT_ERR_INVALID, "PageRank takes a length and p: use lt_walks_init_pagerank");
+  on_device = on_device ? 1 : 0;
   if (app == LT_APP_DEEPWALK) return walks_init_impl(ctx, W, starts, on_device, first_walk_id, app, param, 0.0, seed);
   return walks_init_impl(ctx, W, starts, on_device, first_walk_id, app, 0.0, param, seed);
 }
 
 lt_status lt_walks_init_pagerank(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
                                  uint64_t first_walk_id, uint32_t length, double restart_p, uint64_t seed) {
-  return walks_init_impl(ctx, W, starts, on_device, first_walk_id, LT_APP_PAGERANK, (double)length, restart_p, seed);
+  return walks_init_impl(ctx, W, starts, on_device ? 1 : 0, first_walk_id, LT_APP_PAGERANK, (double)length, restart_p,
+                         seed);
 }
 
 static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
@@ -510,7 +513,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.h2d_bytes = 0;
   ctx->stats.d2h_bytes = 0;
   cudaStream_t s = ctx->stream;
-  // starts
+  // starts (on_device: 1 = caller's device array, validated below; 2 = internal, already validated)
   const uint32_t* d_starts = starts;
   if (!on_device) {
     for (uint64_t i = 0; i < W; ++i)
@@ -547,7 +550,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const bool narrow = ctx->cfg.visit_counts == 1 && (uint64_t)W * stride < 0xFFFFFFFFull;
   if (ctx->cfg.visit_counts) CK(ensure(ctx->d_visits, ctx->visits_cap, ctx->n));
   if (narrow) CK(ensure(ctx->d_visits32, ctx->visits32_cap, ctx->n));
-  if (on_device && W) {
+  if (on_device == 1 && W) {
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
     CK(lt::launch_check_starts(d_starts, W, ctx->n, ctx->d_small + 2, s));
     uint32_t bad = 0;
@@ -928,6 +931,8 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_run_to_host before lt_graph_load");
   if (ctx->cfg.visit_counts) return fail(LT_ERR_INVALID, "lt_run_to_host does not accumulate visit counts; use lt_run");
   if (ctx->cfg.path_mode == 2) return fail(LT_ERR_INVALID, "lt_run_to_host needs stored paths (path_mode 0 or 1)");
+  if (app != LT_APP_DEEPWALK && app != LT_APP_PPR)
+    return fail(LT_ERR_INVALID, "lt_run_to_host runs DeepWalk or PPR walks (PageRank: lt_walks_init_pagerank + lt_run)");
   CK(cudaSetDevice(ctx->cfg.device));
   if (chunks == 0) chunks = 8;
   const uint64_t wc = std::max<uint64_t>((W + chunks - 1) / chunks, 1);
@@ -938,6 +943,19 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
       CK(cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming));
       CK(cudaEventRecord(ctx->ev_copied[i], ctx->copy_stream));
     }
+  }
+  // All starts go H2D once (pinned host memory: at the link rate) and are range-checked on the device,
+  // instead of a host loop over W starts in front of every range's walk: each range then starts from
+  // its slice of the validated device array.
+  CK(ensure(ctx->d_starts_all, ctx->starts_all_cap, std::max<uint64_t>(W, 1)));
+  if (W) {
+    CK(cudaMemcpyAsync(ctx->d_starts_all, starts, W * sizeof(uint32_t), cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), ctx->stream));
+    CK(lt::launch_check_starts(ctx->d_starts_all, W, ctx->n, ctx->d_small + 2, ctx->stream));
+    uint32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, ctx->d_small + 2, sizeof(uint32_t), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (bad) return fail(LT_ERR_INVALID, "a start vertex >= n");
   }
   // the chunk buffers stand in for the context's path/length arrays while this call runs
   uint32_t* save_p = ctx->d_paths;
@@ -956,7 +974,9 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
     ctx->paths_cap = ctx->paths2_cap[b];
     ctx->d_lengths = ctx->d_lengths2[b];
     ctx->lengths_cap = ctx->lengths2_cap[b];
-    st = lt_walks_init_ex(ctx, n, starts + a, 0, first_walk_id + a, app, param, seed);
+    st = app == LT_APP_DEEPWALK
+             ? walks_init_impl(ctx, n, ctx->d_starts_all + a, 2, first_walk_id + a, app, param, 0.0, seed)
+             : walks_init_impl(ctx, n, ctx->d_starts_all + a, 2, first_walk_id + a, app, 0.0, param, seed);
     if (st == LT_OK) st = lt_run(ctx);
     ctx->d_paths2[b] = ctx->d_paths;  // (re)allocated by walks_init as needed
     ctx->paths2_cap[b] = ctx->paths_cap;
@@ -972,7 +992,7 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
     run_ms += ctx->stats.run_ms;
     init_ms += ctx->stats.init_ms;
     update_ms += ctx->stats.update_ms;
-    h2d += ctx->stats.h2d_bytes;
+
     if (n && compact) {  // ragged copy-out: offsets + packed vertices of this range
       uint64_t tot = 0;
       st = pack_compact(ctx, ctx->d_paths2[b], ctx->d_lengths2[b], n, b, vbase, &tot);
@@ -1025,7 +1045,7 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
   ctx->stats.run_ms = run_ms;
   ctx->stats.init_ms = init_ms;
   ctx->stats.update_ms = update_ms;
-  ctx->stats.h2d_bytes = h2d;
+  ctx->stats.h2d_bytes = h2d + W * sizeof(uint32_t);
   ctx->stats.d2h_bytes = d2h;
   return LT_OK;
 }

@@ -93,6 +93,8 @@ struct lt_ctx {
   bool visits_ready = false;
   uint32_t* d_starts = nullptr;
   size_t starts_cap = 0;
+  uint32_t* d_starts_all = nullptr;  // lt_run_to_host*: every start, copied and validated once
+  size_t starts_all_cap = 0;
   // walk admission (lt_config.walk_pool_walks): walks [0, admitted) have been created; at most
   // cap_walks are live; the rest are admitted from adm_starts as walks end
   const uint32_t* adm_starts = nullptr;

@@ -400,6 +400,28 @@ def test_run_to_host_compact(gpu, cfg1, chunks, app, param):
     assert st["steps"] == osteps
 
 
+def test_run_to_host_validates_starts_on_device(gpu, cfg1):
+    """lt_run_to_host copies every start once and range-checks it on the device: a bad start anywhere
+    (here in the last range) fails the call before any walk runs; PageRank is refused (no visit
+    counts on this path); the context is usable afterwards."""
+    W = 3000
+    starts = lt_inputs.deepwalk_starts(W, cfg1.n)
+    bad = starts.copy()
+    bad[-1] = cfg1.n
+    with LT.Engine() as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, 1)
+        with pytest.raises(LT.LTError, match="start"):
+            e.run_to_host(bad, LT.DEEPWALK, 5, 1, chunks=4)
+        with pytest.raises(LT.LTError, match="PageRank"):
+            e.run_to_host(starts, LT.PAGERANK, 5, 1, chunks=4)
+        paths = np.empty((W, 6), dtype=np.uint32)
+        lengths = np.empty(W, dtype=np.uint32)
+        e.run_to_host(starts, LT.DEEPWALK, 5, 1, paths=paths, lengths=lengths, chunks=4)
+    op, ol, _, _ = run_oracle(cfg1, starts, LT.DEEPWALK, 5, 1)
+    np.testing.assert_array_equal(paths, op)
+    np.testing.assert_array_equal(lengths, ol)
+
+
 def test_compact_capacity_error(gpu, cfg1):
     starts = lt_inputs.ppr_starts(2000, cfg1.argmax_deg)
     with LT.Engine() as e:
