@@ -80,6 +80,7 @@ def parse():
     ap.add_argument("--graph-pool-gb", type=float, default=0.0,
                     help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
     ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
+    ap.add_argument("--ooc-prefetch", type=int, default=1, help="out-of-core: load the next partition during a compute")
     ap.add_argument("--continue-resident", type=int, default=1,
                     help="out-of-core: walks keep stepping into partitions resident in the graph pool (f4)")
     ap.add_argument("--app", default="config", choices=["config", "deepwalk", "ppr", "pagerank"],
@@ -331,7 +332,7 @@ def main():
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill,
                     continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start),
-                    l2_persist=args.l2_persist)
+                    l2_persist=args.l2_persist, ooc_prefetch=bool(args.ooc_prefetch))
     torch.cuda.empty_cache()  # generator scratch back to the device before the library reserves its graph
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
@@ -475,7 +476,7 @@ def main():
                      "pool_blocks": last["pool_blocks"], "pool_block_bytes": last["pool_block_bytes"],
                      "iterations": last["iterations"], "explicit_copies": last["explicit_copies"],
                      "pool_hits": last["pool_hits"], "zero_copy_launches": last["zero_copy_launches"],
-                     "preemptive_launches": last["preemptive_launches"],
+                     "preemptive_launches": last["preemptive_launches"], "prefetches": last["prefetches"],
                      "hit_rate": last["pool_hits"] / max(1, last["iterations"]),
                      "continue_resident": bool(args.continue_resident),
                      "visits_per_step": last["visits"] / max(1, last["steps"])}

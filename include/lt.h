@@ -112,7 +112,9 @@ typedef struct lt_config {
                                  invalid; lengths and stats still exact) */
   uint32_t zero_copy;         /* out-of-core: 1 -> adaptive zero copy when alpha*w < S_p */
   uint32_t zc_alpha_bytes;    /* alpha, bytes per walk; 0 -> 256 */
-  uint32_t pad0;
+  uint32_t ooc_prefetch;      /* out-of-core: 1 -> before computing the selected partition, start loading the
+                                 non-resident partition with the most walks into another block so the host
+                                 link stays busy during the compute (parity-neutral); 0 -> off */
   uint64_t graph_pool_bytes;  /* 0 -> HBM-resident graph; > 0 -> out-of-core: the CSR stays in pinned
                                  host memory and a device graph pool of this many bytes caches
                                  partitions. Every partition must fit one block
@@ -183,6 +185,7 @@ typedef struct lt_stats {
                                   vertices (all vertices when world == 1);
                                   0 out of core (see pool_blocks x pool_block_bytes) */
   uint64_t l2_persist_bytes;   /* cudaLimitPersistingL2CacheSize set at lt_create (lt_config.l2_persist) */
+  uint64_t prefetches;         /* out-of-core loads started ahead of the selection (lt_config.ooc_prefetch) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

@@ -674,6 +674,7 @@ lt_status lt_run(lt_ctx* ctx) {
   ctx->stats.pool_hits = 0;
   ctx->stats.zero_copy_launches = 0;
   ctx->stats.preemptive_launches = 0;
+  ctx->stats.prefetches = 0;
   ctx->stats.graph_h2d_bytes = 0;
   ctx->stats.chunks_free_min = ctx->stats.chunks_total;
   ctx->nev = 0;

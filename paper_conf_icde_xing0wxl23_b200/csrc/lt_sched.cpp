@@ -236,6 +236,47 @@ lt_status compute_block(lt_ctx* ctx, uint32_t k) {
   return LT_OK;
 }
 
+// Prefetch (lt_config.ooc_prefetch): with partition i about to be computed and at most one load in
+// flight (typically i's own), queue the load of the non-resident partition with the most pending walks (one a zero-copy launch would
+// not serve) into a free block or the block of the resident partition with the fewest walks — never
+// i's block. The victim is withdrawn from the continuation table BEFORE i's launch is enqueued, so the
+// load only waits for the launches already issued and overlaps the compute of i. The next selection
+// then usually finds that partition resident. Uses the counts of the last read (parity-neutral: only
+// residency changes).
+lt_status prefetch(lt_ctx* ctx, uint32_t i, bool selective, uint64_t alpha, uint64_t seq) {
+  OutOfCore& o = ctx->ooc;
+  if (!ctx->cfg.ooc_prefetch || o.m_g < 2) return LT_OK;
+  uint32_t in_flight = 0;  // keep at most one load queued behind the one in flight
+  for (uint32_t q = 0; q < o.m_g; ++q)
+    if (o.part_in[q] >= 0 && !event_done(o.ev_ready[q])) ++in_flight;
+  if (in_flight >= 2) return LT_OK;
+  int j = -1;
+  for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k) {
+    if (k == i || o.block_of[k] >= 0 || !pending(ctx, k)) continue;
+    if (ctx->cfg.zero_copy && alpha * pending(ctx, k) < partition_bytes(ctx, k)) continue;
+    if (j < 0 || pending(ctx, k) > pending(ctx, (uint32_t)j)) j = (int)k;
+  }
+  if (j < 0) return LT_OK;
+  const int bi = o.block_of[i];
+  int b = -1;
+  for (uint32_t q = 0; q < o.m_g && b < 0; ++q)
+    if (o.part_in[q] < 0 && (int)q != bi) b = (int)q;
+  if (b < 0) {
+    for (uint32_t q = 0; q < o.m_g; ++q) {
+      if ((int)q == bi) continue;
+      if (b < 0) { b = (int)q; continue; }
+      if (selective ? pending(ctx, o.part_in[q]) < pending(ctx, o.part_in[b]) : o.loaded_at[q] < o.loaded_at[b])
+        b = (int)q;
+    }
+    // only displace a partition holding fewer walks than the one brought in
+    if (b < 0 || pending(ctx, o.part_in[b]) >= pending(ctx, (uint32_t)j)) return LT_OK;
+  }
+  ctx->stats.prefetches++;
+  lt_status st = load_partition(ctx, (uint32_t)j, b, seq);
+  ctx->stats.explicit_copies--;  // explicit_copies counts the loads of selected partitions (Table III)
+  return st;
+}
+
 }  // namespace
 
 lt_status run_out_of_core(lt_ctx* ctx) {
@@ -275,6 +316,8 @@ lt_status run_out_of_core(lt_ctx* ctx) {
     ctx->stats.iterations++;
     if (o.block_of[i] >= 0) {  // graph-pool hit
       ctx->stats.pool_hits++;
+      st = prefetch(ctx, i, selective, alpha, ++seq);
+      if (st != LT_OK) return st;
       st = compute_block(ctx, i);
       if (st != LT_OK) return st;
       continue;
@@ -322,6 +365,8 @@ lt_status run_out_of_core(lt_ctx* ctx) {
       if (st != LT_OK) return st;
       if (ctx->h_ctr->err) return LT_OK;
     }
+    st = prefetch(ctx, i, selective, alpha, ++seq);
+    if (st != LT_OK) return st;
     st = compute_block(ctx, i);
     if (st != LT_OK) return st;
   }

@@ -55,7 +55,7 @@ class Config(ctypes.Structure):
         ("path_mode", ctypes.c_uint32),
         ("zero_copy", ctypes.c_uint32),
         ("zc_alpha_bytes", ctypes.c_uint32),
-        ("pad0", ctypes.c_uint32),
+        ("ooc_prefetch", ctypes.c_uint32),
         ("graph_pool_bytes", ctypes.c_uint64),
         ("rank", ctypes.c_uint32),
         ("world", ctypes.c_uint32),
@@ -77,7 +77,7 @@ class Stats(ctypes.Structure):
         ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
-            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes")]
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes", "prefetches")]
 
 
 class PoolState(ctypes.Structure):
@@ -171,7 +171,7 @@ class Engine:
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
                  visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
-                 direct_start: bool = True, l2_persist: int = 0):
+                 direct_start: bool = True, l2_persist: int = 0, ooc_prefetch: bool = False):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -197,6 +197,7 @@ class Engine:
         cfg.walk_pool_walks = int(walk_pool_walks)
         cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
         cfg.l2_persist = int(l2_persist)
+        cfg.ooc_prefetch = int(bool(ooc_prefetch))
         cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
         self.rank, self.world, self.device = rank, world, device

@@ -45,10 +45,12 @@ def g14():
                                     LT.POLICY_PREEMPTIVE_ONLY])
 @pytest.mark.parametrize("blocks", [1, 2, 5])
 @pytest.mark.parametrize("zero_copy", [False, True])
-def test_out_of_core_exact(gpu, g14, policy, blocks, zero_copy):
+@pytest.mark.parametrize("prefetch", [False, True])
+def test_out_of_core_exact(gpu, g14, policy, blocks, zero_copy, prefetch):
     P = 16
     starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
-    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy)
+    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy,
+                             ooc_prefetch=prefetch)
     op, ol, osteps, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
     np.testing.assert_array_equal(lengths, ol)
     np.testing.assert_array_equal(paths, op)
@@ -59,6 +61,8 @@ def test_out_of_core_exact(gpu, g14, policy, blocks, zero_copy):
     assert st["graph_h2d_bytes"] > 0 or st["zero_copy_launches"] > 0
     if policy in (LT.POLICY_ROUND_ROBIN, LT.POLICY_SELECTIVE_ONLY):
         assert st["preemptive_launches"] == 0
+    if not prefetch or blocks == 1:
+        assert st["prefetches"] == 0
 
 
 @pytest.mark.parametrize("P,blocks", [(4, 1), (64, 3), (64, 64)])
@@ -115,18 +119,22 @@ def test_scheduling_counters_table3_shape(gpu):
 @pytest.mark.parametrize("policy", [LT.POLICY_SELECTIVE, LT.POLICY_ROUND_ROBIN])
 @pytest.mark.parametrize("blocks", [1, 3, 16])
 @pytest.mark.parametrize("zero_copy", [False, True])
-def test_continue_into_resident_partitions_exact(gpu, g14, policy, blocks, zero_copy):
+@pytest.mark.parametrize("prefetch", [False, True])
+def test_continue_into_resident_partitions_exact(gpu, g14, policy, blocks, zero_copy, prefetch):
     """with continuation a walk that leaves the launched partition for another
     partition resident in the graph pool keeps stepping there. Paths are unchanged (parity-neutral);
     with more than one block resident, walks need fewer visits (bucket round trips)."""
     P = 16
     starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
     paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy,
-                             continue_resident=True)
+                             continue_resident=True, ooc_prefetch=prefetch)
     op, ol, osteps, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
     np.testing.assert_array_equal(lengths, ol)
     np.testing.assert_array_equal(paths, op)
     assert st["steps"] == osteps
+    assert st["iterations"] == st["pool_hits"] + st["explicit_copies"] + st["zero_copy_launches"]
+    if prefetch:
+        return
     _, _, st0 = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, policy=policy, zero_copy=zero_copy)
     if blocks == P:  # everything resident after the first loads: most steps continue in-kernel
         assert st["visits"] < st0["visits"] // 2
@@ -140,7 +148,8 @@ def test_continue_resident_ppr_and_pagerank(gpu, g14, app, param):
     pool = block_bytes(g14, P) * blocks
     starts = (lt_inputs.ppr_starts(20_000, g14.argmax_deg) if app == LT.PPR
               else lt_inputs.deepwalk_starts(g14.n, g14.n))
-    with LT.Engine(graph_pool_bytes=pool, continue_resident=True, zero_copy=True, visit_counts=True) as e:
+    with LT.Engine(graph_pool_bytes=pool, continue_resident=True, zero_copy=True, visit_counts=True,
+                   ooc_prefetch=True) as e:
         e.graph_load(g14.row_ptr, g14.col, P)
         if app == LT.PAGERANK:
             e.walks_init_pagerank(starts, 12, param, 5)
