@@ -404,11 +404,15 @@ def main():
         peak, peak_src = float(json.load(open(peaks_path))["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
     achieved = (alg_bytes / upd_launches) / (upd_ms / upd_launches / 1000.0) / 1e9 if upd_ms > 0 else None
     traffic = None
+    sector_eff = None
     prof = os.path.join(ROOT, "profiles", "update_kernel_traffic.json")
     if os.path.exists(prof):
         pj = json.load(open(prof))
         if pj.get("config_key") == f"cfg{args.config}-P{P}-layout{args.layout}":
             traffic = pj.get("dram_bytes_per_launch")
+            sector_eff = {"ld_bytes_per_sector": pj.get("sector_efficiency_ld_bytes"),
+                          "st_bytes_per_sector": pj.get("sector_efficiency_st_bytes"),
+                          "source": "ncu, profiles/update_kernel_traffic.json"}
     layout = stats[-1]["layout"]
     # DRAM-missing random gathers issued by the update kernel: one per step (ADJ: adj entry;
     # CSR: col entry) + the row_ptr line per step (CSR) or per visit (ADJ)
@@ -427,7 +431,7 @@ def main():
             "frac": (achieved / peak) if achieved else None, "traffic": traffic,
             "kernel": "k_update", "launches": upd_launches, "avg_launch_ms": upd_ms / max(1, upd_launches),
             "alg_bytes_per_step": alg_bytes / max(1, steps_k), "peak_source": peak_src,
-            "update_share_of_step": upd_ms / ms, "gather": gather}
+            "update_share_of_step": upd_ms / ms, "gather": gather, "sector_efficiency": sector_eff}
 
     # ---- extra partition-count sweep (context; the headline uses P above)
     sweep = {}
