@@ -108,10 +108,22 @@ class ThreadComm:
         offs = [0]
         for c in send_counts:
             offs.append(offs[-1] + c)
-        allv = self._gather((send, offs))
-        parts = [allv[r][0][allv[r][1][self.rank]: allv[r][1][self.rank + 1]] for r in range(self.world)]
-        parts = [p.to(send.device) for p in parts]
-        return torch.cat(parts) if parts else send[:0]
+        # the copies out of the other ranks' send buffers must be complete before the last barrier:
+        # once past it a sender may start its next superstep and pack into the same buffer; and the
+        # sender's pack (on the engine's stream) must be complete before anyone reads its buffer
+        if send.is_cuda:
+            torch.cuda.synchronize(send.device)
+        self.hub.barrier.wait()
+        self.hub.slots[self.rank] = (send, offs)
+        self.hub.barrier.wait()
+        allv = list(self.hub.slots)
+        parts = [allv[r][0][allv[r][1][self.rank]: allv[r][1][self.rank + 1]].to(send.device, copy=True)
+                 for r in range(self.world)]
+        out = torch.cat(parts) if parts else send[:0].clone()
+        if out.is_cuda:
+            torch.cuda.current_stream(out.device).synchronize()
+        self.hub.barrier.wait()
+        return out
 
     def allreduce_sum(self, x: int, device) -> int:
         return sum(self._gather(int(x)))
