@@ -55,7 +55,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.world == 0) c.world = 1;
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
-  if (c.refill > 3) return fail(LT_ERR_INVALID, "bad refill");
+  if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
   if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
   if (c.direct_start > 1) return fail(LT_ERR_INVALID, "direct_start must be 0 (auto) or 1 (off)");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
@@ -533,14 +533,11 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // the lane-refill kernel (the P == 1 default) takes walk j straight from starts[j]: k_init (16-B
   // record write + read back + one bucket cursor atomic per warp) is skipped and, since a walk never
   // leaves the only partition, no record is ever appended: the pool keeps only its per-bucket slack
-  const bool direct = ctx->cfg.direct_start == 0 && ctx->cfg.refill != 1 && ctx->P == 1 &&
+  const bool direct = ctx->cfg.direct_start == 0 && (ctx->cfg.refill == 0 || ctx->cfg.refill == 2) && ctx->P == 1 &&
                       ctx->world == 1 && !ctx->ooc.on && cap == W;
   const uint64_t wc = direct ? 0 : (cap + C - 1) / C;
-  // the ring spans the partially consumed head chunk, the chunks of pending walks, the partially
-  // filled cursor chunk and kAhead chunks installed ahead of it; the pool adds, per bucket, those
-  // partial and installed-ahead chunks, plus a launch's consumed chunks (retired at its end)
-  const uint64_t ring_len = wc + 2 + lt::kAhead;
-  const uint64_t num_chunks = 2 * wc + (2 + lt::kAhead) * (uint64_t)ctx->nb + 64;
+  const uint64_t ring_len = wc + 2;
+  const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
   const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
   // path_mode 2 stores no path entries (the paper's accounting): no path matrix
@@ -610,10 +607,10 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : ((p.wk.adj || p.wk.adj12) ? 1u : 2u);
   // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
   // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
-  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : ctx->cfg.refill == 3 ? 2u : 0u;
+  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
-  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill);
+  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0);
   p.direct = direct ? lt::Direct{d_starts, W} : lt::Direct{nullptr, 0};
   ctx->stats.direct_start = direct ? 1 : 0;
 

@@ -9,7 +9,6 @@ namespace lt {
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;   // empty ring slot / unused path slot
 constexpr uint32_t kErrOOM = 1u;           // device error bits
 constexpr uint32_t kErrRing = 2u;
-constexpr uint32_t kAhead = 2u;            // a6: chunks a bucket's ring is installed ahead of its cursor
 
 // A walk record (D5): 16 bytes, one 128-bit load/store.
 //   x = local walk index (row of the path matrix; walk_id = first_walk_id + x)
@@ -17,9 +16,8 @@ constexpr uint32_t kAhead = 2u;            // a6: chunks a bucket's ring is inst
 
 // Walk pool (a6): `slots` is an arena of num_chunks chunks of C records.
 // Bucket k is the position range [head[k], cursor[k]) (monotone u64 counters); position pos lives
-// in chunk ring[k*ring_len + (pos/C) % ring_len] at offset pos % C. Ring slots are installed
-// kAhead chunks ahead: chunk c exactly once, by the writer whose claim holds the first slot of chunk
-// c - kAhead (chunks 0..kAhead at pool reset).
+// in chunk ring[k*ring_len + (pos/C) % ring_len] at offset pos % C. Ring slots are installed on
+// demand: exactly once per chunk, by the writer whose claim holds the chunk's first slot.
 struct Pool {
   uint4* slots;
   uint32_t C, c_shift;
@@ -103,7 +101,7 @@ struct Params {
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;
-  uint32_t refill;  // 1: lane-refill update kernel (k_update_rf); 2: prefetching lane refill (k_update_pf)
+  uint32_t refill;  // 1: lane-refill update kernel (k_update_rf)
 };
 
 // launchers (lt_kernels.cu); all asynchronous on `s`
@@ -138,7 +136,7 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
                              cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
                                cudaStream_t s);
-int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill);  // resident blocks per SM (update kernel)
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill);  // resident blocks per SM (update kernel)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

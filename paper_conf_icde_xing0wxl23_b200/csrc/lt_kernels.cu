@@ -83,14 +83,11 @@ __device__ __forceinline__ uint32_t find_partition(const uint32_t* B, uint32_t P
   return lo;
 }
 
-// a6: chunk installation, kAhead chunks ahead of the writers. Chunk c of bucket `dest` is installed
-// exactly once, by the writer whose claimed position range holds the first slot of chunk c - kAhead
-// (chunks 0..kAhead-1 of every bucket are installed by k_pool_reset): it pops the free stack and
-// publishes the chunk in the ring slot. Every writer into chunk c waits for that publication, which
-// was started kAhead * C appends earlier, so a wait is rare (installing on demand instead made most
-// writers into a fresh chunk wait for its installer's two atomics: 12 % of the stall samples of the
-// P = 4 update kernel). Installing never waits, and a writer only waits for a chunk installed by a
-// writer at a lower position, so the waits cannot form a cycle.
+// a6: chunk installation. Chunk cidx of bucket `dest` is installed exactly once, by the thread whose
+// claimed position range holds the chunk's first slot (cidx * C): it pops the free stack and
+// publishes the chunk in the ring slot. Every other writer into that chunk waits for the ring slot
+// to be published. Installing never waits, and a waiter only waits for a chunk whose first slot lies
+// at a lower position than its own claim, so the waits cannot form a cycle.
 __device__ uint32_t install_chunk(const Params& p, uint32_t dest, unsigned long long cidx) {
   const Pool& pl = p.pool;
   uint32_t* slot = pl.ring + (uint64_t)dest * pl.ring_len + (cidx % pl.ring_len);
@@ -119,8 +116,8 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
   const unsigned long long cmask = pl.C - 1;
   if (p.insert_mode == 1) {  // "direct write" ablation: one global atomic per walk
     const unsigned long long pos = atomicAdd(pl.cursor + dest, 1ull);
-    if ((pos & cmask) == 0) install_chunk(p, dest, (pos >> pl.c_shift) + kAhead);
-    const uint32_t c = wait_chunk(p, dest, pos >> pl.c_shift);
+    const uint32_t c = (pos & cmask) == 0 ? install_chunk(p, dest, pos >> pl.c_shift)
+                                          : wait_chunk(p, dest, pos >> pl.c_shift);
     pl.slots[((uint64_t)c << pl.c_shift) | (pos & cmask)] = rec;
     return;
   }
@@ -133,10 +130,9 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
     const uint32_t cnt = __popc(grp);  // cnt <= 32 <= C: the range touches at most two chunks
     base = atomicAdd(pl.cursor + dest, (unsigned long long)cnt);
     const unsigned long long ci0 = base >> pl.c_shift, ci1 = (base + cnt - 1) >> pl.c_shift;
-    if (ci1 != ci0) install_chunk(p, dest, ci1 + kAhead);              // chunk ci1 starts inside our range
-    else if ((base & cmask) == 0) install_chunk(p, dest, ci0 + kAhead);  // chunk ci0 starts at base
-    c0 = wait_chunk(p, dest, ci0);
-    c1 = (ci1 != ci0) ? wait_chunk(p, dest, ci1) : c0;
+    if (ci1 != ci0) c1 = install_chunk(p, dest, ci1);  // chunk ci1 starts inside our range
+    c0 = (base & cmask) == 0 ? install_chunk(p, dest, ci0) : wait_chunk(p, dest, ci0);
+    if (ci1 == ci0) c1 = c0;
   }
   base = __shfl_sync(act, base, leader);
   c0 = __shfl_sync(act, c0, leader);
@@ -882,247 +878,6 @@ __global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_
   last_cta_retire(p, (int)k, head, tail);
 }
 
-// --------------------------------------------------------- a3 + a4 + a5, prefetching lane refill
-// k_update_rf stalls the whole warp whenever a lane takes a new walk: the next gather cannot issue
-// before the new walk's dependent chain (claim atomic -> ring slot -> 16-B record -> row_ptr pair)
-// has come back, and with several partitions a walk leaves after ~1.3 steps (visits/step 0.78 at
-// P = 4 on cfg 4), so nearly every step pays that chain. Here each lane keeps a two-stage pipeline of
-// its next walks in SHARED memory, filled by cp.async (no register scoreboard is held across the
-// loop, so the step's gather never waits for them):
-//   stage 1: the next record, copied from its pool slot (16-B cp.async) in an earlier iteration;
-//   stage 2: the record after that + its row_ptr pair (two 8-B cp.async issued once stage 1 landed).
-// `cp.async.wait_all` at the top of an iteration waits only for copies issued one iteration (one
-// random-gather latency) earlier. A lane whose walk ended takes its stage-2 walk with nothing left to
-// load. Positions are assigned statically (warp g takes blocks g, g + G, g + 2G, ... of 64 positions):
-// no claim atomic on the path, and with ~2000 walks per warp per launch the imbalance is a few %.
-#ifndef LT_PF_MINB
-#define LT_PF_MINB 4
-#endif
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
-  const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
-  const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
-template <int APP, int GM, int LAY, int VIS>
-__global__ void __launch_bounds__(256, LT_PF_MINB) k_update_pf(Params p, uint32_t k) {
-  extern __shared__ uint32_t s_bounds[];
-  const Walk& wk = p.wk;
-  const Pool& pl = p.pool;
-  const uint32_t* B = stage_bounds(wk, s_bounds);
-  const unsigned long long head = pl.head[k];
-  const unsigned long long tail = pl.cursor[k];
-  const uint32_t lo = wk.bounds[k];
-  const uint32_t span = wk.bounds[k + 1] - lo;
-  const uint32_t lane = threadIdx.x & 31u;
-  const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
-  const Policies pol = make_policies();
-  const uint64_t pol_last = VIS ? make_evict_last() : 0;
-  unsigned long long my_steps = 0, my_trunc = 0;
-
-  bool has = false;                    // stage 0: the walk being stepped
-  uint4 rec = make_uint4(0, 0, 0, 0);  // .x = row, .y = v, .z = t
-  uint32_t* prow = wk.paths;
-  uint32_t pb[8];
-  uint32_t nb = 0;
-  unsigned long long off = 0;
-  uint32_t d = 0;
-  __shared__ uint4 s_rec[2][256];                // stage-1 / stage-2 records, roles swap (sel)
-  __shared__ unsigned long long s_rp[256][2];    // stage 2's row_ptr[v], row_ptr[v+1]
-  bool s1 = false, s2 = false;
-  uint32_t sel = 0;                              // s_rec[sel] holds stage 2, s_rec[sel ^ 1] stage 1
-  const uint32_t tid = threadIdx.x;
-  const unsigned long long G = (unsigned long long)gridDim.x * (blockDim.x >> 5);
-  unsigned long long q_blk = (unsigned long long)blockIdx.x * (blockDim.x >> 5) + (tid >> 5);
-  unsigned long long q_cur = 0, q_end = 0;
-  bool drained = false;
-  __shared__ uint4 s_qr[8][2 * 32];
-  __shared__ uint32_t s_qd[8][2 * 32];
-  const uint32_t wib = tid >> 5;
-  uint32_t q_cnt = 0;
-#pragma unroll
-  for (int q = 0; q < 8; ++q) pb[q] = 0;
-
-  for (;;) {
-    cp_async_wait_all();  // the copies issued one iteration ago
-    // ---- (a) a lane whose walk ended takes its stage-2 walk (record, offset and degree in smem)
-    if (!has && s2) {
-      rec = s_rec[sel][tid];
-      has = true;
-      s2 = false;
-      if (rec.w) {  // a direct-start walk (a2): its first visit
-        rec.w = 0;
-        if (wk.path_mode == 1) wk.paths[(uint64_t)rec.x * wk.pitch] = rec.y;
-        count_visit<VIS>(wk, rec.y, pol_last);
-      }
-      if (LAY != 0) {
-        off = s_rp[tid][0];
-        d = (uint32_t)(s_rp[tid][1] - off);
-      }
-      prow = wk.paths + (uint64_t)rec.x * wk.pitch;
-      pb[7] = rec.y;
-      nb = ((rec.z & 7u) == 0) ? 1u : 0u;
-    }
-    // ---- (b) stage 1 -> stage 2: issue the row_ptr pair of the record that landed
-    if (!s2 && s1) {
-      sel ^= 1u;
-      s2 = true;
-      s1 = false;
-      if (LAY != 0) {
-        const uint32_t v = s_rec[sel][tid].y;
-        cp_async8(&s_rp[tid][0], wk.row_ptr + v);
-        cp_async8(&s_rp[tid][1], wk.row_ptr + v + 1);
-      }
-    }
-    // ---- (c) stage-1 refill from the warp's statically assigned positions
-    uint32_t need = __ballot_sync(kFull, !s1);
-    while (need && !drained) {
-      if (q_cur >= q_end) {
-        const unsigned long long base = head + q_blk * kRefill;
-        if (base >= tail) { drained = true; break; }
-        q_cur = base;
-        q_end = (base + kRefill < tail) ? base + kRefill : tail;
-        q_blk += G;
-      }
-      const uint32_t avail = (q_end - q_cur < 32ull) ? (uint32_t)(q_end - q_cur) : 32u;
-      const uint32_t r = __popc(need & lanemask_lt());
-      if (!s1 && r < avail) {
-        const unsigned long long pos = q_cur + r;
-        uint4* dst = &s_rec[sel ^ 1u][tid];
-        if (pos < p.direct.count) {  // direct start (a2): the new walk's record {pos, starts[pos], 0, 1}
-          dst->x = (uint32_t)pos;
-          dst->z = 0u;
-          dst->w = 1u;
-          cp_async4(&dst->y, p.direct.starts + pos);
-        } else {
-          const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
-          cp_async16(dst, pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
-        }
-        s1 = true;
-      }
-      q_cur += (avail < (uint32_t)__popc(need)) ? avail : (uint32_t)__popc(need);
-      need = __ballot_sync(kFull, !s1);
-    }
-    cp_async_commit();
-    if (!__any_sync(kFull, has || s1 || s2)) break;
-    // ---- one step of every lane that holds a walk (as in k_update_rf)
-    bool done = false, left = false, trunc = false;
-    if (has) {
-      if (APP != 1 && rec.z == wk.length) {
-        done = true;
-      } else if (APP == 1 && rec.z == wk.lmax) {
-        done = true;
-        trunc = true;
-      } else {
-        if (LAY == 0) {
-          const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
-          const unsigned long long r0 = ld_rp(rp), rr = ld_rp(rp + 1);
-          off = r0 - wk.ebase;
-          d = (uint32_t)(rr - r0);
-        }
-        const uint64_t wid = wk.first_walk_id + rec.x;
-        const uint4 b = philox10(make_uint4(rec.z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
-        const bool restart = APP == 2 && b.x < wk.T;
-        if ((APP == 1 && b.x < wk.T) || (d == 0 && !restart)) {
-          done = true;
-        } else {
-          const uint32_t dd = restart ? wk.n : d;
-          const uint64_t m = (uint64_t)b.y * dd;
-          const uint32_t idx = ((uint32_t)m < dd) ? lemire_slow(dd, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
-                                                               wk.seed_lo, wk.seed_hi)
-                                                  : (uint32_t)(m >> 32);
-          uint32_t nv;
-          if (restart) {
-            nv = idx;
-            if (LAY != 0 && idx - lo < span) {
-              off = __ldg(wk.row_ptr + idx);
-              d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
-            }
-          } else if (LAY == 0) {
-            nv = ld_col<GM>(wk.col + off + idx, pol);
-          } else if (LAY == 1) {
-            const uint4 e = ld_adj<GM>(wk.adj + (off - wk.ebase) + idx, pol);
-            nv = e.x;
-            d = e.y;
-            off = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
-          } else {
-            const Adj e = ld_adj12<GM>(wk.adj12, off - wk.ebase + idx, pol);
-            nv = e.u;
-            d = e.deg;
-            off = e.off;
-          }
-          rec.y = nv;
-          rec.z += 1;
-          count_visit<VIS>(wk, nv, pol_last);
-          const uint32_t t = rec.z;
-          if (wk.path_mode == 0) {
-#pragma unroll
-            for (int q = 0; q < 7; ++q) pb[q] = pb[q + 1];
-            pb[7] = nv;
-            nb += 1;
-            if ((t & 7u) == 7u) {
-              if (nb == 8) {
-                st_sector(prow + (t - 7), pb, pol);
-              } else {
-#pragma unroll
-                for (int q = 0; q < 8; ++q)
-                  if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
-              }
-              nb = 0;
-            }
-          } else if (wk.path_mode == 1) {
-            prow[t] = nv;
-          }
-          left = (nv - lo >= span);
-        }
-      }
-    }
-    // ---- retire the walks that ended this step
-    const bool ended = done || left;
-    if (ended && wk.path_mode == 0) {
-      const uint32_t t = rec.z;
-#pragma unroll
-      for (int q = 0; q < 8; ++q)
-        if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
-      nb = 0;
-    }
-    if (done) {
-      wk.lengths[rec.x] = rec.z + 1;
-      my_steps += rec.z;
-      my_trunc += trunc ? 1 : 0;
-    }
-    const uint32_t lm = __ballot_sync(kFull, left);
-    if (left) {
-      const uint32_t slot = q_cnt + __popc(lm & lanemask_lt());
-      s_qr[wib][slot] = rec;
-      s_qd[wib][slot] = bucket_of(p, find_partition(B, wk.P, rec.y));
-    }
-    q_cnt += __popc(lm);
-    if (q_cnt >= 32) {
-      __syncwarp();
-      flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
-      q_cnt = 0;
-    }
-    if (ended) has = false;
-  }
-  __syncwarp();
-  flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
-  my_steps = warp_sum(my_steps);
-  my_trunc = warp_sum(my_trunc);
-  if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
-  if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
-  last_cta_retire(p, (int)k, head, tail);
-}
-
 // ---------------------------------------------------------------------------- output helpers
 __global__ void k_finalize(Params p, uint64_t W) {
   const Walk& wk = p.wk;
@@ -1285,24 +1040,16 @@ __global__ void k_pool_reset(Params p) {
   const Pool& pl = p.pool;
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  // chunks 0..kAhead-1 of every bucket are installed up front (chunk ids 0 .. npre-1, the rest free;
-  // the writer of chunk 0's first slot installs chunk kAhead), except on a direct-start bucket 0,
-  // whose positions are virtual and which never receives appends
-  const uint32_t first = p.direct.starts ? 1u : 0u;
-  const uint64_t npre = (uint64_t)(pl.nbuckets - first) * kAhead;
-  for (uint64_t i = tid; i < pl.num_chunks - npre; i += stride) pl.free_list[i] = (uint32_t)(npre + i);
+  for (uint64_t i = tid; i < pl.num_chunks; i += stride) pl.free_list[i] = (uint32_t)i;
   const uint64_t nring = (uint64_t)pl.nbuckets * pl.ring_len;
-  for (uint64_t i = tid; i < nring; i += stride) {
-    const uint64_t b = i / pl.ring_len, r = i % pl.ring_len;
-    pl.ring[i] = (b >= first && r < kAhead) ? (uint32_t)((b - first) * kAhead + r) : kEmpty;
-  }
+  for (uint64_t i = tid; i < nring; i += stride) pl.ring[i] = kEmpty;
   for (uint64_t i = tid; i < pl.nbuckets; i += stride) {
     pl.head[i] = 0;
     pl.cursor[i] = (i == 0 && p.direct.starts) ? p.direct.count : 0;  // direct start: W virtual positions
     pl.claim[i] = 0;
   }
   if (tid == 0) {
-    *pl.free_top = (int)(pl.num_chunks - npre);
+    *pl.free_top = (int)pl.num_chunks;
     p.ctr->steps = 0; p.ctr->visits = 0; p.ctr->truncated = 0; p.ctr->err = 0; p.ctr->done_ctas = 0;
   }
 }
@@ -1326,10 +1073,9 @@ int num_sms() {
 
 uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 
-int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill) {
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill) {
   int nb = 0;
-  if (refill == 2) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_pf<0, 3, 1, 0>, (int)block, 0);
-  else if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
+  if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
   else if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
   else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1, 0>, (int)block, 0);
   else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1, 0>, (int)block, 0);
@@ -1423,27 +1169,12 @@ void launch_update_rf_t(const Params& p, uint32_t k, uint32_t grid, uint32_t blo
 }
 
 template <int APP, int GM, int LAY, int VIS>
-void launch_update_pf_t(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_update_pf<APP, GM, LAY, VIS>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         kSmemBoundsCap * 4);
-    attr = true;
-  }
-  k_update_pf<APP, GM, LAY, VIS><<<grid, block, bounds_smem(p), s>>>(p, k);
-}
-
-template <int APP, int GM, int LAY, int VIS>
 void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
   if constexpr (LAY == 0) {
     if (p.cont.table) {
       launch_update_rf_t<APP, GM, LAY, VIS, 1>(p, k, grid, block, s);
       return;
     }
-  }
-  if (p.refill == 2) {
-    launch_update_pf_t<APP, GM, LAY, VIS>(p, k, grid, block, s);
-    return;
   }
   launch_update_rf_t<APP, GM, LAY, VIS, 0>(p, k, grid, block, s);
 }

@@ -35,11 +35,10 @@ def init(e, starts, app, param, seed, length=12):
 @pytest.mark.parametrize("cap", [64, 1000, 7000])
 @pytest.mark.parametrize("P", [1, 4])
 @pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 15), (LT.PPR, 0.15), (LT.PAGERANK, 0.2)])
-@pytest.mark.parametrize("refill", [0, 3])
-def test_admission_exact(gpu, cfg1, cap, P, app, param, refill):
+def test_admission_exact(gpu, cfg1, cap, P, app, param):
     W = 20_000
     starts = lt_inputs.ppr_starts(W, cfg1.argmax_deg) if app == LT.PPR else lt_inputs.deepwalk_starts(W, cfg1.n)
-    with LT.Engine(walk_pool_walks=cap, chunk_walks=64, visit_counts=True, refill=refill) as e:
+    with LT.Engine(walk_pool_walks=cap, chunk_walks=64, visit_counts=True) as e:
         e.graph_load(cfg1.row_ptr, cfg1.col, P)
         init(e, starts, app, param, 4)
         e.run()
@@ -52,7 +51,7 @@ def test_admission_exact(gpu, cfg1, cap, P, app, param, refill):
     np.testing.assert_array_equal(counts, O.visit_counts(op, ol, cfg1.n))
     assert st["steps"] == osteps
     assert st["admissions"] >= -(-W // cap) and st["peak_live"] <= cap
-    assert st["chunks_total"] <= 2 * -(-cap // 64) + (2 + 2) * P + 64  # sized by the cap, not by W (kAhead 2)
+    assert st["chunks_total"] <= 2 * -(-cap // 64) + 2 * P + 64  # the pool is sized by the cap, not by W
 
 
 def test_admission_out_of_core_with_continuation(gpu):

@@ -57,10 +57,9 @@ def g13():
 
 @pytest.mark.parametrize("world", [2, 3, 4])
 @pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
-@pytest.mark.parametrize("refill", [0, 3])
-def test_ownership_deepwalk_exact(gpu, g13, world, layout, refill):
+def test_ownership_deepwalk_exact(gpu, g13, world, layout):
     starts = lt_inputs.deepwalk_starts(3 * g13.n, g13.n)
-    res = run_owned(g13, starts, LT.DEEPWALK, 16, 2, 12, world, layout=layout, chunk_walks=512, refill=refill)
+    res = run_owned(g13, starts, LT.DEEPWALK, 16, 2, 12, world, layout=layout, chunk_walks=512)
     op, ol, osteps, _ = oracle_of(g13, starts, LT.DEEPWALK, 16, 2)
     for paths, lengths, counters, st in res:
         np.testing.assert_array_equal(lengths, ol)
