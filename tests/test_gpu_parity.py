@@ -78,6 +78,28 @@ def test_deepwalk_invariant_to_partition_count(gpu, cfg1, P):
     assert_parity(cfg1, starts, LT.DEEPWALK, 10, 1, P=min(P, cfg1.n))
 
 
+@pytest.mark.parametrize("P", [8191, 8192, 12_000, 0])
+def test_partition_bounds_beyond_shared_memory(gpu, P):
+    """Partition bounds are staged in shared memory for P < 8192 and read from global memory beyond
+    (the exit test and findPartition, a4); P = 0 here means one partition per vertex."""
+    g = _g15()
+    P = P or g.n
+    assert g.n > 12_000
+    starts = lt_inputs.deepwalk_starts(g.n, g.n)
+    st = assert_parity(g, starts, LT.DEEPWALK, 12, 5, P=P, chunk_walks=256)
+    assert st["visits"] > g.n  # walks crossed partitions
+    assert_parity(g, lt_inputs.ppr_starts(8000, g.argmax_deg), LT.PPR, 0.2, 6, P=P, chunk_walks=256)
+
+
+_G15 = {}
+
+
+def _g15():
+    if "g" not in _G15:
+        _G15["g"] = lt_inputs.rmat_cpu(15, 16 * 32_768, seed=2)
+    return _G15["g"]
+
+
 @pytest.mark.parametrize("chunk", [64, 128, 1024, 8192])
 @pytest.mark.parametrize("insert_mode", [LT.INSERT_WARP_AGGREGATED, LT.INSERT_DIRECT])
 @pytest.mark.parametrize("policy", [LT.POLICY_SELECTIVE, LT.POLICY_ROUND_ROBIN])
@@ -429,3 +451,24 @@ def test_compact_capacity_error(gpu, cfg1):
         with pytest.raises(LT.LTError) as ei:
             e.run_to_host_compact(starts, LT.PPR, 0.15, 1, vertices=np.empty(10, dtype=np.uint32))
         assert ei.value.status == LT.lt.LT_ERR_INVALID
+
+
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+def test_lemire_rejection_chain_at_degree_2_31_plus_1(gpu, layout):
+    """Reading R4 at its extreme: a vertex of degree d = 2^31 + 1 rejects each word with probability
+    (2^32 mod d) / 2^32 ~ 1/2, so the GPU's slow path walks the step's word stream well into Philox
+    blocks j >= 1 (1/16 of the draws need a fifth word). Multi-edges make the graph: hub 0 has
+    2^31 + 1 entries, entry i pointing to 1 + (i mod 65,535), and every other vertex one edge back to
+    0, so each hub step's index shows in the path (mod 65,535) and must equal the oracle's."""
+    d = (1 << 31) + 1
+    n = 1 << 16
+    col = np.empty(d + n - 1, dtype=np.uint32)
+    col[:d] = np.resize(np.arange(1, n, dtype=np.uint32), d)  # entry i -> 1 + (i mod 65,535)
+    col[d:] = 0
+    row_ptr = np.empty(n + 1, dtype=np.uint64)
+    row_ptr[0] = 0
+    row_ptr[1:] = d + np.arange(n, dtype=np.uint64)
+    g = lt_inputs.Graph(n, len(col), row_ptr, col, d, 0)
+    starts = np.zeros(20_000, dtype=np.uint32)
+    assert_parity(g, starts, LT.DEEPWALK, 12, 3, P=1, layout=layout)
+    assert_parity(g, starts, LT.PPR, 0.1, 4, P=3, layout=layout)
