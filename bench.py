@@ -88,6 +88,10 @@ def parse():
                          "(PAPER.md:287, SURVEY.md 8(f) f2) of the config's length, with visit counting")
     ap.add_argument("--restart-p", type=float, default=0.15, help="PageRank restart probability")
     ap.add_argument("--visit-counts", type=int, default=-1, help="fused visit counting: -1 auto (on for pagerank)")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
+                    help="--mode own: walks crossing ranks go through lt_exchange_pack + an NCCL all-to-all "
+                         "(nccl), or are appended by the update kernels straight into the owner's receive "
+                         "buffer over peer memory (p2p: CUDA IPC, one small all-reduce per superstep)")
     ap.add_argument("--mode", default="replicas", choices=["replicas", "own"],
                     help="N>1: replicas (each rank its own |V| walks, no collective, weak scaling) or own "
                          "(range ownership: |V| walks in total, NCCL all-to-all of crossing walks per "
@@ -352,14 +356,21 @@ def main():
             torch.cuda.synchronize()
 
     comm = None
+    p2p = own and args.exchange == "p2p"
     if own:
         from paper_conf_icde_xing0wxl23_b200 import dist as ltdist
         comm = ltdist.TorchComm()
     superstep_counters = {}
+    attached = []
 
     def one_step():
         init_walks(eng, c, starts_d, args.seed, first)
-        if own:
+        if p2p:
+            if not attached:  # receive buffers for every walk, shared once through CUDA IPC
+                ltdist.attach_peers(eng, comm, W)
+                attached.append(True)
+            superstep_counters.update(ltdist.run_supersteps_p2p(eng, comm, f"cuda:{local}"))
+        elif own:
             superstep_counters.update(ltdist.run_supersteps(eng, comm, f"cuda:{local}"))
         else:
             eng.run()
@@ -633,7 +644,7 @@ def main():
         if host_link:
             line["host_link"] = host_link
         if own:
-            line["ownership"] = dict(superstep_counters)
+            line["ownership"] = dict(superstep_counters, exchange=args.exchange)
         if sweep:
             line["partition_sweep"] = sweep
         print(json.dumps(line), flush=True)

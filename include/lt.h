@@ -313,6 +313,36 @@ lt_status lt_exchange_pack(lt_ctx* ctx, void* d_send, uint64_t capacity, uint64_
  * until the next synchronising call, e.g. lt_run) into the owned buckets. Asynchronous. */
 lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count);
 
+/* ---- Peer exchange: the same superstep without the pack kernel and the all-to-all. Each rank
+ * allocates two receive buffers (superstep parity 0 / 1) of `capacity` 16-B records and two u64
+ * cursors with lt_exchange_buffers, the ranks share their buffers (device pointers valid in this
+ * process: CUDA IPC through lt_ipc_handle / lt_ipc_open across processes, the pointers themselves
+ * within one), and lt_exchange_attach installs the table. From then on the update kernels append a
+ * walk whose next partition rank q owns straight into rank q's receive buffer of the current parity
+ * (peer stores over NVLink, one atomic per (warp, rank) on q's cursor), overlapping the transfer with
+ * the walk steps. Superstep (dist.run_supersteps_p2p): lt_run -> lt_exchange_sent -> a sum over
+ * ranks of the records sent (the barrier after which every buffer of this parity is complete; 0 ends
+ * the loop) -> lt_exchange_take (insert what arrived, reset that cursor, flip the parity).
+ * Every rank must take in every superstep so that the parities stay aligned. */
+/* This rank's buffers: recv[e] (capacity records) and cursor[e] for e = 0, 1; cursor[1] is
+ * cursor[0] + 8 bytes (one allocation). Reallocated only when the capacity changes (not once attached).
+ * Zeroed cursors. LT_ERR_INVALID if world < 2. */
+lt_status lt_exchange_buffers(lt_ctx* ctx, uint64_t capacity, void** recv, void** cursor);
+/* Install the tables recv[e * world + q], cursor[e * world + q] (host arrays of device pointers,
+ * 2 * world each; entry q = rank must be this rank's own buffers). All ranks' capacities must match. */
+lt_status lt_exchange_attach(lt_ctx* ctx, void* const* recv, void* const* cursor);
+/* Records this rank appended to other ranks' buffers in the current superstep (from lt_run's last
+ * count read). LT_ERR_INVALID if a receive buffer overflowed. */
+lt_status lt_exchange_sent(lt_ctx* ctx, uint64_t* sent);
+/* After every rank's lt_run of this superstep has completed (the caller's collective): insert the
+ * records that arrived in this rank's buffer of the current parity into the owned buckets, reset its
+ * cursor and the sent count, flip the parity. *received = the number inserted. Stream-ordered. */
+lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received);
+/* CUDA IPC of a device allocation's base pointer (handle: 64 bytes), and opening another process's
+ * handle on this context's device (closed at lt_destroy). */
+lt_status lt_ipc_handle(const void* dptr, void* handle);
+lt_status lt_ipc_open(lt_ctx* ctx, const void* handle, void** dptr);
+
 /* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:
  * pending + finished == num_walks; free_chunks + ring_chunks == total_chunks. */
 typedef struct lt_pool_state {

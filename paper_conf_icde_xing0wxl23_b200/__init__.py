@@ -5,8 +5,8 @@ is its thin Python binding. Importing it fails loudly when the CUDA extension is
 """
 from .lt import (DEEPWALK, EMPTY, INSERT_DIRECT, INSERT_WARP_AGGREGATED, LAYOUT_ADJ, LAYOUT_ADJ12, LAYOUT_AUTO,  # noqa: F401
                  LAYOUT_CSR, POLICY_PREEMPTIVE_ONLY, POLICY_ROUND_ROBIN, POLICY_SELECTIVE,
-                 POLICY_SELECTIVE_ONLY, PPR, PAGERANK, Engine, LTError, partition_bounds)
+                 POLICY_SELECTIVE_ONLY, PPR, PAGERANK, Engine, LTError, ipc_handle, partition_bounds)
 
-__all__ = ["Engine", "LTError", "partition_bounds", "DEEPWALK", "PPR", "PAGERANK", "EMPTY", "POLICY_SELECTIVE",
+__all__ = ["Engine", "LTError", "partition_bounds", "ipc_handle", "DEEPWALK", "PPR", "PAGERANK", "EMPTY", "POLICY_SELECTIVE",
            "POLICY_ROUND_ROBIN", "INSERT_WARP_AGGREGATED", "INSERT_DIRECT", "LAYOUT_AUTO", "LAYOUT_CSR", "LAYOUT_ADJ", "LAYOUT_ADJ12",
            "POLICY_SELECTIVE_ONLY", "POLICY_PREEMPTIVE_ONLY"]

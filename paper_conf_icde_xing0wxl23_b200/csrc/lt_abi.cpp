@@ -139,6 +139,12 @@ void lt_destroy(lt_ctx* ctx) {
     if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
   }
   if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
+  for (void* q : ctx->ipc_opened) cudaIpcCloseMemHandle(q);
+  cudaFree(ctx->d_xbuf[0]);
+  cudaFree(ctx->d_xbuf[1]);
+  cudaFree(ctx->d_xcur);
+  cudaFree(ctx->d_peer_recv);
+  cudaFree(ctx->d_peer_cur);
   cudaFree(ctx->d_starts);
   cudaFree(ctx->d_starts_all);
   cudaFree(ctx->d_visits);
@@ -612,6 +618,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0);
   p.direct = direct ? lt::Direct{d_starts, W} : lt::Direct{nullptr, 0};
+  p.peer = ctx->peer_on ? lt::Peer{ctx->d_peer_recv, ctx->d_peer_cur, ctx->xcap, ctx->peer_epoch} : lt::Peer{};
   ctx->stats.direct_start = direct ? 1 : 0;
 
   ctx->W = W;
@@ -709,6 +716,8 @@ lt_status lt_run(lt_ctx* ctx) {
   ctx->ran = true;
   ctx->visits_ready = ctx->cfg.visit_counts != 0;
   if (ctx->h_ctr->err & lt::kErrOOM) return fail(LT_ERR_CUDA, "walk pool exhausted on the device (invariant violated)");
+  if (ctx->h_ctr->err & lt::kErrPeer)
+    return fail(LT_ERR_INVALID, "a peer receive buffer overflowed; raise the lt_exchange_buffers capacity");
   if (ctx->h_ctr->err) return fail(LT_ERR_CUDA, "device invariant violated (ring slot reinstalled)");
   return LT_OK;
 }
@@ -917,6 +926,105 @@ lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count) {
   CK(lt::launch_insert_records(ctx->params, (const uint4*)d_recv, count, ctx->stream));
   if (count) ctx->stats.kernel_launches++;
   return LT_OK;  // stream-ordered: the next lt_run's first count read synchronises
+}
+
+// ---- peer exchange (walks appended straight into the owner's receive buffer over peer memory)
+lt_status lt_exchange_buffers(lt_ctx* ctx, uint64_t capacity, void** recv, void** cursor) {
+  if (!ctx || !recv || !cursor) return fail(LT_ERR_INVALID, "NULL argument");
+  if (ctx->world < 2) return fail(LT_ERR_INVALID, "lt_exchange_buffers needs world > 1");
+  if (!capacity) return fail(LT_ERR_INVALID, "capacity must be > 0");
+  CK(cudaSetDevice(ctx->cfg.device));
+  if (ctx->xcap != capacity) {
+    if (ctx->peer_on) return fail(LT_ERR_STATE, "peer buffers are attached; their capacity is fixed");
+    for (int e = 0; e < 2; ++e) {
+      cudaFree(ctx->d_xbuf[e]);
+      ctx->d_xbuf[e] = nullptr;
+      CK(cudaMalloc(&ctx->d_xbuf[e], capacity * sizeof(uint4)));
+    }
+    if (!ctx->d_xcur) CK(cudaMalloc(&ctx->d_xcur, 2 * sizeof(unsigned long long)));
+    CK(cudaMemset(ctx->d_xcur, 0, 2 * sizeof(unsigned long long)));
+    ctx->xcap = capacity;
+  }
+  for (int e = 0; e < 2; ++e) {
+    recv[e] = ctx->d_xbuf[e];
+    cursor[e] = ctx->d_xcur + e;
+  }
+  return LT_OK;
+}
+
+lt_status lt_exchange_attach(lt_ctx* ctx, void* const* recv, void* const* cursor) {
+  if (!ctx || !recv || !cursor) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->xcap) return fail(LT_ERR_STATE, "lt_exchange_attach before lt_exchange_buffers");
+  const uint32_t R = ctx->world;
+  for (uint32_t i = 0; i < 2 * R; ++i)
+    if (!recv[i] || !cursor[i]) return fail(LT_ERR_INVALID, "NULL peer buffer or cursor");
+  if (recv[ctx->rank] != ctx->d_xbuf[0] || recv[R + ctx->rank] != ctx->d_xbuf[1])
+    return fail(LT_ERR_INVALID, "the table's entry for this rank must be this rank's own buffers");
+  CK(cudaSetDevice(ctx->cfg.device));
+  if (!ctx->d_peer_recv) CK(cudaMalloc(&ctx->d_peer_recv, 2 * R * sizeof(uint4*)));
+  if (!ctx->d_peer_cur) CK(cudaMalloc(&ctx->d_peer_cur, 2 * R * sizeof(unsigned long long*)));
+  CK(cudaMemcpy(ctx->d_peer_recv, recv, 2 * R * sizeof(void*), cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(ctx->d_peer_cur, cursor, 2 * R * sizeof(void*), cudaMemcpyHostToDevice));
+  ctx->peer_on = true;
+  ctx->params.peer = lt::Peer{ctx->d_peer_recv, ctx->d_peer_cur, ctx->xcap, ctx->peer_epoch};
+  return LT_OK;
+}
+
+lt_status lt_exchange_sent(lt_ctx* ctx, uint64_t* sent) {
+  if (!ctx || !sent) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  CK(cudaSetDevice(ctx->cfg.device));
+  lt_status st = lt::snapshot_cached(ctx);
+  if (st != LT_OK) return st;
+  if (ctx->h_ctr->err & lt::kErrPeer) return fail(LT_ERR_INVALID, "a peer receive buffer overflowed; raise its capacity");
+  *sent = ctx->h_ctr->sent;
+  return LT_OK;
+}
+
+lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received) {
+  if (!ctx || !received) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->peer_on) return fail(LT_ERR_STATE, "lt_exchange_take before lt_exchange_attach");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  CK(cudaSetDevice(ctx->cfg.device));
+  const uint32_t e = ctx->peer_epoch;
+  unsigned long long cnt = 0;
+  CK(cudaMemcpyAsync(&cnt, ctx->d_xcur + e, sizeof(cnt), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaStreamSynchronize(ctx->stream));
+  if (cnt > ctx->xcap) return fail(LT_ERR_INVALID, "a peer receive buffer overflowed; raise its capacity");
+  if (cnt) {
+    ctx->snap_valid = false;
+    CK(lt::launch_insert_records(ctx->params, ctx->d_xbuf[e], cnt, ctx->stream));
+    ctx->stats.kernel_launches++;
+  }
+  // stream-ordered after the insert: the buffer of epoch e is written again only in superstep s + 2,
+  // whose senders start after this rank's next lt_run (hence this reset) has completed
+  CK(cudaMemsetAsync(ctx->d_xcur + e, 0, sizeof(unsigned long long), ctx->stream));
+  CK(cudaMemsetAsync(&ctx->d_ctr->sent, 0, sizeof(unsigned long long), ctx->stream));
+  ctx->snap_valid = false;
+  ctx->peer_epoch ^= 1u;
+  ctx->params.peer.epoch = ctx->peer_epoch;
+  *received = cnt;
+  return LT_OK;
+}
+
+lt_status lt_ipc_handle(const void* dptr, void* handle) {
+  if (!dptr || !handle) return fail(LT_ERR_INVALID, "NULL argument");
+  cudaIpcMemHandle_t h;
+  CK(cudaIpcGetMemHandle(&h, const_cast<void*>(dptr)));
+  std::memcpy(handle, &h, sizeof(h));
+  return LT_OK;
+}
+
+lt_status lt_ipc_open(lt_ctx* ctx, const void* handle, void** dptr) {
+  if (!ctx || !handle || !dptr) return fail(LT_ERR_INVALID, "NULL argument");
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  void* q = nullptr;
+  CK(cudaIpcOpenMemHandle(&q, h, cudaIpcMemLazyEnablePeerAccess));
+  ctx->ipc_opened.push_back(q);
+  *dptr = q;
+  return LT_OK;
 }
 
 // lt_run_to_host / lt_run_to_host_compact: dense rows (paths != NULL) or the ragged layout

@@ -137,6 +137,16 @@ struct lt_ctx {
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t ev_computed[2] = {nullptr, nullptr}, ev_copied[2] = {nullptr, nullptr};
   cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+  // peer exchange (lt_exchange_buffers / lt_exchange_attach): this rank's two receive buffers and
+  // cursors (epoch 0 / 1), and the device tables of every rank's buffers and cursors
+  uint4* d_xbuf[2] = {nullptr, nullptr};
+  unsigned long long* d_xcur = nullptr;  // [2]
+  uint64_t xcap = 0;
+  uint4** d_peer_recv = nullptr;                // [2 * world]
+  unsigned long long** d_peer_cur = nullptr;    // [2 * world]
+  bool peer_on = false;
+  uint32_t peer_epoch = 0;
+  std::vector<void*> ipc_opened;                // peer buffers opened through CUDA IPC (closed at destroy)
 };
 
 #define CK(call)                                                                        \

@@ -9,6 +9,7 @@ namespace lt {
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;   // empty ring slot / unused path slot
 constexpr uint32_t kErrOOM = 1u;           // device error bits
 constexpr uint32_t kErrRing = 2u;
+constexpr uint32_t kErrPeer = 4u;          // a peer receive buffer overflowed
 
 // A walk record (D5): 16 bytes, one 128-bit load/store.
 //   x = local walk index (row of the path matrix; walk_id = first_walk_id + x)
@@ -62,6 +63,7 @@ struct Counters {
   unsigned long long steps, visits, truncated;
   uint32_t err;
   uint32_t done_ctas;
+  unsigned long long sent;  // records appended to other ranks' receive buffers (peer exchange)
 };
 
 // Range ownership across ranks (north star 8-GPU mode): this rank owns partitions
@@ -91,8 +93,22 @@ struct Direct {
   unsigned long long count;
 };
 
+// Peer exchange (lt_exchange_attach; the multi-GPU mode without pack + all-to-all): a walk whose
+// next partition is owned by rank q is appended by the insertion epilogue straight into rank q's
+// receive buffer over peer memory (NVLink), with one atomic per (warp, destination rank) on q's
+// cursor. Receive buffers and cursors are double-buffered by superstep parity `epoch`, so senders of
+// superstep s+1 never touch the buffer a receiver is still draining from superstep s.
+// recv == nullptr: off (walks for other ranks go to the local send buckets).
+struct Peer {
+  uint4* const* recv;                    // [2 * world]: buffer of rank q for epoch e at [e * world + q]
+  unsigned long long* const* cursor;     // [2 * world]: same indexing, one u64 each
+  unsigned long long cap;                // records per buffer
+  uint32_t epoch;
+};
+
 struct Params {
   Walk wk;
+  Peer peer;
   Cont cont;
   Pool pool;
   Counters* ctr;

@@ -124,6 +124,19 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
   const uint32_t grp = __match_any_sync(act, dest);
   const uint32_t leader = __ffs(grp) - 1;
   const uint32_t rank = __popc(grp & lanemask_lt());
+  if (p.peer.recv && dest >= p.wk.P) {  // a walk for rank q: straight into q's receive buffer (peer memory)
+    const uint32_t slot = p.peer.epoch * (pl.nbuckets - p.wk.P) + (dest - p.wk.P);
+    unsigned long long base = 0;
+    if (lane == leader) {
+      const uint32_t cnt = __popc(grp);
+      base = atomicAdd(p.peer.cursor[slot], (unsigned long long)cnt);
+      if (base + cnt > p.peer.cap) atomicOr(&p.ctr->err, kErrPeer);
+      atomicAdd(&p.ctr->sent, (unsigned long long)cnt);
+    }
+    base = __shfl_sync(grp, base, leader);
+    if (base + rank < p.peer.cap) p.peer.recv[slot][base + rank] = rec;
+    return;
+  }
   unsigned long long base = 0;
   uint32_t c0 = 0, c1 = 0;
   if (lane == leader) {
@@ -134,9 +147,11 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
     c0 = (base & cmask) == 0 ? install_chunk(p, dest, ci0) : wait_chunk(p, dest, ci0);
     if (ci1 == ci0) c1 = c0;
   }
-  base = __shfl_sync(act, base, leader);
-  c0 = __shfl_sync(act, c0, leader);
-  c1 = __shfl_sync(act, c1, leader);
+  // each lane needs only its group leader's values (lanes of groups that went to a peer buffer above
+  // have returned, so the mask is the group, not every active lane)
+  base = __shfl_sync(grp, base, leader);
+  c0 = __shfl_sync(grp, c0, leader);
+  c1 = __shfl_sync(grp, c1, leader);
   const unsigned long long pos = base + rank;
   const uint32_t c = ((pos >> pl.c_shift) == (base >> pl.c_shift)) ? c0 : c1;
   pl.slots[((uint64_t)c << pl.c_shift) | (pos & cmask)] = rec;
@@ -154,7 +169,8 @@ __device__ void last_cta_retire(const Params& p, int k, unsigned long long head,
   __shared__ bool s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence();
+    if (p.peer.recv) __threadfence_system();  // peer-memory appends performed before the grid ends
+    else __threadfence();
     const uint32_t ticket = atomicAdd(&p.ctr->done_ctas, 1u);
     s_last = (ticket == gridDim.x - 1);
   }
@@ -922,6 +938,7 @@ __global__ void k_snapshot(const unsigned long long* __restrict__ hc, uint64_t n
     out_ctr->truncated = ctr->truncated;
     out_ctr->err = ctr->err;
     out_ctr->done_ctas = ctr->done_ctas;
+    out_ctr->sent = ctr->sent;
     *out_free = *free_top;
   }
 }
@@ -1051,6 +1068,7 @@ __global__ void k_pool_reset(Params p) {
   if (tid == 0) {
     *pl.free_top = (int)pl.num_chunks;
     p.ctr->steps = 0; p.ctr->visits = 0; p.ctr->truncated = 0; p.ctr->err = 0; p.ctr->done_ctas = 0;
+    p.ctr->sent = 0;
   }
 }
 

@@ -73,6 +73,13 @@ class TorchComm:
         ops = {"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM}
         self.dist.all_reduce(t, op=ops[op], group=self.group)
 
+    def allgather_obj(self, obj):
+        out = [None] * self.world
+        self.dist.all_gather_object(out, obj, group=self.group)
+        return out
+
+    same_process = False
+
 
 class ThreadComm:
     """In-process collectives between `world` threads (each driving one Engine), used to exercise
@@ -128,6 +135,11 @@ class ThreadComm:
     def allreduce_sum(self, x: int, device) -> int:
         return sum(self._gather(int(x)))
 
+    def allgather_obj(self, obj):
+        return self._gather(obj)
+
+    same_process = True
+
     def allreduce_(self, t, op: str):
         allv = self._gather(t.clone())
         acc = allv[0].to(t.device)
@@ -166,6 +178,50 @@ def run_supersteps(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
         recv_counts = [mat[r][comm.rank] for r in range(comm.world)]
         recv = comm.alltoallv(buf, counts, recv_counts)
         engine.exchange_insert(recv, sum(recv_counts))
+        if supersteps >= max_supersteps:
+            raise RuntimeError("ownership supersteps did not converge")
+
+
+def attach_peers(engine, comm, capacity: int):
+    """Peer exchange setup (lt_exchange_buffers / lt_exchange_attach): every rank allocates its two
+    receive buffers of `capacity` records, the ranks share them — raw device addresses between
+    threads of one process, CUDA IPC handles between processes (lt_ipc_handle / lt_ipc_open) — and
+    each rank installs the table of every rank's buffers."""
+    recv, cur = engine.exchange_buffers(capacity)
+    R, me = comm.world, comm.rank
+    if comm.same_process:
+        allv = comm.allgather_obj((recv, cur))
+    else:
+        from .lt import ipc_handle
+        mine = (ipc_handle(recv[0]), ipc_handle(recv[1]), ipc_handle(cur[0]))
+        hs = comm.allgather_obj(mine)
+        allv = []
+        for q in range(R):
+            if q == me:
+                allv.append((recv, cur))
+                continue
+            r0, r1, c0 = (engine.ipc_open(h) for h in hs[q])
+            allv.append(([r0, r1], [c0, c0 + 8]))  # cursor[1] = cursor[0] + 8 bytes (one allocation)
+    table_r = [allv[q][0][e] for e in range(2) for q in range(R)]
+    table_c = [allv[q][1][e] for e in range(2) for q in range(R)]
+    engine.exchange_attach(table_r, table_c)
+
+
+def run_supersteps_p2p(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
+    """Superstep loop of the peer exchange: the update kernels already appended every walk that
+    crossed ranks into its owner's receive buffer (peer memory, overlapped with the steps), so a
+    superstep is lt_run, ONE small collective (the sum of records sent, which is also the barrier
+    after which every receive buffer of this parity is complete) and lt_exchange_take."""
+    supersteps, moved = 0, 0
+    while True:
+        engine.run()
+        sent = engine.exchange_sent()
+        total = comm.allreduce_sum(sent, device)
+        supersteps += 1
+        moved += sent
+        if total == 0:
+            return {"supersteps": supersteps, "records_sent": moved}
+        engine.exchange_take()
         if supersteps >= max_supersteps:
             raise RuntimeError("ownership supersteps did not converge")
 

@@ -34,6 +34,8 @@ EXPORTED = [
     "lt_get_paths", "lt_get_paths_rows", "lt_get_paths_device", "lt_get_stats", "lt_get_pool_state",
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
     "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
+    "lt_exchange_buffers", "lt_exchange_attach", "lt_exchange_sent", "lt_exchange_take", "lt_ipc_handle",
+    "lt_ipc_open",
 ]
 
 
@@ -112,9 +114,22 @@ _lib.lt_get_pool_state.argtypes = [_vp, ctypes.POINTER(PoolState)]
 _lib.lt_pending.argtypes = [_vp, ctypes.POINTER(_u64), _vp]
 _lib.lt_exchange_pack.argtypes = [_vp, _vp, _u64, _vp]
 _lib.lt_exchange_insert.argtypes = [_vp, _vp, _u64]
+_lib.lt_exchange_buffers.argtypes = [_vp, _u64, _vp, _vp]
+_lib.lt_exchange_attach.argtypes = [_vp, _vp, _vp]
+_lib.lt_exchange_sent.argtypes = [_vp, ctypes.POINTER(_u64)]
+_lib.lt_exchange_take.argtypes = [_vp, ctypes.POINTER(_u64)]
+_lib.lt_ipc_handle.argtypes = [_vp, _vp]
+_lib.lt_ipc_open.argtypes = [_vp, _vp, ctypes.POINTER(_vp)]
 _lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
 _lib.lt_run_to_host_compact.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u64, _u32]
 _lib.lt_get_paths_compact.argtypes = [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]
+
+
+def ipc_handle(dptr: int) -> bytes:
+    """CUDA IPC handle (64 bytes) of the device allocation at dptr (an allocation base)."""
+    buf = ctypes.create_string_buffer(64)
+    _check(_lib.lt_ipc_handle(_vp(dptr), buf))
+    return buf.raw
 
 
 class LTError(RuntimeError):
@@ -388,6 +403,37 @@ class Engine:
             raise ValueError("exchange_insert needs a CUDA tensor")
         _check(_lib.lt_exchange_insert(self._h, pp, count))
         self._recv_keep = d_recv  # read asynchronously by the insert kernel (stream-ordered)
+
+    # ---- peer exchange (lt_exchange_buffers / attach / sent / take; dist.run_supersteps_p2p)
+    def exchange_buffers(self, capacity: int):
+        """This rank's receive buffers and cursors (device addresses) for parity 0 and 1."""
+        recv = (_vp * 2)()
+        cur = (_vp * 2)()
+        _check(_lib.lt_exchange_buffers(self._h, int(capacity), recv, cur))
+        return [int(x) for x in recv], [int(x) for x in cur]
+
+    def exchange_attach(self, recv, cursor):
+        """recv / cursor: 2 * world device addresses, [e * world + q] = rank q's buffer of parity e."""
+        r = (_vp * len(recv))(*recv)
+        c = (_vp * len(cursor))(*cursor)
+        _check(_lib.lt_exchange_attach(self._h, r, c))
+
+    def exchange_sent(self) -> int:
+        x = _u64()
+        _check(_lib.lt_exchange_sent(self._h, ctypes.byref(x)))
+        return int(x.value)
+
+    def exchange_take(self) -> int:
+        x = _u64()
+        _check(_lib.lt_exchange_take(self._h, ctypes.byref(x)))
+        return int(x.value)
+
+    def ipc_open(self, handle: bytes) -> int:
+        """Open another process's CUDA IPC handle (64 bytes) on this engine's device."""
+        buf = ctypes.create_string_buffer(bytes(handle), 64)
+        out = _vp()
+        _check(_lib.lt_ipc_open(self._h, buf, ctypes.byref(out)))
+        return int(out.value)
 
     def partial_paths(self):
         """This rank's share of paths (CUDA int32 tensors [W, stride], [W]) for the cross-rank merge."""

@@ -113,3 +113,161 @@ def test_ownership_out_of_core_ranks(gpu, g13, cont):
     for paths, lengths, _, st in res:
         np.testing.assert_array_equal(paths, op)
         assert st["out_of_core"] == 1
+
+
+# ---- peer exchange (lt_exchange_buffers / attach / sent / take): walks for another rank are
+# appended by the update kernels straight into that rank's receive buffer (peer memory)
+
+def run_owned_p2p(g, starts, app, param, seed, P, world, capacity=None, **cfg):
+    import torch
+    hub = ltdist.ThreadComm.Hub(world)
+    results, errors = [None] * world, []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world, **cfg) as e:
+                e.graph_load(g.row_ptr, g.col, P)
+                if app == LT.PAGERANK:
+                    e.walks_init_pagerank(starts, int(param[0]), param[1], seed)
+                else:
+                    e.walks_init(starts, app, param, seed)
+                comm = ltdist.ThreadComm(hub, r)
+                ltdist.attach_peers(e, comm, capacity or len(starts))
+                counters = ltdist.run_supersteps_p2p(e, comm, "cuda")
+                paths, lengths = ltdist.merge_paths(e, comm)
+                torch.cuda.synchronize()
+                results[r] = (paths.cpu().numpy().view(np.uint32), lengths.cpu().numpy().view(np.uint32),
+                              counters, e.stats())
+        except Exception as ex:  # surface thread failures
+            errors.append(ex)
+            hub.barrier.abort()
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errors:
+        raise errors[0]
+    return results
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 16), (LT.PPR, 0.15)])
+def test_peer_exchange_exact(gpu, g13, world, layout, app, param):
+    starts = (lt_inputs.deepwalk_starts(3 * g13.n, g13.n) if app == LT.DEEPWALK
+              else lt_inputs.ppr_starts(20_000, g13.argmax_deg))
+    res = run_owned_p2p(g13, starts, app, param, 2, 12, world, layout=layout, chunk_walks=512)
+    op, ol, osteps, _ = oracle_of(g13, starts, app, param, 2)
+    for paths, lengths, counters, st in res:
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+    assert sum(r[3]["steps"] for r in res) == osteps
+    assert res[0][2]["supersteps"] == res[-1][2]["supersteps"]
+    assert sum(r[2]["records_sent"] for r in res) > 0
+
+
+def test_peer_exchange_out_of_core_and_repeat(gpu, g13):
+    """Peer exchange with every rank out of core (continuation on), then a second epoch on the same
+    engines: the superstep parities stay aligned across epochs."""
+    import torch
+    world = 2
+    hub = ltdist.ThreadComm.Hub(world)
+    starts = lt_inputs.deepwalk_starts(g13.n, g13.n)
+    out, errors = [None] * world, []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world, graph_pool_bytes=8 << 20, zero_copy=True,
+                           continue_resident=True) as e:
+                e.graph_load(g13.row_ptr, g13.col, 8)
+                comm = ltdist.ThreadComm(hub, r)
+                res = []
+                for seed in (4, 5):
+                    e.walks_init(starts, LT.DEEPWALK, 10, seed)
+                    if seed == 4:
+                        ltdist.attach_peers(e, comm, len(starts))
+                    ltdist.run_supersteps_p2p(e, comm, "cuda")
+                    paths, lengths = ltdist.merge_paths(e, comm)
+                    torch.cuda.synchronize()
+                    res.append(paths.cpu().numpy().view(np.uint32))
+                out[r] = res
+        except Exception as ex:
+            errors.append(ex)
+            hub.barrier.abort()
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errors:
+        raise errors[0]
+    for i, seed in enumerate((4, 5)):
+        op, _, _, _ = oracle_of(g13, starts, LT.DEEPWALK, 10, seed)
+        for r in range(world):
+            np.testing.assert_array_equal(out[r][i], op)
+
+
+def test_peer_exchange_overflow_is_an_error(gpu, g13):
+    starts = lt_inputs.deepwalk_starts(g13.n, g13.n)
+    with pytest.raises(LT.LTError, match="overflow"):
+        run_owned_p2p(g13, starts, LT.DEEPWALK, 10, 1, 12, 2, capacity=16)
+
+
+def _p2p_proc(rank, world, port, out_q):
+    import os
+
+    import torch
+    import torch.distributed as tdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        g = lt_inputs.rmat_cpu(13, 8 * 2 ** 13, seed=3)
+        starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+        with LT.Engine(rank=rank, world=world) as e:
+            e.graph_load(g.row_ptr, g.col, 2 * world)
+            e.walks_init(starts, LT.DEEPWALK, 12, 7)
+            comm = ltdist.TorchComm()
+            ltdist.attach_peers(e, comm, len(starts))  # CUDA IPC between the processes
+            counters = ltdist.run_supersteps_p2p(e, comm, "cpu")
+            paths, lengths = e.partial_paths()
+            paths, lengths = paths.cpu(), lengths.cpu()
+            paths ^= ltdist.SIGN
+            comm.allreduce_(paths, "min")
+            paths ^= ltdist.SIGN
+            comm.allreduce_(lengths, "max")
+            if rank == 0:
+                out_q.put((paths.numpy().view(np.uint32).copy(), lengths.numpy().view(np.uint32).copy(), counters))
+    finally:
+        tdist.destroy_process_group()
+
+
+def test_peer_exchange_processes_cuda_ipc(gpu):
+    """Two processes on one GPU, each rank's receive buffers opened by the other through CUDA IPC
+    (lt_ipc_handle / lt_ipc_open): the multi-process wiring of the peer exchange."""
+    import socket
+
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_p2p_proc, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    paths, lengths, counters = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    g = lt_inputs.rmat_cpu(13, 8 * 2 ** 13, seed=3)
+    starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+    op, ol, _, _ = oracle_of(g, starts, LT.DEEPWALK, 12, 7)
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)
+    assert counters["records_sent"] > 0
