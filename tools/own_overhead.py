@@ -2,6 +2,7 @@
 """Range-ownership superstep overhead on ONE GPU: `world` engines in threads (dist.ThreadComm), all on
 cuda:0, DeepWalk l=80 over |V| walks of a BASELINE config's graph. Prints one JSON line: wall time of
 the superstep loop, supersteps, and the host-side share (wall minus the summed update-kernel time).
+--p2p runs the peer exchange (walks appended into the owner's receive buffer by the update kernels).
 --legacy runs the superstep loop of the first version (all-to-all of counts, then an all-reduce for
 termination); pair it with LT_LIBRARY pointing at a build of that version (synchronising pack /
 insert / pending). Not a multi-GPU number: the ranks share one device."""
@@ -41,6 +42,7 @@ def main():
     ap.add_argument("--world", type=int, default=2)
     ap.add_argument("--partitions", type=int, default=0, help="0: one per rank")
     ap.add_argument("--legacy", action="store_true")
+    ap.add_argument("--p2p", action="store_true", help="peer exchange (dist.run_supersteps_p2p)")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--refill", type=int, default=0, help="lt_config.refill: 0 auto, 1 off, 2 on")
     a = ap.parse_args()
@@ -58,6 +60,9 @@ def main():
         with LT.Engine(rank=r, world=a.world, timing=True, refill=a.refill) as e:
             e.graph_load(g.row_ptr, g.col, P)
             comm = ltdist.ThreadComm(hub, r)
+            if a.p2p:
+                e.walks_init(starts, LT.DEEPWALK, 80, 1)
+                ltdist.attach_peers(e, comm, g.n)
             for rep in range(a.reps + 1):
                 e.walks_init(starts, LT.DEEPWALK, 80, 1)
                 hub.barrier.wait()
@@ -66,6 +71,8 @@ def main():
                 upd = 0.0
                 if a.legacy:
                     cnt = legacy_supersteps(e, comm, "cuda")
+                elif a.p2p:
+                    cnt = ltdist.run_supersteps_p2p(e, comm, "cuda")
                 else:
                     cnt = ltdist.run_supersteps(e, comm, "cuda")
                 torch.cuda.synchronize()
@@ -82,7 +89,7 @@ def main():
         t.join()
     wall = min(max(res[r][i][0] for r in range(a.world)) for i in range(a.reps))
     ss = res[0][-1][1]
-    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "refill": a.refill,
+    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "p2p": a.p2p, "refill": a.refill,
            "wall_ms": wall * 1e3,
            "supersteps": ss, "ms_per_superstep": wall * 1e3 / ss, "n": g.n,
            "library": os.environ.get("LT_LIBRARY", "liblt.so")}
