@@ -158,7 +158,8 @@ def test_pagerank_out_of_core(gpu, blocks, zero_copy):
 
 
 @pytest.mark.parametrize("world", [2, 3])
-def test_pagerank_ownership_and_merged_visit_counts(gpu, world):
+@pytest.mark.parametrize("p2p", [False, True])
+def test_pagerank_ownership_and_merged_visit_counts(gpu, world, p2p):
     """Range ownership with restarts: a restart may send a walk to any rank. Merged
     paths equal the oracle; visit counts summed over ranks equal the oracle's."""
     import torch
@@ -173,7 +174,11 @@ def test_pagerank_ownership_and_merged_visit_counts(gpu, world):
                 e.graph_load(g.row_ptr, g.col, 12)
                 e.walks_init_pagerank(starts, 12, 0.2, 6)
                 comm = ltdist.ThreadComm(hub, r)
-                ltdist.run_supersteps(e, comm, "cuda")
+                if p2p:  # peer exchange: restarts send walks to any rank's receive buffer
+                    ltdist.attach_peers(e, comm, len(starts))
+                    ltdist.run_supersteps_p2p(e, comm, "cuda")
+                else:
+                    ltdist.run_supersteps(e, comm, "cuda")
                 paths, lengths = ltdist.merge_paths(e, comm)
                 counts = ltdist.merge_visit_counts(e, comm, "cuda")
                 torch.cuda.synchronize()

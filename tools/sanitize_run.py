@@ -4,7 +4,7 @@ initcheck): resident P=1 (refill), P=4 (batch kernel, CSR and ADJ), PPR, out-of-
 two-rank ownership, streamed run_to_host (dense and ragged), ragged copy-out, PageRank with u32 / u64
 visit counters, out-of-core continuation, walk admission, paths off, the direct start (P = 1, both
 path modes, device starts), the compact ADJ12 layout, slice-only ownership (CSR / ADJ / ADJ12, host and
-borrowed device graphs)."""
+borrowed device graphs), the peer exchange (CSR / ADJ)."""
 import os
 import sys
 import threading
@@ -88,6 +88,24 @@ for layout, device_graph in [(LT.LAYOUT_AUTO, False), (LT.LAYOUT_CSR, False), (L
             ltdist.merge_paths(e, comm)
 
     th = [threading.Thread(target=rank, args=(r,)) for r in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+# peer exchange (walks appended into the owner's receive buffer by the update kernels), CSR and ADJ
+for layout in (LT.LAYOUT_CSR, LT.LAYOUT_ADJ):
+    hub = ltdist.ThreadComm.Hub(2)
+
+    def rank_p2p(r):
+        with LT.Engine(rank=r, world=2, chunk_walks=256, layout=layout) as e:
+            e.graph_load(g.row_ptr, g.col, 4)
+            e.walks_init(starts, LT.DEEPWALK, 10, 1)
+            comm = ltdist.ThreadComm(hub, r)
+            ltdist.attach_peers(e, comm, len(starts))
+            ltdist.run_supersteps_p2p(e, comm, "cuda")
+            ltdist.merge_paths(e, comm)
+
+    th = [threading.Thread(target=rank_p2p, args=(r,)) for r in range(2)]
     for t in th:
         t.start()
     for t in th:
