@@ -191,17 +191,9 @@ def attach_peers(engine, comm, capacity: int):
     R, me = comm.world, comm.rank
     if comm.same_process:
         allv = comm.allgather_obj((recv, cur))
-    else:
-        from .lt import ipc_handle
-        mine = (ipc_handle(recv[0]), ipc_handle(recv[1]), ipc_handle(cur[0]))
-        hs = comm.allgather_obj(mine)
-        allv = []
-        for q in range(R):
-            if q == me:
-                allv.append((recv, cur))
-                continue
-            r0, r1, c0 = (engine.ipc_open(h) for h in hs[q])
-            allv.append(([r0, r1], [c0, c0 + 8]))  # cursor[1] = cursor[0] + 8 bytes (one allocation)
+    else:  # CUDA IPC handles (Engine.export_buffers / import_buffers)
+        hs = comm.allgather_obj(engine.export_buffers())
+        allv = [(recv, cur) if q == me else engine.import_buffers(hs[q]) for q in range(R)]
     table_r = [allv[q][0][e] for e in range(2) for q in range(R)]
     table_c = [allv[q][1][e] for e in range(2) for q in range(R)]
     engine.exchange_attach(table_r, table_c)

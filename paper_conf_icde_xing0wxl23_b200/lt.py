@@ -410,6 +410,7 @@ class Engine:
         recv = (_vp * 2)()
         cur = (_vp * 2)()
         _check(_lib.lt_exchange_buffers(self._h, int(capacity), recv, cur))
+        self._xcap = int(capacity)
         return [int(x) for x in recv], [int(x) for x in cur]
 
     def exchange_attach(self, recv, cursor):
@@ -427,6 +428,16 @@ class Engine:
         x = _u64()
         _check(_lib.lt_exchange_take(self._h, ctypes.byref(x)))
         return int(x.value)
+
+    def export_buffers(self):
+        """CUDA IPC handles of this rank's receive buffers (parity 0, 1) and of its cursor pair."""
+        recv, cur = self.exchange_buffers(self._xcap)
+        return ipc_handle(recv[0]), ipc_handle(recv[1]), ipc_handle(cur[0])
+
+    def import_buffers(self, handles):
+        """Open another rank's export_buffers() handles: ([recv0, recv1], [cursor0, cursor1])."""
+        r0, r1, c0 = (self.ipc_open(h) for h in handles)
+        return [r0, r1], [c0, c0 + 8]  # cursor[1] = cursor[0] + 8 bytes (one allocation)
 
     def ipc_open(self, handle: bytes) -> int:
         """Open another process's CUDA IPC handle (64 bytes) on this engine's device."""

@@ -5,7 +5,13 @@ exchange_pack, exchange_insert, partial_paths) with per-visit stepping built on 
 primitives (Philox and Lemire from oracle/), so the multi-process protocol (ownership ranges,
 send buckets, count + payload all-to-all, termination, min/max merge) can run on CPU under gloo.
 It is not the product: the product's kernels are exercised by tests/test_gpu_ownership.py.
+
+The peer exchange (dist.attach_peers / run_supersteps_p2p) is emulated with POSIX shared memory:
+rank q's receive buffer of parity e is one segment per sender (no cross-process atomics needed on
+CPU), "device addresses" are (segment name, ...) tuples, export/import pass the names.
 """
+from multiprocessing import shared_memory
+
 import numpy as np
 
 import oracle as O
@@ -23,6 +29,66 @@ class CpuOwnerEngine:
         self.owner = np.zeros(P, dtype=np.int64)
         for r in range(world):
             self.owner[P * r // world: P * (r + 1) // world] = r
+
+    # ---- peer exchange emulation (shared memory): segment layout per rank: [2 parities][world
+    # senders] x (cursor u64 + capacity records of 4 u32)
+    def exchange_buffers(self, capacity):
+        self.xcap = int(capacity)
+        self._seg_bytes = 8 + 16 * self.xcap
+        name = f"ltp2p_{id(self) & 0xFFFFFF:x}_{self.rank}_{np.random.randint(1 << 30)}"
+        self._own_shm = shared_memory.SharedMemory(name=name, create=True, size=2 * self.world * self._seg_bytes)
+        self._own_shm.buf[:] = bytes(len(self._own_shm.buf))
+        self._shms = {}
+        return [(name, 0), (name, 1)], [(name, 0), (name, 1)]
+
+    def export_buffers(self):
+        return self._own_shm.name
+
+    def import_buffers(self, name):
+        return [(name, 0), (name, 1)], [(name, 0), (name, 1)]
+
+    def exchange_attach(self, recv, cursor):
+        self.peers = [recv[q][0] for q in range(self.world)]  # segment name of rank q
+        for nm in self.peers:
+            if nm != self._own_shm.name and nm not in self._shms:
+                self._shms[nm] = shared_memory.SharedMemory(name=nm)
+        self.epoch, self.sent = 0, 0
+
+    def _seg(self, name, epoch, sender):
+        shm = self._own_shm if name == self._own_shm.name else self._shms[name]
+        off = (epoch * self.world + sender) * self._seg_bytes
+        cur = np.ndarray((1,), dtype=np.uint64, buffer=shm.buf, offset=off)
+        recs = np.ndarray((self.xcap, 4), dtype=np.uint32, buffer=shm.buf, offset=off + 8)
+        return cur, recs
+
+    def _send(self, q, rec):
+        cur, recs = self._seg(self.peers[q], self.epoch, self.rank)
+        i = int(cur[0])
+        assert i < self.xcap, "peer receive buffer overflow"
+        recs[i] = (rec[0], rec[1], rec[2], 0)
+        cur[0] = i + 1
+        self.sent += 1
+
+    def exchange_sent(self):
+        return self.sent
+
+    def exchange_take(self):
+        got = 0
+        for sender in range(self.world):
+            cur, recs = self._seg(self._own_shm.name, self.epoch, sender)
+            for w, v, t, _ in recs[: int(cur[0])]:
+                self.buckets[self._bucket(self._part(int(v)))].append((int(w), int(v), int(t)))
+            got += int(cur[0])
+            cur[0] = 0
+        self.sent = 0
+        self.epoch ^= 1
+        return got
+
+    def close_exchange(self):
+        for shm in self._shms.values():
+            shm.close()
+        self._own_shm.close()
+        self._own_shm.unlink()
 
     def _part(self, v):
         return int(np.searchsorted(self.bounds, v, side="right") - 1)
@@ -100,7 +166,11 @@ class CpuOwnerEngine:
                 for rec in recs:
                     out = self._visit(rec, lo, hi)
                     if out is not None:
-                        self.buckets[self._bucket(self._part(out[1]))].append(out)
+                        b = self._bucket(self._part(out[1]))
+                        if b >= self.P and getattr(self, "peers", None):  # peer exchange: into rank q's buffer
+                            self._send(b - self.P, out)
+                        else:
+                            self.buckets[b].append(out)
 
     def pending(self):
         loc = sum(len(self.buckets[k]) for k in range(self.own_lo, self.own_hi))

@@ -77,3 +77,65 @@ def test_ownership_protocol_gloo(world, app, param):
     np.testing.assert_array_equal(paths, op)
     np.testing.assert_array_equal(counts, O.visit_counts(op, ol, g.n))  # summed over ranks
     assert counters["supersteps"] >= 2 and counters["records_sent"] > 0
+
+
+def _worker_p2p(rank, world, port, app, param, P, out_q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import torch.distributed as dist
+
+    from cpu_owner_engine import CpuOwnerEngine
+    from paper_conf_icde_xing0wxl23_b200 import dist as ltdist
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    eng = None
+    try:
+        g = lt_inputs.rmat_cpu(9, 3000, seed=5)
+        W = 700
+        starts = lt_inputs.ppr_starts(W, g.argmax_deg) if app == LT.PPR else lt_inputs.deepwalk_starts(W, g.n)
+        eng = CpuOwnerEngine(g, P, rank, world)
+        comm = ltdist.TorchComm()
+        res = []
+        for seed in (11, 12):  # two epochs: the parities stay aligned
+            eng.walks_init(starts, app, param, seed)
+            if seed == 11:
+                ltdist.attach_peers(eng, comm, W)
+            counters = ltdist.run_supersteps_p2p(eng, comm, "cpu")
+            paths, lengths = ltdist.merge_paths(eng, comm)
+            res.append((paths.numpy().view(np.uint32).copy(), lengths.numpy().view(np.uint32).copy(), counters))
+        dist.barrier()
+        if rank == 0:
+            out_q.put(res)
+    finally:
+        if eng is not None and hasattr(eng, "_own_shm"):
+            dist.barrier()
+            eng.close_exchange()
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 12), (LT.PPR, 0.2)])
+def test_peer_exchange_protocol_gloo(world, app, param):
+    """dist.attach_peers + run_supersteps_p2p over gloo (the CPU stand-in emulates the receive buffers
+    with shared memory): merged paths equal the oracle over two epochs."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_p2p, args=(r, world, port, app, param, 8, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    g = lt_inputs.rmat_cpu(9, 3000, seed=5)
+    W = 700
+    starts = lt_inputs.ppr_starts(W, g.argmax_deg) if app == LT.PPR else lt_inputs.deepwalk_starts(W, g.n)
+    for (paths, lengths, counters), seed in zip(res, (11, 12)):
+        kw = dict(app=O.DEEPWALK, length=param) if app == LT.DEEPWALK else dict(app=O.PPR, alpha=param)
+        op, ol, _, _ = O.walks(g.row_ptr, g.col, starts, seed=seed, **kw)
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+        assert counters["records_sent"] > 0
