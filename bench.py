@@ -88,10 +88,11 @@ def parse():
                          "(PAPER.md:287, SURVEY.md 8(f) f2) of the config's length, with visit counting")
     ap.add_argument("--restart-p", type=float, default=0.15, help="PageRank restart probability")
     ap.add_argument("--visit-counts", type=int, default=-1, help="fused visit counting: -1 auto (on for pagerank)")
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
-                    help="--mode own: walks crossing ranks go through lt_exchange_pack + an NCCL all-to-all "
-                         "(nccl), or are appended by the update kernels straight into the owner's receive "
-                         "buffer over peer memory (p2p: CUDA IPC, one small all-reduce per superstep)")
+    ap.add_argument("--exchange", default="p2p", choices=["nccl", "p2p"],
+                    help="--mode own: walks crossing ranks are appended by the update kernels straight into "
+                         "the owner's receive buffer over peer memory (p2p, default: CUDA IPC, one small "
+                         "all-reduce per superstep), or go through lt_exchange_pack + an NCCL all-to-all "
+                         "(nccl, the baseline)")
     ap.add_argument("--mode", default="replicas", choices=["replicas", "own"],
                     help="N>1: replicas (each rank its own |V| walks, no collective, weak scaling) or own "
                          "(range ownership: |V| walks in total, NCCL all-to-all of crossing walks per "

@@ -15,6 +15,6 @@ python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.
   > gpurun_out/multirank_own_p2p_n2.json 2> gpurun_out/multirank_own_p2p_n2.err
 echo "own p2p n=2 rc=$?"
 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29514 \
-  bench.py --gpus 2 --steps 3 --warmup 3 --config 2 --no-cpu-baseline --no-e2e --mode own \
+  bench.py --gpus 2 --steps 3 --warmup 3 --config 2 --no-cpu-baseline --no-e2e --mode own --exchange nccl \
   > gpurun_out/multirank_own_nccl_n2.json 2> gpurun_out/multirank_own_nccl_n2.err
 echo "own all-to-all n=2 rc=$?"
