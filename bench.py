@@ -238,6 +238,18 @@ def cores():
         return os.cpu_count()
 
 
+def cpu_model():
+    """The host CPU's model name (the oracle baseline states its cores and CPU)."""
+    try:
+        with open("/proc/cpuinfo") as fh:
+            for line in fh:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cfg_json(c, g, W, extra):
     d = {"workload": f"{c['name']} (BASELINE.json configs[{c['idx'] - 1}])", "scale": c["scale"],
          "rmat_tuples": c["tuples"], "kronecker": bool(c["permute"]), "vertices": g.n, "csr_entries": g.m,
@@ -282,7 +294,7 @@ def run_reference(args):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * secs / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
             "data": "synthetic", "config": cfg_json(c, g, W, {"partitions": None}),
-            "cpu_baseline": {"value": value, "unit": "steps/s", "cores": cores(), "kind": "oracle",
+            "cpu_baseline": {"value": value, "unit": "steps/s", "cores": cores(), "cpu_model": cpu_model(), "kind": "oracle",
                              "sample": f"walks 0..{ns - 1} of the workload per step (oracle/ C + OpenMP, {cores()} threads)"},
             "e2e": {"value": value, "unit": "steps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -602,7 +614,7 @@ def main():
         eng.run()
         gh = g_host if g_host is not None else host_graph(g)
         r = oracle_sample(c, gh, W, first, args.cpu_seconds)
-        cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "kind": "oracle",
+        cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "cpu_model": cpu_model(), "kind": "oracle",
                "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
                          f"{r['seconds']:.1f} s; oracle/ C + OpenMP, {cores()} threads)"}
         idx = np.linspace(0, r["walks"] - 1, num=min(r["walks"], 20000)).astype(np.uint64)
