@@ -617,6 +617,8 @@ def main():
         cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "cpu_model": cpu_model(), "kind": "oracle",
                "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
                          f"{r['seconds']:.1f} s; oracle/ C + OpenMP, {cores()} threads)"}
+        r1 = oracle_sample(c, gh, W, first, min(3.0, args.cpu_seconds / 4), threads=1)  # per-core context
+        cpu["single_thread"] = {"value": r1["value"], "cores": 1, "sample": f"walks {first}..{first + r1['walks'] - 1}"}
         idx = np.linspace(0, r["walks"] - 1, num=min(r["walks"], 20000)).astype(np.uint64)
         gp, gl = eng.get_paths_rows(idx)
         ii = idx.astype(np.int64)
