@@ -433,7 +433,10 @@ __device__ __forceinline__ Adj ld_adj12(const uint32_t* a12, unsigned long long 
 //            vertex's degree and offset, so only a visit's first step reads row_ptr.
 // Offsets are global CSR positions; col / adj hold the entries from wk.ebase on (an out-of-core
 // block's slice, or the owned slice with range ownership), so every gather subtracts ebase.
-template <int ILP> struct MinBlocks { static constexpr int v = 4; };
+#ifndef LT_UPD_MINB
+#define LT_UPD_MINB 4  // resident 256-thread blocks per SM the batch kernel's registers are cut for (ILP 1)
+#endif
+template <int ILP> struct MinBlocks { static constexpr int v = LT_UPD_MINB; };
 template <> struct MinBlocks<2> { static constexpr int v = 3; };
 template <> struct MinBlocks<4> { static constexpr int v = 2; };
 
