@@ -382,7 +382,10 @@ def main():
             if not attached:  # receive buffers for every walk, shared once through CUDA IPC
                 ltdist.attach_peers(eng, comm, W)
                 attached.append(True)
-            superstep_counters.update(ltdist.run_supersteps_p2p(eng, comm, f"cuda:{local}"))
+            # one owned partition per rank, HBM-resident: the fused superstep (one host round trip each)
+            fused = P == world and not ooc
+            run = ltdist.run_supersteps_p2p_fused if fused else ltdist.run_supersteps_p2p
+            superstep_counters.update(run(eng, comm, f"cuda:{local}"), fused=fused)
         elif own:
             superstep_counters.update(ltdist.run_supersteps(eng, comm, f"cuda:{local}"))
         else:

@@ -338,6 +338,14 @@ lt_status lt_exchange_sent(lt_ctx* ctx, uint64_t* sent);
  * records that arrived in this rank's buffer of the current parity into the owned buckets, reset its
  * cursor and the sent count, flip the parity. *received = the number inserted. Stream-ordered. */
 lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received);
+/* One fused superstep of the peer exchange, with no host synchronisation (one owned partition per
+ * rank, HBM-resident, no walk-pool cap): insert the walks peers appended in the previous superstep
+ * (count read on the device), reset that cursor, advance every owned walk in one update launch (walks
+ * end or are appended to their owner's buffer of this superstep's parity), write the number of records
+ * this rank sent to *d_sent (device u64), flip the parity. Loop (dist.run_supersteps_p2p_fused):
+ * lt_superstep_p2p -> sum of d_sent over ranks (a device all-reduce; 0 ends it) -> ..., then one
+ * lt_run to finalise statistics and visit counts. */
+lt_status lt_superstep_p2p(lt_ctx* ctx, unsigned long long* d_sent);
 /* CUDA IPC of a device allocation's base pointer (handle: 64 bytes), and opening another process's
  * handle on this context's device (closed at lt_destroy). */
 lt_status lt_ipc_handle(const void* dptr, void* handle);

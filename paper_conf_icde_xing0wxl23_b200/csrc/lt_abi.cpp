@@ -1007,6 +1007,33 @@ lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received) {
   return LT_OK;
 }
 
+lt_status lt_superstep_p2p(lt_ctx* ctx, unsigned long long* d_sent) {
+  if (!ctx || !d_sent) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->peer_on) return fail(LT_ERR_STATE, "lt_superstep_p2p before lt_exchange_attach");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "no walks");
+  if (ctx->own_hi - ctx->own_lo != 1 || ctx->ooc.on || ctx->cap_walks < ctx->W)
+    return fail(LT_ERR_INVALID, "lt_superstep_p2p needs one owned partition per rank, an HBM-resident graph "
+                                "and no walk-pool cap; use lt_run + lt_exchange_take");
+  CK(cudaSetDevice(ctx->cfg.device));
+  cudaStream_t s = ctx->stream;
+  // (1) the walks peers appended in the previous superstep (parity epoch ^ 1) into the owned bucket
+  const uint32_t prev = ctx->peer_epoch ^ 1u;
+  CK(lt::launch_insert_records_dev(ctx->params, ctx->d_xbuf[prev], ctx->d_xcur + prev, s));
+  CK(cudaMemsetAsync(ctx->d_xcur + prev, 0, sizeof(unsigned long long), s));
+  CK(cudaMemsetAsync(&ctx->d_ctr->sent, 0, sizeof(unsigned long long), s));
+  // (2) every owned walk steps until it ends or leaves for a peer (parity epoch), in one launch: the
+  // owned bucket is the only one this rank consumes and walks stay in the kernel while inside it
+  ctx->params.peer.epoch = ctx->peer_epoch;
+  lt_status st = lt::launch_update_timed(ctx, ctx->params, ctx->own_lo, ~0ull >> 8);
+  if (st != LT_OK) return st;
+  CK(cudaMemcpyAsync(d_sent, &ctx->d_ctr->sent, sizeof(unsigned long long), cudaMemcpyDeviceToDevice, s));
+  ctx->stats.kernel_launches += 1;
+  ctx->snap_valid = false;
+  ctx->peer_epoch ^= 1u;
+  ctx->params.peer.epoch = ctx->peer_epoch;
+  return LT_OK;
+}
+
 lt_status lt_ipc_handle(const void* dptr, void* handle) {
   if (!dptr || !handle) return fail(LT_ERR_INVALID, "NULL argument");
   cudaIpcMemHandle_t h;

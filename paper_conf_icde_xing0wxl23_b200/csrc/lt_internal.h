@@ -124,6 +124,9 @@ struct Params {
 // walks [first_row, first_row + W) from starts[0..W): records, visit counts, insertion (a2)
 cudaError_t launch_init(const Params& p, const uint32_t* starts, uint64_t W, uint64_t first_row, cudaStream_t s);
 cudaError_t launch_insert_records(const Params& p, const uint4* recs, uint64_t count, cudaStream_t s);
+// the same with the record count read from device memory (fused superstep of the peer exchange)
+cudaError_t launch_insert_records_dev(const Params& p, const uint4* recs, const unsigned long long* dcount,
+                                      cudaStream_t s);
 cudaError_t launch_pack(const Params& p, uint32_t bucket, uint4* out, uint64_t count, cudaStream_t s);
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s);
 cudaError_t launch_finalize_paths(const Params& p, uint64_t W, cudaStream_t s);

@@ -253,8 +253,10 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
 
 // a9 receive side: records that arrived from other ranks go into the buckets of their (owned)
 // partitions with the same warp-aggregated insertion.
-__global__ void __launch_bounds__(256) k_insert_records(Params p, const uint4* __restrict__ recs, uint64_t count) {
+__global__ void __launch_bounds__(256) k_insert_records(Params p, const uint4* __restrict__ recs, uint64_t count,
+                                                        const unsigned long long* __restrict__ dcount) {
   extern __shared__ uint32_t s_bounds[];
+  if (dcount) count = *dcount;  // fused superstep: the count is read on the device (no host round trip)
   const Walk& wk = p.wk;
   const uint32_t* B = stage_bounds(wk, s_bounds);
   const uint32_t lane = threadIdx.x & 31u;
@@ -1147,7 +1149,14 @@ cudaError_t launch_insert_records(const Params& p, const uint4* recs, uint64_t c
   uint64_t want = (count + 255) / 256;
   uint32_t grid = (uint32_t)std::min<uint64_t>(want, (uint64_t)num_sms() * 8);
   cudaFuncSetAttribute(k_insert_records, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-  k_insert_records<<<grid, 256, bounds_smem(p), s>>>(p, recs, count);
+  k_insert_records<<<grid, 256, bounds_smem(p), s>>>(p, recs, count, nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_insert_records_dev(const Params& p, const uint4* recs, const unsigned long long* dcount,
+                                      cudaStream_t s) {
+  cudaFuncSetAttribute(k_insert_records, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
+  k_insert_records<<<num_sms() * 8, 256, bounds_smem(p), s>>>(p, recs, 0, dcount);
   return cudaGetLastError();
 }
 

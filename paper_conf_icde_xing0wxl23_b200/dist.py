@@ -73,6 +73,11 @@ class TorchComm:
         ops = {"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM}
         self.dist.all_reduce(t, op=ops[op], group=self.group)
 
+    def allreduce_sum_dev(self, t) -> int:
+        """In-place sum of a device tensor over ranks (NCCL), then its value on the host."""
+        self.dist.all_reduce(t, group=self.group)
+        return int(t.item())
+
     def allgather_obj(self, obj):
         out = [None] * self.world
         self.dist.all_gather_object(out, obj, group=self.group)
@@ -137,6 +142,11 @@ class ThreadComm:
 
     def allgather_obj(self, obj):
         return self._gather(obj)
+
+    def allreduce_sum_dev(self, t) -> int:
+        total = sum(self._gather(int(t.item())))
+        t.fill_(total)
+        return total
 
     same_process = True
 
@@ -214,6 +224,27 @@ def run_supersteps_p2p(engine, comm, device, max_supersteps: int = 1 << 20) -> d
         if total == 0:
             return {"supersteps": supersteps, "records_sent": moved}
         engine.exchange_take()
+        if supersteps >= max_supersteps:
+            raise RuntimeError("ownership supersteps did not converge")
+
+
+def run_supersteps_p2p_fused(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
+    """The peer-exchange superstep loop with ONE host round trip per superstep (one owned partition per
+    rank): lt_superstep_p2p (insert arrivals, step every owned walk, count what was sent — all
+    stream-ordered) and a device all-reduce of the sent count, whose value ends the loop at 0. A final
+    lt_run (no walk left) finalises statistics and visit counts."""
+    import torch
+    sent = torch.zeros(1, dtype=torch.int64, device=device)
+    moved = torch.zeros(1, dtype=torch.int64, device=device)  # this rank's records sent, summed on the device
+    supersteps = 0
+    while True:
+        engine.superstep_p2p(sent)
+        moved += sent
+        total = comm.allreduce_sum_dev(sent)
+        supersteps += 1
+        if total == 0:
+            engine.run()
+            return {"supersteps": supersteps, "records_sent": int(moved.item())}
         if supersteps >= max_supersteps:
             raise RuntimeError("ownership supersteps did not converge")
 

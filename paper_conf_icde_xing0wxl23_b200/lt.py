@@ -35,7 +35,7 @@ EXPORTED = [
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
     "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
     "lt_exchange_buffers", "lt_exchange_attach", "lt_exchange_sent", "lt_exchange_take", "lt_ipc_handle",
-    "lt_ipc_open",
+    "lt_ipc_open", "lt_superstep_p2p",
 ]
 
 
@@ -120,6 +120,7 @@ _lib.lt_exchange_sent.argtypes = [_vp, ctypes.POINTER(_u64)]
 _lib.lt_exchange_take.argtypes = [_vp, ctypes.POINTER(_u64)]
 _lib.lt_ipc_handle.argtypes = [_vp, _vp]
 _lib.lt_ipc_open.argtypes = [_vp, _vp, ctypes.POINTER(_vp)]
+_lib.lt_superstep_p2p.argtypes = [_vp, _vp]
 _lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
 _lib.lt_run_to_host_compact.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u64, _u32]
 _lib.lt_get_paths_compact.argtypes = [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]
@@ -428,6 +429,14 @@ class Engine:
         x = _u64()
         _check(_lib.lt_exchange_take(self._h, ctypes.byref(x)))
         return int(x.value)
+
+    def superstep_p2p(self, d_sent):
+        """One fused superstep (lt_superstep_p2p); d_sent: CUDA int64 tensor [1] receiving the number of
+        records this rank sent. No host synchronisation."""
+        pp, dev, _ = _ptr(d_sent, np.uint64)
+        if not dev:
+            raise ValueError("superstep_p2p needs a CUDA tensor")
+        _check(_lib.lt_superstep_p2p(self._h, pp))
 
     def export_buffers(self):
         """CUDA IPC handles of this rank's receive buffers (parity 0, 1) and of its cursor pair."""

@@ -271,3 +271,66 @@ def test_peer_exchange_processes_cuda_ipc(gpu):
     np.testing.assert_array_equal(lengths, ol)
     np.testing.assert_array_equal(paths, op)
     assert counters["records_sent"] > 0
+
+
+@pytest.mark.parametrize("world", [2, 3, 4])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 16), (LT.PPR, 0.15)])
+def test_fused_superstep_exact(gpu, g13, world, layout, app, param):
+    """lt_superstep_p2p (one owned partition per rank, one host round trip per superstep): merged
+    paths equal the oracle, the same walks cross ranks as with the unfused loop, and a second epoch on
+    the same engines works (parities stay aligned)."""
+    import torch
+    starts = (lt_inputs.deepwalk_starts(3 * g13.n, g13.n) if app == LT.DEEPWALK
+              else lt_inputs.ppr_starts(20_000, g13.argmax_deg))
+    hub = ltdist.ThreadComm.Hub(world)
+    out, errors = [None] * world, []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world, layout=layout, chunk_walks=512) as e:
+                e.graph_load(g13.row_ptr, g13.col, world)
+                comm = ltdist.ThreadComm(hub, r)
+                res = []
+                for seed in (2, 3):
+                    e.walks_init(starts, app, param, seed)
+                    if seed == 2:
+                        ltdist.attach_peers(e, comm, len(starts))
+                    cnt = ltdist.run_supersteps_p2p_fused(e, comm, "cuda")
+                    paths, lengths = ltdist.merge_paths(e, comm)
+                    torch.cuda.synchronize()
+                    res.append((paths.cpu().numpy().view(np.uint32), lengths.cpu().numpy().view(np.uint32), cnt,
+                                e.stats()))
+                out[r] = res
+        except Exception as ex:
+            errors.append(ex)
+            hub.barrier.abort()
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errors:
+        raise errors[0]
+    for i, seed in enumerate((2, 3)):
+        op, ol, osteps, _ = oracle_of(g13, starts, app, param, seed)
+        for r in range(world):
+            paths, lengths, cnt, st = out[r][i]
+            np.testing.assert_array_equal(lengths, ol)
+            np.testing.assert_array_equal(paths, op)
+        assert sum(out[r][i][3]["steps"] for r in range(world)) == osteps
+        assert sum(out[r][i][2]["records_sent"] for r in range(world)) > 0
+
+
+def test_fused_superstep_preconditions(gpu, g13):
+    with LT.Engine(rank=0, world=2) as e:
+        e.graph_load(g13.row_ptr, g13.col, 4)  # two owned partitions
+        e.walks_init(lt_inputs.deepwalk_starts(100, g13.n), LT.DEEPWALK, 5, 1)
+        import torch
+        sent = torch.zeros(1, dtype=torch.int64, device="cuda")
+        with pytest.raises(LT.LTError):
+            e.superstep_p2p(sent)  # not attached
+        e.exchange_buffers(100)
+        with pytest.raises(LT.LTError):
+            e.superstep_p2p(sent)

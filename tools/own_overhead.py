@@ -43,6 +43,7 @@ def main():
     ap.add_argument("--partitions", type=int, default=0, help="0: one per rank")
     ap.add_argument("--legacy", action="store_true")
     ap.add_argument("--p2p", action="store_true", help="peer exchange (dist.run_supersteps_p2p)")
+    ap.add_argument("--fused", action="store_true", help="peer exchange, fused superstep (run_supersteps_p2p_fused)")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--refill", type=int, default=0, help="lt_config.refill: 0 auto, 1 off, 2 on")
     a = ap.parse_args()
@@ -60,7 +61,7 @@ def main():
         with LT.Engine(rank=r, world=a.world, timing=True, refill=a.refill) as e:
             e.graph_load(g.row_ptr, g.col, P)
             comm = ltdist.ThreadComm(hub, r)
-            if a.p2p:
+            if a.p2p or a.fused:
                 e.walks_init(starts, LT.DEEPWALK, 80, 1)
                 ltdist.attach_peers(e, comm, g.n)
             for rep in range(a.reps + 1):
@@ -71,6 +72,8 @@ def main():
                 upd = 0.0
                 if a.legacy:
                     cnt = legacy_supersteps(e, comm, "cuda")
+                elif a.fused:
+                    cnt = ltdist.run_supersteps_p2p_fused(e, comm, "cuda")
                 elif a.p2p:
                     cnt = ltdist.run_supersteps_p2p(e, comm, "cuda")
                 else:
@@ -89,7 +92,7 @@ def main():
         t.join()
     wall = min(max(res[r][i][0] for r in range(a.world)) for i in range(a.reps))
     ss = res[0][-1][1]
-    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "p2p": a.p2p, "refill": a.refill,
+    out = {"config": a.config, "world": a.world, "partitions": P, "legacy": a.legacy, "p2p": a.p2p, "fused": a.fused, "refill": a.refill,
            "wall_ms": wall * 1e3,
            "supersteps": ss, "ms_per_superstep": wall * 1e3 / ss, "n": g.n,
            "library": os.environ.get("LT_LIBRARY", "liblt.so")}
