@@ -73,10 +73,9 @@ class TorchComm:
         ops = {"min": self.dist.ReduceOp.MIN, "max": self.dist.ReduceOp.MAX, "sum": self.dist.ReduceOp.SUM}
         self.dist.all_reduce(t, op=ops[op], group=self.group)
 
-    def allreduce_sum_dev(self, t) -> int:
-        """In-place sum of a device tensor over ranks (NCCL), then its value on the host."""
+    def allreduce_dev_(self, t):
+        """In-place sum of a device tensor over ranks (NCCL: enqueued, no host synchronisation)."""
         self.dist.all_reduce(t, group=self.group)
-        return int(t.item())
 
     def allgather_obj(self, obj):
         out = [None] * self.world
@@ -143,10 +142,8 @@ class ThreadComm:
     def allgather_obj(self, obj):
         return self._gather(obj)
 
-    def allreduce_sum_dev(self, t) -> int:
-        total = sum(self._gather(int(t.item())))
-        t.fill_(total)
-        return total
+    def allreduce_dev_(self, t):
+        t.fill_(sum(self._gather(int(t.item()))))
 
     same_process = True
 
@@ -228,11 +225,14 @@ def run_supersteps_p2p(engine, comm, device, max_supersteps: int = 1 << 20) -> d
             raise RuntimeError("ownership supersteps did not converge")
 
 
-def run_supersteps_p2p_fused(engine, comm, device, max_supersteps: int = 1 << 20) -> dict:
-    """The peer-exchange superstep loop with ONE host round trip per superstep (one owned partition per
+def run_supersteps_p2p_fused(engine, comm, device, max_supersteps: int = 1 << 20, sync_every: int = 4) -> dict:
+    """The peer-exchange superstep loop without per-superstep host decisions (one owned partition per
     rank): lt_superstep_p2p (insert arrivals, step every owned walk, count what was sent — all
-    stream-ordered) and a device all-reduce of the sent count, whose value ends the loop at 0. A final
-    lt_run (no walk left) finalises statistics and visit counts."""
+    stream-ordered) and a device all-reduce of the sent count. The host reads that sum only every
+    `sync_every` supersteps: a superstep after the last walk ended is empty and cheap (nothing to
+    insert, an update launch over an empty bucket), so running up to sync_every - 1 of them costs less
+    than a host round trip per superstep. A zero sum ends the loop; a final lt_run (no walk left)
+    finalises statistics and visit counts."""
     import torch
     sent = torch.zeros(1, dtype=torch.int64, device=device)
     moved = torch.zeros(1, dtype=torch.int64, device=device)  # this rank's records sent, summed on the device
@@ -240,11 +240,12 @@ def run_supersteps_p2p_fused(engine, comm, device, max_supersteps: int = 1 << 20
     while True:
         engine.superstep_p2p(sent)
         moved += sent
-        total = comm.allreduce_sum_dev(sent)
+        comm.allreduce_dev_(sent)  # NCCL: asynchronous; threads: a host gather
         supersteps += 1
-        if total == 0:
-            engine.run()
-            return {"supersteps": supersteps, "records_sent": int(moved.item())}
+        if supersteps % sync_every == 0 or comm.same_process:
+            if int(sent.item()) == 0:
+                engine.run()
+                return {"supersteps": supersteps, "records_sent": int(moved.item())}
         if supersteps >= max_supersteps:
             raise RuntimeError("ownership supersteps did not converge")
 

@@ -216,7 +216,7 @@ def test_peer_exchange_overflow_is_an_error(gpu, g13):
         run_owned_p2p(g13, starts, LT.DEEPWALK, 10, 1, 12, 2, capacity=16)
 
 
-def _p2p_proc(rank, world, port, out_q):
+def _p2p_proc(rank, world, port, out_q, fused=False):
     import os
 
     import torch
@@ -229,11 +229,14 @@ def _p2p_proc(rank, world, port, out_q):
         g = lt_inputs.rmat_cpu(13, 8 * 2 ** 13, seed=3)
         starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
         with LT.Engine(rank=rank, world=world) as e:
-            e.graph_load(g.row_ptr, g.col, 2 * world)
+            e.graph_load(g.row_ptr, g.col, world if fused else 2 * world)
             e.walks_init(starts, LT.DEEPWALK, 12, 7)
             comm = ltdist.TorchComm()
             ltdist.attach_peers(e, comm, len(starts))  # CUDA IPC between the processes
-            counters = ltdist.run_supersteps_p2p(e, comm, "cpu")
+            if fused:  # speculative supersteps: the host reads the sent sum every 4th superstep
+                counters = ltdist.run_supersteps_p2p_fused(e, comm, "cuda:0")
+            else:
+                counters = ltdist.run_supersteps_p2p(e, comm, "cpu")
             paths, lengths = e.partial_paths()
             paths, lengths = paths.cpu(), lengths.cpu()
             paths ^= ltdist.SIGN
@@ -246,7 +249,8 @@ def _p2p_proc(rank, world, port, out_q):
         tdist.destroy_process_group()
 
 
-def test_peer_exchange_processes_cuda_ipc(gpu):
+@pytest.mark.parametrize("fused", [False, True])
+def test_peer_exchange_processes_cuda_ipc(gpu, fused):
     """Two processes on one GPU, each rank's receive buffers opened by the other through CUDA IPC
     (lt_ipc_handle / lt_ipc_open): the multi-process wiring of the peer exchange."""
     import socket
@@ -258,7 +262,7 @@ def test_peer_exchange_processes_cuda_ipc(gpu):
     s.close()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_p2p_proc, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_p2p_proc, args=(r, 2, port, q, fused)) for r in range(2)]
     for p in procs:
         p.start()
     paths, lengths, counters = q.get(timeout=300)
