@@ -84,6 +84,27 @@ class CpuOwnerEngine:
         self.epoch ^= 1
         return got
 
+    def superstep_p2p(self, sent):
+        """Fused superstep (lt_superstep_p2p): arrivals of the previous parity into the owned bucket,
+        then the owned partition stepped once; `sent` (a tensor [1]) receives the records sent."""
+        assert self.own_hi - self.own_lo == 1
+        prev = self.epoch ^ 1
+        for sender in range(self.world):
+            cur, recs = self._seg(self._own_shm.name, prev, sender)
+            for w, v, t, _ in recs[: int(cur[0])]:
+                self.buckets[self._bucket(self._part(int(v)))].append((int(w), int(v), int(t)))
+            cur[0] = 0
+        self.sent = 0
+        k = self.own_lo
+        lo, hi = int(self.bounds[k]), int(self.bounds[k + 1])
+        recs, self.buckets[k] = self.buckets[k], []
+        for rec in recs:
+            out = self._visit(rec, lo, hi)
+            if out is not None:
+                self._send(self._bucket(self._part(out[1])) - self.P, out)
+        sent.fill_(self.sent)
+        self.epoch ^= 1
+
     def close_exchange(self):
         for shm in self._shms.values():
             shm.close()

@@ -79,7 +79,7 @@ def test_ownership_protocol_gloo(world, app, param):
     assert counters["supersteps"] >= 2 and counters["records_sent"] > 0
 
 
-def _worker_p2p(rank, world, port, app, param, P, out_q):
+def _worker_p2p(rank, world, port, app, param, P, out_q, fused=False):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
     import torch.distributed as dist
@@ -102,7 +102,10 @@ def _worker_p2p(rank, world, port, app, param, P, out_q):
             eng.walks_init(starts, app, param, seed)
             if seed == 11:
                 ltdist.attach_peers(eng, comm, W)
-            counters = ltdist.run_supersteps_p2p(eng, comm, "cpu")
+            if fused:  # one owned partition per rank; the host reads the sum every 4th superstep
+                counters = ltdist.run_supersteps_p2p_fused(eng, comm, "cpu")
+            else:
+                counters = ltdist.run_supersteps_p2p(eng, comm, "cpu")
             paths, lengths = ltdist.merge_paths(eng, comm)
             res.append((paths.numpy().view(np.uint32).copy(), lengths.numpy().view(np.uint32).copy(), counters))
         dist.barrier()
@@ -117,13 +120,15 @@ def _worker_p2p(rank, world, port, app, param, P, out_q):
 
 @pytest.mark.parametrize("world", [2, 3])
 @pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 12), (LT.PPR, 0.2)])
-def test_peer_exchange_protocol_gloo(world, app, param):
+@pytest.mark.parametrize("fused", [False, True])
+def test_peer_exchange_protocol_gloo(world, app, param, fused):
     """dist.attach_peers + run_supersteps_p2p over gloo (the CPU stand-in emulates the receive buffers
     with shared memory): merged paths equal the oracle over two epochs."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker_p2p, args=(r, world, port, app, param, 8, q)) for r in range(world)]
+    P = world if fused else 8
+    procs = [ctx.Process(target=_worker_p2p, args=(r, world, port, app, param, P, q, fused)) for r in range(world)]
     for p in procs:
         p.start()
     res = q.get(timeout=300)
