@@ -256,7 +256,9 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
 __global__ void __launch_bounds__(256) k_insert_records(Params p, const uint4* __restrict__ recs, uint64_t count,
                                                         const unsigned long long* __restrict__ dcount) {
   extern __shared__ uint32_t s_bounds[];
-  if (dcount) count = *dcount;  // fused superstep: the count is read on the device (no host round trip)
+  // fused superstep: the count is read on the device (no host round trip); a cursor past the buffer
+  // (an overflow, flagged by the sender and reported by its lt_run) is clamped to what was stored
+  if (dcount) count = (*dcount < p.peer.cap) ? *dcount : p.peer.cap;
   const Walk& wk = p.wk;
   const uint32_t* B = stage_bounds(wk, s_bounds);
   const uint32_t lane = threadIdx.x & 31u;

@@ -338,3 +338,33 @@ def test_fused_superstep_preconditions(gpu, g13):
         e.exchange_buffers(100)
         with pytest.raises(LT.LTError):
             e.superstep_p2p(sent)
+
+
+def test_fused_superstep_overflow_is_an_error(gpu, g13):
+    """A receive buffer too small for one superstep's arrivals: the fused loop still ends (the
+    receiver inserts only what was stored) and the sending rank's final lt_run reports the overflow."""
+    import torch
+    world = 2
+    hub = ltdist.ThreadComm.Hub(world)
+    errors = []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world) as e:
+                e.graph_load(g13.row_ptr, g13.col, world)
+                e.walks_init(lt_inputs.deepwalk_starts(g13.n, g13.n), LT.DEEPWALK, 10, 1)
+                comm = ltdist.ThreadComm(hub, r)
+                ltdist.attach_peers(e, comm, 16)
+                try:
+                    ltdist.run_supersteps_p2p_fused(e, comm, "cuda")
+                finally:
+                    torch.cuda.synchronize()
+        except LT.LTError as ex:
+            errors.append(ex)
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert errors and all("overflow" in str(x) for x in errors)
