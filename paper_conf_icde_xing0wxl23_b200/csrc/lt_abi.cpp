@@ -616,7 +616,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
-  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0);
+  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0, p.wk.app);
   p.direct = direct ? lt::Direct{d_starts, W} : lt::Direct{nullptr, 0};
   p.peer = ctx->peer_on ? lt::Peer{ctx->d_peer_recv, ctx->d_peer_cur, ctx->xcap, ctx->peer_epoch} : lt::Peer{};
   ctx->stats.direct_start = direct ? 1 : 0;

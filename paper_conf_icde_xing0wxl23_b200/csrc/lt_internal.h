@@ -155,7 +155,7 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
                              cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
                                cudaStream_t s);
-int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill);  // resident blocks per SM (update kernel)
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill, uint32_t app);  // resident blocks per SM (update kernel)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

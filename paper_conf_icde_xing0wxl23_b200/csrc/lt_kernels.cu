@@ -667,9 +667,17 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
 // without refill most lanes of a warp idle most of the time. A warp claims kRefill positions of the
 // bucket at a time (one atomic per kRefill walks) and hands them to its idle lanes.
 constexpr uint32_t kRefill = 64;
-#ifndef LT_RF_MINB
-#define LT_RF_MINB 4  // resident 256-thread blocks per SM the register budget is cut for (64 regs)
+// Resident 256-thread blocks per SM the register budget is cut for. Measured on one B200 (DESIGN.md §8,
+// profiles/r01_rf_minb_cmp.jsonl): 3 (up to 85 registers, no spills) is 2.6-3.0 % faster than 4 (64
+// registers, 2 spilled) for DeepWalk cfg 4 and 1.2-1.7 % for PageRank; PPR's short walks want the 4th
+// block (3: 1.3 % slower). LT_RF_MINB overrides all apps (experiments).
+template <int APP> struct RfMinBlocks {
+#ifdef LT_RF_MINB
+  static constexpr int v = LT_RF_MINB;
+#else
+  static constexpr int v = APP == 1 ? 4 : 3;
 #endif
+};
 
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
@@ -687,7 +695,7 @@ __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, c
 // covers); a walk that leaves the view for a partition whose block is in p.cont.table switches to that
 // block's view and keeps stepping.
 template <int APP, int GM, int LAY, int VIS, int CONT>
-__global__ void __launch_bounds__(256, LT_RF_MINB) k_update_rf(Params p, uint32_t k) {
+__global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p, uint32_t k) {
   extern __shared__ uint32_t s_bounds[];
   const Walk& wk = p.wk;
   const Pool& pl = p.pool;
@@ -1098,9 +1106,10 @@ int num_sms() {
 
 uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 
-int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill) {
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill, uint32_t app) {
   int nb = 0;
-  if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
+  if (refill && app == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<1, 3, 1, 0, 0>, (int)block, 0);
+  else if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
   else if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
   else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1, 0>, (int)block, 0);
   else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 2, 1, 0>, (int)block, 0);
