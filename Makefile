@@ -43,7 +43,7 @@ $(CSRC)/%.o: $(CSRC)/%.cpp $(LT_H)
 	$(CXX) -O3 -fPIC -std=c++17 -Wall -Wextra -Iinclude -I/usr/local/cuda/include -c $< -o $@
 
 $(PKG)/liblt.so: $(LT_CU:.cu=.o) $(LT_CPP:.cpp=.o)
-	$(NVCC) $(ARCH) -shared $^ -o $@
+	$(NVCC) $(ARCH) -shared $^ -o $@ -ldl
 
 # Experiment builds of liblt.so with compile-time switches (tools/variants/ is not shipped product):
 #   make variant VTAG=nohint VDEFS="-DLT_PATH_HINT=0 -DLT_VIS_HINT=0"; run with LT_LIBRARY=tools/variants/liblt_nohint.so

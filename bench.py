@@ -21,8 +21,16 @@ a3-a7). Workload (default): BASELINE.json configs[3], the Friendster-shaped R-MA
   cpu_baseline  the CPU oracle (oracle/, as it stands) on this box's host cores over a bounded
             sample of the same workload's walks (rank 0, N=1 only).
 
-Multi-GPU (torchrun, N>1): "replicas" mode — every rank holds the whole graph and runs its own |V|
-walks (walk IDs offset by rank*|V|): no data-path collective, weak scaling.
+Multi-GPU (N>1, one process per GPU; `--gpus N` without torchrun re-launches itself under
+torch.distributed.run): the north star's range-ownership mode by default — |V| walks in total over N
+ranks, rank r owning a contiguous edge-balanced vertex range, walks crossing ranks appended by the
+update kernels straight into the owner's receive buffer over peer memory, one small all-reduce per
+superstep (strong scaling). The line adds a per-superstep breakdown and a `replicas_upper_bound` leg
+(every rank the whole graph and |V|/N of the walks, no exchange: the communication-free bound).
+`--mode replicas` makes the replicas run the headline instead (weak scaling: |V| walks per rank).
+At N=1 the line adds `projection_8gpu`: the ownership mode's 8-GPU time predicted from one-GPU
+measurements (the P=8 partitioned kernel's update time / 8 plus a per-superstep cost), stated with
+its assumptions.
 `--impl reference` times the oracle (the reference arm of this tier) on the host cores instead.
 """
 from __future__ import annotations
@@ -93,11 +101,30 @@ def parse():
                          "the owner's receive buffer over peer memory (p2p, default: CUDA IPC, one small "
                          "all-reduce per superstep), or go through lt_exchange_pack + an NCCL all-to-all "
                          "(nccl, the baseline)")
-    ap.add_argument("--mode", default="replicas", choices=["replicas", "own"],
-                    help="N>1: replicas (each rank its own |V| walks, no collective, weak scaling) or own "
-                         "(range ownership: |V| walks in total, NCCL all-to-all of crossing walks per "
-                         "superstep, strong scaling)")
+    ap.add_argument("--mode", default=None, choices=["replicas", "own"],
+                    help="N>1: own (default: range ownership, |V| walks in total, the crossing walks exchanged "
+                         "every superstep, strong scaling) or replicas (each rank its own |V| walks, no "
+                         "collective, weak scaling)")
+    ap.add_argument("--project-gpus", type=int, default=8,
+                    help="N=1, DeepWalk: predict the ownership mode's time at this many GPUs from one-GPU "
+                         "measurements (0: off)")
+    ap.add_argument("--no-replicas-bound", action="store_true", help="N>1 own mode: skip the replicas leg")
     return ap.parse_args()
+
+
+def free_port():
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def launch_ranks(args):
+    """`--gpus N` (N > 1) outside torchrun: run this script under torch.distributed.run with one
+    process per GPU (the driver's own launch line) and pass its output through."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 DEFAULT_P = {1: 4, 2: 1, 3: 1, 4: 1, 5: 1}
@@ -189,29 +216,36 @@ class Clocks:
 
 
 # ------------------------------------------------------------------------------ CPU oracle legs
-def oracle_sample(c, g_host, W, first, seconds, threads=None):
-    """Time the oracle (as it stands) on a bounded prefix sample of the workload's walks, with one
-    OpenMP thread per host core this process may use (explicitly: torchrun exports
-    OMP_NUM_THREADS=1, which would otherwise leave the oracle on one core)."""
+def oracle_sample(c, g_host, W, first, seconds, threads=None, runs=1):
+    """Time the oracle (as it stands) on a bounded sample of the workload's walks — `runs` repetitions of
+    the same spread sample (every k-th walk), median and spread reported — with one OpenMP thread per
+    host core this process may use (explicitly: torchrun exports OMP_NUM_THREADS=1, which would otherwise
+    leave the oracle on one core). The clock brackets the oracle's walk loop only (oracle_walks through
+    ctypes, output buffers preallocated by the binding)."""
     if threads is None:
         threads = cores()
     import oracle as O
     app = {"deepwalk": O.DEEPWALK, "ppr": O.PPR, "pagerank": O.PAGERANK}[c["app"]]
     alpha = float(c["restart_p"]) if c["app"] == "pagerank" else float(c.get("alpha", 0.15))
     kw = dict(app=app, length=int(c.get("length", 0)), alpha=alpha, seed=c["seed"], threads=threads)
-    # calibrate on a small prefix, then size the sample for ~`seconds` of work
+    all_starts = starts_for(c, g_host, W, first)
+    # calibrate on a small spread sample, then size the sample for ~`seconds` / runs of work per run
     n0 = min(W, 200_000)
-    st = starts_for(c, g_host, n0, first)
+    ids0 = np.linspace(0, W - 1, num=n0).astype(np.uint64)
     t0 = time.perf_counter()
-    O.walks(g_host.row_ptr, g_host.col, st, ids=np.arange(first, first + n0, dtype=np.uint64), **kw)
+    O.walks(g_host.row_ptr, g_host.col, all_starts[ids0.astype(np.int64)], ids=ids0 + np.uint64(first), **kw)
     dt = max(time.perf_counter() - t0, 1e-4)
-    ns = int(min(W, max(n0, n0 * seconds / dt)))
-    ids = np.arange(first, first + ns, dtype=np.uint64)
-    st = starts_for(c, g_host, ns, first)
-    t0 = time.perf_counter()
-    paths, lengths, steps, _ = O.walks(g_host.row_ptr, g_host.col, st, ids=ids, **kw)
-    dt = time.perf_counter() - t0
-    return dict(value=steps / dt, steps=steps, seconds=dt, walks=ns, paths=paths, lengths=lengths)
+    ns = int(min(W, max(n0, n0 * seconds / runs / dt)))
+    rows = np.linspace(0, W - 1, num=ns).astype(np.uint64)
+    st = all_starts[rows.astype(np.int64)]
+    vals, secs = [], []
+    for _ in range(runs):
+        t0 = time.perf_counter()
+        paths, lengths, steps, _ = O.walks(g_host.row_ptr, g_host.col, st, ids=rows + np.uint64(first), **kw)
+        secs.append(time.perf_counter() - t0)
+        vals.append(steps / secs[-1])
+    return dict(value=statistics.median(vals), values=vals, steps=steps, seconds=statistics.median(secs), walks=ns,
+                rows=rows, paths=paths, lengths=lengths)
 
 
 def host_graph(g):
@@ -304,6 +338,12 @@ def run_reference(args):
 # ------------------------------------------------------------------------------ CUDA arm
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return launch_ranks(args)
+    if int(os.environ.get("WORLD_SIZE", "1")) != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={os.environ.get('WORLD_SIZE')} processes were "
+              f"launched; run one process per GPU", file=sys.stderr)
+        return 2
     if args.impl == "reference":
         return run_reference(args)
     import torch
@@ -333,7 +373,8 @@ def main():
     g = make_graph(c, local)
     gen_s = time.time() - t0
     W = num_walks(c, g)
-    own = args.mode == "own" and world > 1
+    mode = args.mode or ("own" if world > 1 else "replicas")
+    own = mode == "own" and world > 1
     if own and args.partitions is None:
         P = c["partitions"] = world  # one contiguous partition per rank: fewest crossings
     first = 0 if own else rank * W
@@ -355,12 +396,21 @@ def main():
     eng.graph_load(g.row_ptr, g.col, P)
     load_s = time.time() - t0
     g_host = None
-    if args.release_col and not ooc and eng.stats()["layout"] != LT.LAYOUT_CSR and not isinstance(g.col, np.ndarray) \
-            and not args.sweep:
-        if rank == 0 and world == 1 and not args.no_cpu_baseline:
-            g_host = host_graph(g)
-        g = lt_inputs.Graph(g.n, g.m, g.row_ptr, None, g.max_deg, g.argmax_deg)
-        torch.cuda.empty_cache()
+    want_projection = world == 1 and args.project_gpus > 1 and c["app"] == "deepwalk" and not ooc and P == 1
+
+    def release_col():
+        """Once an augmented layout is built the steps never read col: keep a host copy for the oracle legs
+        and free the device one (room for the e2e buffers)."""
+        nonlocal g, g_host
+        if args.release_col and not ooc and eng.stats()["layout"] != LT.LAYOUT_CSR and \
+                not isinstance(g.col, np.ndarray) and g.col is not None and not args.sweep:
+            if rank == 0 and world == 1 and not args.no_cpu_baseline:
+                g_host = host_graph(g)
+            g = lt_inputs.Graph(g.n, g.m, g.row_ptr, None, g.max_deg, g.argmax_deg)
+            torch.cuda.empty_cache()
+
+    if not want_projection:
+        release_col()
 
     def barrier():
         torch.cuda.synchronize()
@@ -430,16 +480,21 @@ def main():
     if os.path.exists(peaks_path):
         peak, peak_src = float(json.load(open(peaks_path))["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
     achieved = (alg_bytes / upd_launches) / (upd_ms / upd_launches / 1000.0) / 1e9 if upd_ms > 0 else None
+    # DRAM traffic of the update kernel: not measurable inside a timed run (ncu replays the kernel), so it
+    # is the static figure of the last `ncu --set full` capture of this configuration, marked as such
     traffic = None
+    traffic_source = None
     sector_eff = None
     prof = os.path.join(ROOT, "profiles", "update_kernel_traffic.json")
     if os.path.exists(prof):
         pj = json.load(open(prof))
-        if pj.get("config_key") == f"cfg{args.config}-P{P}-layout{args.layout}":
+        if pj.get("config_key") == f"cfg{args.config}-P{P}-layout{args.layout}" and not own and not ooc:
             traffic = pj.get("dram_bytes_per_launch")
+            traffic_source = (f"static: ncu --set full capture {pj.get('source', 'profiles/update_kernel_traffic.json')} "
+                              f"of this configuration ({pj.get('captured', 'see file')}), not measured in this run")
             sector_eff = {"ld_bytes_per_sector": pj.get("sector_efficiency_ld_bytes"),
                           "st_bytes_per_sector": pj.get("sector_efficiency_st_bytes"),
-                          "source": "ncu, profiles/update_kernel_traffic.json"}
+                          "source": "static: ncu, profiles/update_kernel_traffic.json"}
     layout = stats[-1]["layout"]
     # DRAM-missing random gathers issued by the update kernel: one per step (ADJ: adj entry;
     # CSR: col entry) + the row_ptr line per step (CSR) or per visit (ADJ)
@@ -451,14 +506,51 @@ def main():
         gather = {"gathers_per_s": gathers / (upd_ms / 1000.0), "per_step": gathers / max(1, steps_k)}
         if os.path.exists(gc_path):
             gc = json.load(open(gc_path))
-            gather["ceiling_per_s"] = gc["ceiling_gathers_per_s"]
-            gather["frac"] = gather["gathers_per_s"] / gc["ceiling_gathers_per_s"]
-            gather["ceiling_source"] = "profiles/gather_ceiling.json (tools/gather_bench)"
+            gather["microbench_per_s"] = gc["microbench_gathers_per_s"]
+            gather["vs_microbench"] = gather["gathers_per_s"] / gc["microbench_gathers_per_s"]
+            gather["microbench_source"] = ("profiles/gather_ceiling.json (tools/gather_bench at the workload's "
+                                           "footprint; a reference rate, not a proven ceiling: it can be exceeded)")
+    frac = (achieved / peak) if achieved else None
+    if frac is not None and frac > 1.0:  # algorithmic bytes above the copy peak: the timing is broken
+        print(f"bench.py: roofline frac {frac:.3f} > 1 (update_ms {upd_ms}, {upd_launches} launches): refusing "
+              f"to report it", file=sys.stderr)
+        achieved, frac = None, None
     roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": (achieved / peak) if achieved else None, "traffic": traffic,
+            "frac": frac, "traffic": traffic, "traffic_source": traffic_source,
             "kernel": "k_update", "launches": upd_launches, "avg_launch_ms": upd_ms / max(1, upd_launches),
             "alg_bytes_per_step": alg_bytes / max(1, steps_k), "peak_source": peak_src,
             "update_share_of_step": upd_ms / ms, "gather": gather, "sector_efficiency": sector_eff}
+
+    # ---- ownership mode at R GPUs predicted from one-GPU measurements (N=1, DeepWalk, HBM-resident)
+    projection = None
+    if want_projection:
+        R = args.project_gpus
+        eng.graph_load(g.row_ptr, g.col, R)  # same engine, R partitions: the R ranks' partitions on one GPU
+        sts2 = []
+        for i in range(3):
+            init_walks(eng, c, starts_d, args.seed, first)
+            eng.run()
+            if i:
+                sts2.append(eng.stats())
+        upd = sum(s["update_ms"] for s in sts2) / len(sts2)
+        run_ms = sum(s["run_ms"] for s in sts2) / len(sts2)
+        sweeps = sts2[-1]["sweeps"]
+        launches = sts2[-1]["update_launches"]
+        gap = (run_ms - upd) / max(1, launches)  # host + launch time per update launch on one GPU
+        allreduce_ms = 0.020  # ASSUMED: one 8-byte NCCL all-reduce over NVSwitch per superstep
+        t_r = upd / R + sweeps * (2 * gap + allreduce_ms)
+        projection = {
+            "gpus": R, "projected_ms_per_step": t_r, "projected_speedup": (ms_max / args.steps) / t_r,
+            "projected_steps_per_s": steps_local / args.steps / (t_r / 1e3),
+            "inputs": {"update_ms_all_partitions_1gpu": upd, "supersteps": sweeps, "update_launches_1gpu": launches,
+                       "gap_ms_per_launch_1gpu": gap, "allreduce_ms_assumed": allreduce_ms,
+                       "kernel": "refill auto at P = R", "visits_per_step": sts2[-1]["visits"] / max(1, sts2[-1]["steps"])},
+            "model": ("ownership, one partition per rank: every superstep each rank runs one update launch over its "
+                      "partition's bucket (the P = R run's update time split evenly over R ranks: edge-balanced "
+                      "ranges, stationary load proportional to degree) plus an insert launch and one 8-byte "
+                      "all-reduce; supersteps = the P = R run's sweeps. Not a measurement: no multi-GPU box.")}
+        eng.graph_load(g.row_ptr, g.col, P)  # back to the headline configuration for the legs below
+        release_col()
 
     # ---- extra partition-count sweep (context; the headline uses P above)
     sweep = {}
@@ -616,17 +708,17 @@ def main():
         init_walks(eng, c, starts_d, args.seed, first)
         eng.run()
         gh = g_host if g_host is not None else host_graph(g)
-        r = oracle_sample(c, gh, W, first, args.cpu_seconds)
+        r = oracle_sample(c, gh, W, first, args.cpu_seconds, runs=5)
         cpu = {"value": r["value"], "unit": "steps/s", "cores": cores(), "cpu_model": cpu_model(), "kind": "oracle",
-               "sample": f"walks {first}..{first + r['walks'] - 1} of the workload ({r['steps']} steps, "
-                         f"{r['seconds']:.1f} s; oracle/ C + OpenMP, {cores()} threads)"}
+               "runs": 5, "stat": "median", "spread": [min(r["values"]), max(r["values"])],
+               "sample": f"{r['walks']} walks spread evenly over the workload's {W} ({r['steps']} steps, "
+                         f"median {r['seconds']:.2f} s per run; oracle/ C + OpenMP, {cores()} threads)"}
         r1 = oracle_sample(c, gh, W, first, min(3.0, args.cpu_seconds / 4), threads=1)  # per-core context
-        cpu["single_thread"] = {"value": r1["value"], "cores": 1, "sample": f"walks {first}..{first + r1['walks'] - 1}"}
-        idx = np.linspace(0, r["walks"] - 1, num=min(r["walks"], 20000)).astype(np.uint64)
-        gp, gl = eng.get_paths_rows(idx)
-        ii = idx.astype(np.int64)
-        mism = int(np.sum(np.any(gp != r["paths"][ii], axis=1) | (gl != r["lengths"][ii])))
-        parity = {"sampled_walks": int(len(idx)), "mismatched_walks": mism, "vs": "oracle (bit-exact)"}
+        cpu["single_thread"] = {"value": r1["value"], "cores": 1, "sample": f"{r1['walks']} walks spread evenly"}
+        # sampled parity: every walk of the timed sample (the oracle's paths) against the GPU's rows
+        gp, gl = eng.get_paths_rows(r["rows"])
+        mism = int(np.sum(np.any(gp != r["paths"], axis=1) | (gl != r["lengths"])))
+        parity = {"sampled_walks": int(len(r["rows"])), "mismatched_walks": mism, "vs": "oracle (bit-exact)"}
         if vis:  # the counts are a global sum: check their total and one sampled property exactly
             import oracle as O
             cnt = eng.visit_counts().astype(np.int64)
@@ -634,6 +726,47 @@ def main():
             parity["visit_counts_total_ok"] = bool(cnt.sum() == eng.stats()["steps"] + W)
             parity["visit_counts_of_sample_le_gpu"] = bool(np.all(
                 O.visit_counts(r["paths"], r["lengths"], g.n).astype(np.int64) <= cnt))
+
+    # ---- N>1 ownership: the communication-free bound (every rank the whole graph and 1/N of the walks)
+    replicas_bound = None
+    breakdown = None
+    if own:
+        upd = torch.tensor([sum(s["update_ms"] for s in stats) / len(stats)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(upd, op=dist.ReduceOp.MAX)
+        breakdown = {"supersteps": superstep_counters.get("supersteps"),
+                     "records_sent_rank0": superstep_counters.get("records_sent"),
+                     "update_ms_per_step_max_rank": float(upd.item()),
+                     "exchange_sync_ms_per_step": ms_max / args.steps - float(upd.item()),
+                     "exchange": args.exchange, "fused": superstep_counters.get("fused")}
+    if own and not args.no_replicas_bound:
+        eng.close()
+        torch.cuda.empty_cache()
+        a0, a1 = rank * W // world, (rank + 1) * W // world
+        with LT.Engine(device=local, timing=True, layout=args.layout, chunk_walks=args.chunk_walks,
+                       visit_counts=vis) as er:
+            er.graph_load(g.row_ptr, g.col, 1)
+            st_r = torch.from_numpy(starts_h[a0:a1].view(np.int32)).cuda(local)
+
+            def one_r():
+                init_walks(er, c, st_r, args.seed, a0)
+                er.run()
+                return er.stats()["steps"]
+
+            one_r()
+            barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            rs = sum(one_r() for _ in range(args.steps))
+            e1.record()
+            barrier()
+            rt = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device="cuda")
+            rsum = torch.tensor([rs], dtype=torch.float64, device="cuda")
+            dist.all_reduce(rt, op=dist.ReduceOp.MAX)
+            dist.all_reduce(rsum)
+            replicas_bound = {"value": float(rsum.item()) / (float(rt.item()) / 1e3), "unit": "steps/s",
+                              "ms_per_step": float(rt.item()) / args.steps, "walks_per_rank": a1 - a0,
+                              "what": "upper bound of the ownership mode: every rank holds the whole graph and "
+                                      "walks 1/N of the workload's walks, no exchange"}
 
     last = stats[-1]
     if rank == 0:
@@ -663,6 +796,11 @@ def main():
             line["host_link"] = host_link
         if own:
             line["ownership"] = dict(superstep_counters, exchange=args.exchange)
+            line["superstep_breakdown"] = breakdown
+            if replicas_bound:
+                line["replicas_upper_bound"] = replicas_bound
+        if projection:
+            line["projection_8gpu" if projection["gpus"] == 8 else f"projection_{projection['gpus']}gpu"] = projection
         if sweep:
             line["partition_sweep"] = sweep
         print(json.dumps(line), flush=True)

@@ -120,8 +120,10 @@ typedef struct lt_config {
                                  partitions. Every partition must fit one block
                                  (block = the largest partition's CSR slice). */
   uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
-  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P == 1, the measured
-                                 best), 1 off, 2 on */
+  uint32_t refill;            /* update kernel: 0 auto (lane refill when P == 1, the measured best),
+                                 1 the batch kernel, 2 lane refill, 3 the warp-specialised kernel (7
+                                 stepping warps with prefetched records + 1 inserting warp per CTA;
+                                 needs chunk_walks >= 256, else the batch kernel) */
   uint32_t visit_counts;      /* 1 -> count per-vertex visit frequency ("the visit
                                  frequency of each vertex is recorded") into a u64[n] device array
                                  reserved at lt_walks_init* and zeroed there: every path entry (start
@@ -132,7 +134,13 @@ typedef struct lt_config {
                                  partition resident in the graph pool keeps stepping there instead of
                                  being appended to its bucket (parity-neutral);
                                  uses the lane-refill kernel. Ignored when the graph is HBM-resident. */
-  uint32_t reserved0;
+  uint32_t walk_spill;        /* with walk_pool_walks < W: 0 -> walk admission (below); 1 -> spill: every
+                                 walk exists from the start and the walk pool EVICTS whole chunks of the
+                                 buckets with the fewest pending walks to pinned host memory when it is
+                                 full, and loads a partition's evicted chunks back before the partition
+                                 is computed (reading R17). Eviction (D2H)
+                                 and loading (H2D) run on their own stream through double-buffered
+                                 staging. Single-rank contexts only. Paths are unchanged. */
   uint64_t walk_pool_walks;   /* m_w, the walk pool's capacity in walks (D4; SURVEY.md
                                  8(f) f3): 0 -> sized for all W walks. When W > m_w the walks are
                                  admitted in index order as the pool drains: lt_walks_init creates the
@@ -186,6 +194,18 @@ typedef struct lt_stats {
                                   0 out of core (see pool_blocks x pool_block_bytes) */
   uint64_t l2_persist_bytes;   /* cudaLimitPersistingL2CacheSize set at lt_create (lt_config.l2_persist) */
   uint64_t prefetches;         /* out-of-core loads started ahead of the selection (lt_config.ooc_prefetch) */
+  /* walk spill (lt_config.walk_spill) in the last lt_walks_init + lt_run */
+  uint64_t spilled_chunks;     /* walk-pool chunks evicted to pinned host memory */
+  uint64_t reloaded_chunks;    /* evicted chunks loaded back before their partition was computed */
+  uint64_t spill_d2h_bytes;    /* walk records moved device -> host by evictions */
+  uint64_t spill_h2d_bytes;    /* walk records moved host -> device by reloads */
+  uint64_t host_chunks_peak;   /* most chunks held in host memory at once */
+  /* per-phase breakdown of the last lt_run (update vs reshuffle vs loading). The
+     reshuffle (bucket insertion, a5) is fused into the update kernels, so update_ms covers both. With
+     lt_config.timing: */
+  double load_ms;              /* graph-partition H2D copies on the load stream (out-of-core) */
+  double spill_xfer_ms;        /* walk-spill D2H + H2D copies on the transfer stream */
+  uint64_t host_syncs;         /* scheduler round trips: count reads that wait for the device */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,
@@ -356,7 +376,7 @@ lt_status lt_ipc_open(lt_ctx* ctx, const void* handle, void** dptr);
 typedef struct lt_pool_state {
   int64_t free_chunks;     /* free-stack depth */
   uint64_t ring_chunks;    /* installed (non-empty) ring slots over all partitions */
-  uint64_t reserved0;
+  uint64_t host_chunks;    /* chunks evicted to host memory (walk spill) */
   uint64_t total_chunks;
   uint64_t pending;        /* sum over partitions of cursor - head (walks waiting in buckets) */
   uint64_t finished;       /* walks with a recorded length */

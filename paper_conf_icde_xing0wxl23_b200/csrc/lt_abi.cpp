@@ -55,9 +55,10 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.world == 0) c.world = 1;
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
-  if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
+  if (c.refill > 3) return fail(LT_ERR_INVALID, "bad refill");
   if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
   if (c.direct_start > 1) return fail(LT_ERR_INVALID, "direct_start must be 0 (auto) or 1 (off)");
+  if (c.walk_spill > 1) return fail(LT_ERR_INVALID, "walk_spill must be 0 or 1");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
   CK(cudaGetDeviceCount(&ndev));
@@ -122,6 +123,9 @@ void lt_destroy(lt_ctx* ctx) {
   cudaSetDevice(ctx->cfg.device);
   if (ctx->stream) cudaStreamSynchronize(ctx->stream); else cudaDeviceSynchronize();
   free_ooc(ctx);
+  lt::free_spill(ctx);
+  ctx->load_ev.destroy();
+  ctx->xfer_ev.destroy();
   if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
   cudaFree(ctx->d_adj);
   cudaFree(ctx->d_adj12);
@@ -490,6 +494,7 @@ lt_status lt_walks_init_pagerank(lt_ctx* ctx, uint64_t W, const uint32_t* starts
 static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts, int on_device,
                                  uint64_t first_walk_id, lt_app app, double length_d, double alpha, uint64_t seed) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  lt::Range rg("lt_walks_init");
   if (!ctx->graph_loaded) return fail(LT_ERR_STATE, "lt_walks_init before lt_graph_load");
   if (W && !starts) return fail(LT_ERR_INVALID, "starts is NULL");
   if (W >= 0xFFFFFFFFull) return fail(LT_ERR_INVALID, "num_walks must be < 2^32 - 1");
@@ -542,7 +547,15 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const bool direct = ctx->cfg.direct_start == 0 && (ctx->cfg.refill == 0 || ctx->cfg.refill == 2) && ctx->P == 1 &&
                       ctx->world == 1 && !ctx->ooc.on && cap == W;
   const uint64_t wc = direct ? 0 : (cap + C - 1) / C;
-  const uint64_t ring_len = wc + 2;
+  // A bucket spans at most wc + 2 chunks, except with continuation during a zero-copy launch of
+  // partition i: a walk that goes i -> resident q -> i finds no block for i and is appended to bucket i
+  // while that launch still consumes [head, tail), so the bucket can span twice the walks.
+  const bool reenter = ctx->ooc.on && ctx->cfg.continue_resident && ctx->cfg.zero_copy;
+  // with walk spill a bucket's positions [head, cursor) may hold every walk (evicted chunks keep their
+  // ring slots), so its ring spans all W walks, not just the pool's
+  const bool spill = ctx->cfg.walk_spill == 1 && cap < W;
+  const uint64_t wr = spill ? (W + C - 1) / C : wc;
+  const uint64_t ring_len = reenter ? 2 * wr + 3 : wr + 2;
   const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
   const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
@@ -607,6 +620,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.cont = lt::Cont{};
   if (ctx->ooc.on && ctx->cfg.continue_resident)
     p.cont = lt::Cont{ctx->ooc.d_table, ctx->ooc.d_gpool, ctx->ooc.block_bytes, ctx->ooc.rp_bytes};
+  p.tail_cap = ~0ull;
   p.insert_mode = ctx->cfg.insert_mode;
   p.gather_mode = ctx->cfg.gather_mode;
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
@@ -614,9 +628,12 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
   // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
   p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
+  // warp-specialised kernel (refill 3): claims kWsMinChunk positions at a time, so it needs C >= that
+  if (ctx->cfg.refill == 3) p.refill = C >= lt::kWsMinChunk ? 3u : 0u;
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
-  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill != 0, p.wk.app);
+  ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm
+                                    : lt::update_kernel_occupancy(ctx->block, p.ilp, p.refill, p.wk.app, ctx->P);
   p.direct = direct ? lt::Direct{d_starts, W} : lt::Direct{nullptr, 0};
   p.peer = ctx->peer_on ? lt::Peer{ctx->d_peer_recv, ctx->d_peer_cur, ctx->xcap, ctx->peer_epoch} : lt::Peer{};
   ctx->stats.direct_start = direct ? 1 : 0;
@@ -633,6 +650,62 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.num_walks = W;
   ctx->stats.chunks_total = num_chunks;
   ctx->stats.kernel_launches = 0;
+  // per-epoch statistics: with range ownership lt_run (and lt_superstep_p2p) is called once per
+  // superstep and these accumulate over the epoch's supersteps, like the device step counter
+  ctx->stats.sweeps = 0;
+  ctx->stats.update_launches = 0;
+  ctx->stats.update_ms = 0;
+  ctx->stats.iterations = 0;
+  ctx->stats.explicit_copies = 0;
+  ctx->stats.pool_hits = 0;
+  ctx->stats.zero_copy_launches = 0;
+  ctx->stats.preemptive_launches = 0;
+  ctx->stats.prefetches = 0;
+  ctx->stats.graph_h2d_bytes = 0;
+  ctx->stats.run_ms = 0;
+  ctx->stats.chunks_free_min = num_chunks;
+  ctx->stats.spilled_chunks = 0;
+  ctx->stats.reloaded_chunks = 0;
+  ctx->stats.spill_d2h_bytes = 0;
+  ctx->stats.spill_h2d_bytes = 0;
+  ctx->stats.host_chunks_peak = 0;
+  ctx->stats.load_ms = 0;
+  ctx->stats.spill_xfer_ms = 0;
+  ctx->stats.host_syncs = 0;
+  ctx->load_ev.n = 0;
+  ctx->xfer_ev.n = 0;
+  ctx->nev = 0;
+  // walk spill (lt_config.walk_spill): every walk exists from lt_run's start; the pool of num_chunks
+  // chunks evicts to a pinned host store of one slot per chunk the W walks can fill (+ partial chunks)
+  {
+    lt::Spill& sp = ctx->spill;
+    sp.on = ctx->cfg.walk_spill == 1 && cap < W;
+    if (sp.on) {
+      const uint64_t host_cap = (W + C - 1) / C + ctx->nb + 2;
+      if (sp.host_cap < host_cap) {
+        if (sp.xfer) CK(cudaStreamSynchronize(sp.xfer));
+        if (sp.h_store) cudaFreeHost(sp.h_store);
+        sp.h_store = nullptr;
+        sp.host_cap = 0;
+        CK(cudaHostAlloc((void**)&sp.h_store, host_cap * C * sizeof(uint4), cudaHostAllocPortable));
+        sp.host_cap = host_cap;
+      }
+      for (int b = 0; b < 2; ++b) {
+        CK(ensure(sp.d_stage[b], sp.stage_cap[b], (size_t)lt::kSpillBatch * C));
+        if (!sp.ev_ready[b]) CK(cudaEventCreateWithFlags(&sp.ev_ready[b], cudaEventDisableTiming));
+        if (!sp.ev_free[b]) CK(cudaEventCreateWithFlags(&sp.ev_free[b], cudaEventDisableTiming));
+      }
+      if (!sp.xfer) CK(cudaStreamCreateWithFlags(&sp.xfer, cudaStreamNonBlocking));
+      if (sp.used[0] || sp.used[1]) CK(cudaStreamSynchronize(sp.xfer));  // the previous epoch's transfers
+      sp.used[0] = sp.used[1] = false;
+      sp.next = 0;
+      sp.spilled.assign(ctx->nb, {});
+      sp.host_free.resize(sp.host_cap);
+      for (uint64_t i = 0; i < sp.host_cap; ++i) sp.host_free[i] = (uint32_t)(sp.host_cap - 1 - i);
+      sp.host_used = 0;
+      sp.free_chunks = (int64_t)num_chunks;
+    }
+  }
   CK(cudaEventRecord(ctx->ev_a, s));
   ctx->snap_valid = false;
   CK(lt::launch_pool_reset(p, s));
@@ -642,7 +715,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   else if (ctx->cfg.visit_counts) CK(cudaMemsetAsync(ctx->d_visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
-  if (W && ctx->world > 1) CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
+  // (path_mode 2 stores no rows: d_paths is a placeholder of 8 entries and there is nothing to merge)
+  if (W && ctx->world > 1 && ctx->cfg.path_mode != 2)
+    CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
   ctx->adm_starts = d_starts;
   ctx->cap_walks = cap;
   ctx->admitted = cap;
@@ -662,6 +737,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
 
 lt_status lt_run(lt_ctx* ctx) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  lt::Range rg("lt_run");
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "lt_run before lt_walks_init");
   if (ctx->ran && ctx->world == 1)
     return fail(LT_ERR_STATE, "lt_run already done for these walks; call lt_walks_init again");
@@ -673,21 +749,18 @@ lt_status lt_run(lt_ctx* ctx) {
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
     ctx->stats.init_ms = ms;
   }
-  ctx->stats.sweeps = 0;
-  ctx->stats.update_launches = 0;
-  ctx->stats.update_ms = 0;
-  ctx->stats.iterations = 0;
-  ctx->stats.explicit_copies = 0;
-  ctx->stats.pool_hits = 0;
-  ctx->stats.zero_copy_launches = 0;
-  ctx->stats.preemptive_launches = 0;
-  ctx->stats.prefetches = 0;
-  ctx->stats.graph_h2d_bytes = 0;
-  ctx->stats.chunks_free_min = ctx->stats.chunks_total;
-  ctx->nev = 0;
+  // (update launches recorded since the last lt_run — e.g. by lt_superstep_p2p — stay in events[0, nev)
+  // and are summed below; the per-epoch counters were reset by lt_walks_init)
   CK(cudaEventRecord(ctx->ev_a, s));
-  lt_status st = ctx->ooc.on ? lt::run_out_of_core(ctx) : lt::run_resident(ctx);
+  lt_status st = LT_OK;
+  if (ctx->spill.on && !ctx->ran) st = lt::spill_admit_all(ctx);  // walk spill: every walk exists from here on
   if (st != LT_OK) return st;
+  st = ctx->ooc.on ? lt::run_out_of_core(ctx) : lt::run_resident(ctx);
+  if (st != LT_OK) return st;
+  if (ctx->spill.on) {
+    for (const auto& m : ctx->spill.spilled)
+      if (!m.empty()) return fail(LT_ERR_CUDA, "walk spill: evicted chunks left behind (invariant violated)");
+  }
   // Path rows hold entries 0..length-1; the 0xFFFFFFFF padding of the rest is output formatting and is
   // written lazily by the first copy-out (ensure_padded). With ownership the rows were pre-filled.
   ctx->padded = ctx->world > 1;
@@ -702,13 +775,21 @@ lt_status lt_run(lt_ctx* ctx) {
   {
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, ctx->ev_a, ctx->ev_b));
-    ctx->stats.run_ms = ms;
+    ctx->stats.run_ms += ms;
     double tot = 0;
     for (size_t i = 0; i + 1 < ctx->nev; i += 2) {
       CK(cudaEventElapsedTime(&ms, ctx->events[i], ctx->events[i + 1]));
       tot += ms;
     }
-    ctx->stats.update_ms = tot;
+    ctx->stats.update_ms += tot;
+    ctx->nev = 0;
+    double t = 0;
+    if (ctx->ooc.load_stream) CK(cudaStreamSynchronize(ctx->ooc.load_stream));
+    CK(ctx->load_ev.total_ms(&t));
+    ctx->stats.load_ms += t;
+    if (ctx->spill.xfer) CK(cudaStreamSynchronize(ctx->spill.xfer));
+    CK(ctx->xfer_ev.total_ms(&t));
+    ctx->stats.spill_xfer_ms += t;
   }
   ctx->stats.steps = ctx->h_ctr->steps;
   ctx->stats.visits = ctx->h_ctr->visits;
@@ -870,7 +951,10 @@ lt_status lt_get_pool_state(lt_ctx* ctx, lt_pool_state* out) {
   if (ctx->W) CK(cudaMemcpy(len.data(), ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToHost));
   out->free_chunks = small[0];
   out->total_chunks = p.pool.num_chunks;
-  for (uint32_t r : ring) out->ring_chunks += (r != lt::kEmpty);
+  for (uint32_t r : ring) {
+    out->ring_chunks += (r != lt::kEmpty && r != lt::kSpilled);
+    out->host_chunks += (r == lt::kSpilled);
+  }
   for (uint32_t k = 0; k < ctx->nb; ++k) out->pending += hc[ctx->nb + k] - hc[k];
   if (ctx->ran) out->finished = ctx->W;  // every walk terminated
   else for (uint32_t l : len) out->finished += (l != 0 && l != lt::kEmpty);
@@ -961,6 +1045,26 @@ lt_status lt_exchange_attach(lt_ctx* ctx, void* const* recv, void* const* cursor
   if (recv[ctx->rank] != ctx->d_xbuf[0] || recv[R + ctx->rank] != ctx->d_xbuf[1])
     return fail(LT_ERR_INVALID, "the table's entry for this rank must be this rank's own buffers");
   CK(cudaSetDevice(ctx->cfg.device));
+  // Peer buffers on another device of this process (threads driving several GPUs): the update kernels'
+  // atomics and stores into them need peer access from this context's device (IPC-opened buffers
+  // already map with cudaIpcMemLazyEnablePeerAccess).
+  for (uint32_t i = 0; i < 2 * R; ++i) {
+    for (const void* q : {static_cast<const void*>(recv[i]), static_cast<const void*>(cursor[i])}) {
+      cudaPointerAttributes a{};
+      CK(cudaPointerGetAttributes(&a, q));
+      if (a.type != cudaMemoryTypeDevice)
+        return fail(LT_ERR_INVALID, "peer buffers and cursors must be device memory");
+      if (a.device == ctx->cfg.device) continue;
+      int can = 0;
+      CK(cudaDeviceCanAccessPeer(&can, ctx->cfg.device, a.device));
+      if (!can)
+        return fail(LT_ERR_INVALID, "device " + std::to_string(ctx->cfg.device) + " cannot access peer device " +
+                                        std::to_string(a.device));
+      const cudaError_t e = cudaDeviceEnablePeerAccess(a.device, 0);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) (void)cudaGetLastError();
+      else CK(e);
+    }
+  }
   if (!ctx->d_peer_recv) CK(cudaMalloc(&ctx->d_peer_recv, 2 * R * sizeof(uint4*)));
   if (!ctx->d_peer_cur) CK(cudaMalloc(&ctx->d_peer_cur, 2 * R * sizeof(unsigned long long*)));
   CK(cudaMemcpy(ctx->d_peer_recv, recv, 2 * R * sizeof(void*), cudaMemcpyHostToDevice));

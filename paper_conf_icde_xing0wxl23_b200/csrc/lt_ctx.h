@@ -4,6 +4,7 @@
 #include "lt_internal.h"
 
 #include <algorithm>
+#include <map>
 #include <string>
 #include <vector>
 
@@ -46,6 +47,71 @@ struct OutOfCore {
   std::vector<uint32_t> table;
 };
 
+// Walk spill (lt_config.walk_spill): the walk pool keeps at most its
+// num_chunks chunks on the device; full chunks of buckets with the fewest pending walks are evicted to a
+// pinned host store (PAPER.md:118 "evict a batch when full", :202 "the same way") and loaded back before
+// their partition is computed. Transfers run on `xfer` through two staging buffers of kSpillBatch chunks.
+struct Spill {
+  bool on = false;
+  uint4* h_store = nullptr;                 // pinned host chunk slots (host_cap x C records)
+  uint64_t host_cap = 0;
+  std::vector<uint32_t> host_free;          // free host slots
+  std::vector<std::map<uint64_t, uint32_t>> spilled;  // per bucket: chunk index -> host slot
+  uint64_t host_used = 0;
+  uint4* d_stage[2] = {nullptr, nullptr};
+  size_t stage_cap[2] = {0, 0};
+  cudaStream_t xfer = nullptr;
+  cudaEvent_t ev_ready[2] = {nullptr, nullptr};  // stage b's contents are complete (recorded by its producer)
+  cudaEvent_t ev_free[2] = {nullptr, nullptr};   // stage b may be overwritten (recorded by its consumer)
+  bool used[2] = {false, false};
+  int next = 0;
+  int64_t free_chunks = 0;                  // host mirror of the device free stack, kept exact between snapshots
+};
+
+// Per-phase timing ("update vs reshuffle vs loading"): CUDA-event pairs
+// around the transfers of a phase on its own stream, summed at the end of lt_run (with lt_config.timing).
+struct PhaseEvents {
+  std::vector<cudaEvent_t> ev;
+  size_t n = 0;  // events in use (pairs)
+  cudaError_t begin(cudaStream_t s) {
+    while (ev.size() < n + 2) {
+      cudaEvent_t e;
+      cudaError_t r = cudaEventCreate(&e);
+      if (r != cudaSuccess) return r;
+      ev.push_back(e);
+    }
+    return cudaEventRecord(ev[n], s);
+  }
+  cudaError_t end(cudaStream_t s) {
+    cudaError_t r = cudaEventRecord(ev[n + 1], s);
+    n += 2;
+    return r;
+  }
+  cudaError_t total_ms(double* out) {  // sums and resets
+    double t = 0;
+    for (size_t i = 0; i + 1 < n; i += 2) {
+      float ms = 0;
+      cudaError_t r = cudaEventElapsedTime(&ms, ev[i], ev[i + 1]);
+      if (r != cudaSuccess) return r;
+      t += ms;
+    }
+    n = 0;
+    *out = t;
+    return cudaSuccess;
+  }
+  void destroy() {
+    for (auto e : ev) cudaEventDestroy(e);
+    ev.clear();
+    n = 0;
+  }
+};
+
+// NVTX ranges around the scheduler's phases (header-only NVTX3; a profiler shows them, free otherwise)
+struct Range {
+  explicit Range(const char* name);
+  ~Range();
+};
+
 }  // namespace lt
 
 struct lt_ctx {
@@ -74,6 +140,8 @@ struct lt_ctx {
   uint32_t* d_bounds = nullptr;
   size_t bounds_cap = 0;
   lt::OutOfCore ooc;
+  lt::Spill spill;
+  lt::PhaseEvents load_ev, xfer_ev;  // graph loads (load stream), walk-spill transfers (spill stream)
   // walks
   bool walks_ready = false;
   bool ran = false;
@@ -165,4 +233,7 @@ lt_status run_out_of_core(lt_ctx* ctx);
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound);
 // admit walks while live < cap_walks (returns true in *did if any were admitted)
 lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did);
+// walk spill: create every remaining walk, evicting chunks as the pool fills (lt_run's first step)
+lt_status spill_admit_all(lt_ctx* ctx);
+void free_spill(lt_ctx* ctx);
 }  // namespace lt

@@ -10,6 +10,7 @@ constexpr uint32_t kEmpty = 0xFFFFFFFFu;   // empty ring slot / unused path slot
 constexpr uint32_t kErrOOM = 1u;           // device error bits
 constexpr uint32_t kErrRing = 2u;
 constexpr uint32_t kErrPeer = 4u;          // a peer receive buffer overflowed
+constexpr uint32_t kSpilled = 0xFFFFFFFEu; // ring slot of a chunk evicted to host memory (walk spill)
 
 // A walk record (D5): 16 bytes, one 128-bit load/store.
 //   x = local walk index (row of the path matrix; walk_id = first_walk_id + x)
@@ -117,7 +118,15 @@ struct Params {
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;
-  uint32_t refill;  // 1: lane-refill update kernel (k_update_rf)
+  uint32_t refill;  // 0: batch kernel (k_update), 1: lane refill (k_update_rf), 3: warp-specialised (k_update_ws)
+  unsigned long long tail_cap;  // an update launch consumes [head, min(cursor, tail_cap)) (walk spill); ~0 otherwise
+};
+
+// Walk spill (lt_config.walk_spill): chunks moved between the device pool and host memory per launch.
+constexpr uint32_t kSpillBatch = 64;
+struct SpillList {
+  uint32_t bucket[kSpillBatch];
+  unsigned long long chunk[kSpillBatch];  // chunk index within the bucket (position / C)
 };
 
 // launchers (lt_kernels.cu); all asynchronous on `s`
@@ -139,6 +148,9 @@ cudaError_t launch_compact_rows(const uint32_t* paths, const uint32_t* lengths, 
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
+// walk spill: chunks list[0..count) -> stage (ring slots marked kSpilled, chunks freed) / stage -> fresh chunks
+cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* stage, cudaStream_t s);
+cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* stage, cudaStream_t s);
 // compact path output: (1) tile sums + their exclusive scan (total -> *total); (2) offsets[i] = base +
 // exclusive prefix of lengths for i < n, rows packed into vertices (indexed from 0 for this range)
 uint64_t paths_scan_tiles(uint64_t n);  // tile_sum entries launch_paths_scan needs
@@ -155,7 +167,9 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
                              cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
                                cudaStream_t s);
-int update_kernel_occupancy(uint32_t block, uint32_t ilp, bool refill, uint32_t app);  // resident blocks per SM (update kernel)
+// resident blocks per SM of the update kernel the launch uses (refill: 0 batch, 1 lane refill, 3 warp-specialised)
+int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill, uint32_t app, uint32_t P);
+constexpr uint32_t kWsMinChunk = 256;  // the warp-specialised kernel claims 256 positions at a time (<= C)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

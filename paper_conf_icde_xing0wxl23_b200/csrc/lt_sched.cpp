@@ -14,6 +14,8 @@
 // and a partition is computed only after its load finished (:208).
 #include "lt_ctx.h"
 
+#include <nvtx3/nvToolsExt.h>
+
 #include <cstring>
 
 namespace lt {
@@ -38,7 +40,12 @@ bool event_done(cudaEvent_t e) {
 
 }  // namespace
 
+Range::Range(const char* name) { nvtxRangePushA(name); }
+Range::~Range() { nvtxRangePop(); }
+
 lt_status snapshot(lt_ctx* ctx) {
+  Range r("lt snapshot (host round trip)");
+  ctx->stats.host_syncs++;
   unsigned long long* dh = nullptr;
   Counters* dc = nullptr;
   int* df = nullptr;
@@ -75,6 +82,219 @@ lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did) {
   return LT_OK;
 }
 
+// ------------------------------------------------------------------------------- walk spill (f3)
+// The walk pool evicts whole chunks to pinned host memory when it is full and loads a partition's
+// evicted chunks back before that partition is computed (reading R17:
+// the chunks of the buckets with the fewest pending walks go first). Chunk c of bucket q may be evicted
+// only when it lies wholly inside [head_q, cursor_q) — full and never written again (appends go to the
+// cursor's chunk or later) — and q is not being launched; its ring slot then holds kSpilled and its
+// device chunk is free. A launch of partition k consumes [head_k, tail_cap): every chunk there is on the
+// device (tail_cap = the start of k's first chunk still on the host, or the prefix the free chunks can
+// absorb). Eviction: k_spill (compute stream) copies the chunks into a staging buffer, the D2H to their
+// host slots runs on the transfer stream. Reload: H2D into a staging buffer on the transfer stream, then
+// k_reload installs fresh device chunks. Two staging buffers alternate; events order their reuse.
+namespace {
+
+// The writer stream of stage b waits until its previous consumer is done with it.
+int stage_take(lt_ctx* ctx, cudaStream_t writer) {
+  Spill& sp = ctx->spill;
+  const int b = sp.next;
+  sp.next ^= 1;
+  if (sp.used[b]) cudaStreamWaitEvent(writer, sp.ev_free[b], 0);
+  sp.used[b] = true;
+  return b;
+}
+
+// chunks a launch over n walks may need for its appends: one per C walks plus a partial tail chunk
+// per destination bucket
+inline uint64_t append_chunks(const lt_ctx* ctx, uint64_t n) {
+  const uint64_t C = ctx->params.pool.C;
+  return (n + C - 1) / C + ctx->nb + 1;
+}
+
+// Evict up to `want` chunks of buckets other than `keep` (fewest pending walks first, highest chunk
+// index first). Uses the last snapshot's head/cursor. Returns the number evicted in *done.
+lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done) {
+  Range rg("lt walk spill: evict");
+  Spill& sp = ctx->spill;
+  const uint64_t C = ctx->params.pool.C;
+  const uint32_t nb = ctx->nb;
+  *done = 0;
+  if (!want) return LT_OK;
+  std::vector<uint32_t> order;
+  for (uint32_t q = 0; q < nb; ++q)
+    if ((int)q != keep && ctx->h_hc[nb + q] > ctx->h_hc[q]) order.push_back(q);
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
+    return ctx->h_hc[nb + a] - ctx->h_hc[a] < ctx->h_hc[nb + b] - ctx->h_hc[b];
+  });
+  SpillList list;
+  uint32_t cnt = 0;
+  auto flush = [&]() -> lt_status {
+    if (!cnt) return LT_OK;
+    const cudaStream_t s = ctx->stream;
+    const int b = stage_take(ctx, s);
+    CK(launch_spill(ctx->params, list, cnt, sp.d_stage[b], s));
+    CK(cudaEventRecord(sp.ev_ready[b], s));
+    CK(cudaStreamWaitEvent(sp.xfer, sp.ev_ready[b], 0));
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer));
+    for (uint32_t i = 0; i < cnt; ++i) {
+      const uint32_t slot = sp.host_free.back();
+      sp.host_free.pop_back();
+      CK(cudaMemcpyAsync(sp.h_store + (uint64_t)slot * C, sp.d_stage[b] + (uint64_t)i * C, C * sizeof(uint4),
+                         cudaMemcpyDeviceToHost, sp.xfer));
+      sp.spilled[list.bucket[i]][list.chunk[i]] = slot;
+    }
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer));
+    CK(cudaEventRecord(sp.ev_free[b], sp.xfer));
+    sp.host_used += cnt;
+    sp.free_chunks += cnt;
+    ctx->stats.spilled_chunks += cnt;
+    ctx->stats.spill_d2h_bytes += (uint64_t)cnt * C * sizeof(uint4);
+    ctx->stats.host_chunks_peak = std::max<uint64_t>(ctx->stats.host_chunks_peak, sp.host_used);
+    ctx->stats.kernel_launches++;
+    ctx->snap_valid = false;
+    cnt = 0;
+    return LT_OK;
+  };
+  for (uint32_t q : order) {
+    const uint64_t head = ctx->h_hc[q], cur = ctx->h_hc[nb + q];
+    const uint64_t lo = (head + C - 1) / C;  // first chunk wholly at or after head
+    const uint64_t hi = cur / C;             // chunks [lo, hi) end at or before cursor
+    for (uint64_t ci = hi; ci-- > lo && *done < want;) {
+      if (sp.spilled[q].count(ci)) continue;
+      if (sp.host_free.empty()) return fail(LT_ERR_OOM, "walk spill: host store full (invariant violated)");
+      list.bucket[cnt] = q;
+      list.chunk[cnt] = ci;
+      ++*done;
+      if (++cnt == kSpillBatch) {
+        lt_status st = flush();
+        if (st != LT_OK) return st;
+      }
+    }
+    if (*done >= want) break;
+  }
+  return flush();
+}
+
+// Load the first r evicted chunks of bucket k (lowest chunk index first) back into device chunks.
+lt_status reload_chunks(lt_ctx* ctx, uint32_t k, uint64_t r) {
+  Range rg("lt walk spill: reload");
+  Spill& sp = ctx->spill;
+  const uint64_t C = ctx->params.pool.C;
+  auto& sk = sp.spilled[k];
+  while (r) {
+    SpillList list;
+    uint32_t cnt = 0;
+    const int b = stage_take(ctx, sp.xfer);
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer));
+    for (auto it = sk.begin(); it != sk.end() && cnt < kSpillBatch && cnt < r;) {
+      list.bucket[cnt] = k;
+      list.chunk[cnt] = it->first;
+      CK(cudaMemcpyAsync(sp.d_stage[b] + (uint64_t)cnt * C, sp.h_store + (uint64_t)it->second * C, C * sizeof(uint4),
+                         cudaMemcpyHostToDevice, sp.xfer));
+      sp.host_free.push_back(it->second);  // later D2H into this slot are ordered after this H2D (same stream)
+      it = sk.erase(it);
+      ++cnt;
+    }
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer));
+    CK(cudaEventRecord(sp.ev_ready[b], sp.xfer));
+    CK(cudaStreamWaitEvent(ctx->stream, sp.ev_ready[b], 0));
+    CK(launch_reload(ctx->params, list, cnt, sp.d_stage[b], ctx->stream));
+    CK(cudaEventRecord(sp.ev_free[b], ctx->stream));
+    sp.host_used -= cnt;
+    sp.free_chunks -= cnt;
+    ctx->stats.reloaded_chunks += cnt;
+    ctx->stats.spill_h2d_bytes += (uint64_t)cnt * C * sizeof(uint4);
+    ctx->stats.kernel_launches++;
+    ctx->snap_valid = false;
+    r -= cnt;
+  }
+  return LT_OK;
+}
+
+// Before a launch of partition k: make [head_k, tail_cap) device-resident and leave enough free chunks
+// for the launch's appends, evicting other buckets' chunks as needed. *tail_cap = ~0 when all of k fits.
+lt_status ensure_walks(lt_ctx* ctx, uint32_t k, unsigned long long* tail_cap) {
+  Spill& sp = ctx->spill;
+  *tail_cap = ~0ull;
+  lt_status st = snapshot(ctx);
+  if (st != LT_OK) return st;
+  sp.free_chunks = std::max(*ctx->h_free, 0);
+  const uint64_t C = ctx->params.pool.C;
+  const uint64_t head = ctx->h_hc[k], cur = ctx->h_hc[ctx->nb + k];
+  auto& sk = sp.spilled[k];
+  // walks a launch would cover after reloading the first r evicted chunks of k
+  auto covered = [&](uint64_t r) -> uint64_t {
+    if (r >= sk.size()) return cur - head;
+    auto it = sk.begin();
+    std::advance(it, (long)r);
+    return it->first * C - head;
+  };
+  const uint64_t all = sk.size();
+  const int64_t want_free = (int64_t)(all + append_chunks(ctx, cur - head));
+  if (sp.free_chunks < want_free) {
+    uint64_t done = 0;
+    st = evict_chunks(ctx, (int)k, (uint64_t)(want_free - sp.free_chunks), &done);
+    if (st != LT_OK) return st;
+  }
+  uint64_t r = all;
+  while (r > 0 && sp.free_chunks - (int64_t)r < (int64_t)append_chunks(ctx, covered(r))) --r;
+  st = reload_chunks(ctx, k, r);
+  if (st != LT_OK) return st;
+  // the launch stops at k's first chunk still on the host, or earlier if the free chunks cannot absorb
+  // the appends of every device-resident walk before it
+  unsigned long long cap = sk.empty() ? ~0ull : sk.begin()->first * C;
+  const int64_t room = sp.free_chunks - (int64_t)ctx->nb - 1;  // chunks left for full chunks of appends
+  if (room < 1) return fail(LT_ERR_OOM, "walk spill: the walk pool cannot hold one chunk of appends; raise walk_pool_walks");
+  const unsigned long long fit = head + (unsigned long long)room * C;
+  if (fit < std::min<unsigned long long>(cap, cur)) cap = fit;
+  if (cap <= head) return fail(LT_ERR_OOM, "walk spill: no walk of the selected partition fits the walk pool");
+  *tail_cap = cap;
+  return LT_OK;
+}
+
+}  // namespace
+
+lt_status spill_admit_all(lt_ctx* ctx) {
+  Spill& sp = ctx->spill;
+  const uint64_t C = ctx->params.pool.C;
+  const uint64_t batch = std::max<uint64_t>(C, ctx->cap_walks / 2);
+  while (ctx->admitted < ctx->W) {
+    lt_status st = snapshot(ctx);
+    if (st != LT_OK) return st;
+    sp.free_chunks = std::max(*ctx->h_free, 0);
+    const uint64_t n0 = std::min<uint64_t>(batch, ctx->W - ctx->admitted);
+    const int64_t need = (int64_t)append_chunks(ctx, n0);  // a k_init of n walks appends like a launch
+    if (sp.free_chunks < need) {
+      uint64_t done = 0;
+      st = evict_chunks(ctx, -1, (uint64_t)(need - sp.free_chunks), &done);
+      if (st != LT_OK) return st;
+    }
+    const int64_t room = sp.free_chunks - (int64_t)ctx->nb - 1;
+    if (room < 1) return fail(LT_ERR_OOM, "walk spill: the walk pool cannot hold one chunk of new walks");
+    const uint64_t n = std::min<uint64_t>(n0, (uint64_t)room * C);
+    ctx->snap_valid = false;
+    CK(launch_init(ctx->params, ctx->adm_starts + ctx->admitted, n, ctx->admitted, ctx->stream));
+    ctx->admitted += n;
+    ctx->stats.admissions++;
+    ctx->stats.kernel_launches++;
+  }
+  return LT_OK;
+}
+
+void free_spill(lt_ctx* ctx) {
+  Spill& sp = ctx->spill;
+  if (sp.xfer) cudaStreamSynchronize(sp.xfer);
+  if (sp.h_store) cudaFreeHost(sp.h_store);
+  for (int b = 0; b < 2; ++b) {
+    if (sp.d_stage[b]) cudaFree(sp.d_stage[b]);
+    if (sp.ev_ready[b]) cudaEventDestroy(sp.ev_ready[b]);
+    if (sp.ev_free[b]) cudaEventDestroy(sp.ev_free[b]);
+  }
+  if (sp.xfer) cudaStreamDestroy(sp.xfer);
+  sp = Spill();
+}
+
 lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
   cudaStream_t s = ctx->stream;
   const uint64_t max_grid = (uint64_t)ctx->num_sms * ctx->occ;
@@ -89,6 +309,7 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
     CK(cudaEventRecord(ctx->events[ctx->nev], s));
   }
   ctx->snap_valid = false;
+  Range rg("lt update launch");
   CK(launch_update(p, k, (uint32_t)grid, ctx->block, s));
   if (ctx->cfg.timing) {
     CK(cudaEventRecord(ctx->events[ctx->nev + 1], s));
@@ -99,7 +320,28 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
   return LT_OK;
 }
 
+// One partition's update launch; with walk spill, as many launches as it takes to consume every walk
+// that was in bucket k when the call began (each preceded by ensure_walks).
+lt_status launch_partition(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
+  if (!ctx->spill.on) return launch_update_timed(ctx, p, k, walks_bound);
+  Params pv = p;
+  unsigned long long end = 0;
+  for (bool first = true;; first = false) {
+    unsigned long long cap = ~0ull;
+    lt_status st = ensure_walks(ctx, k, &cap);
+    if (st != LT_OK) return st;
+    const unsigned long long head = ctx->h_hc[k], cur = ctx->h_hc[ctx->nb + k];
+    if (first) end = cur;
+    if (head >= end || head >= cur) return LT_OK;
+    pv.tail_cap = cap;
+    st = launch_update_timed(ctx, pv, k, std::min<unsigned long long>(cap, cur) - head);
+    if (st != LT_OK) return st;
+    if (cap >= cur) return LT_OK;
+  }
+}
+
 lt_status run_resident(lt_ctx* ctx) {
+  Range rg("lt run (HBM-resident scheduler)");
   const uint64_t max_len = (ctx->app == LT_APP_PPR) ? ctx->lmax : ctx->length;
   std::vector<uint32_t> order;
   order.reserve(ctx->P);
@@ -129,7 +371,7 @@ lt_status run_resident(lt_ctx* ctx) {
       // walks present at launch time <= pending now + everything launched before in this sweep
       const uint64_t bound = pending(ctx, k) + earlier;
       earlier += pending(ctx, k);
-      st = launch_update_timed(ctx, ctx->params, k, bound);
+      st = launch_partition(ctx, ctx->params, k, bound);
       if (st != LT_OK) return st;
     }
     ctx->stats.sweeps++;
@@ -210,9 +452,12 @@ lt_status load_partition(lt_ctx* ctx, uint32_t k, int b, uint64_t seq) {
     CK(cudaEventRecord(o.ev_used[b], ctx->stream));  // after every launch that could read the block
   }
   CK(cudaStreamWaitEvent(o.load_stream, o.ev_used[b], 0));  // the block's last reader is done
+  Range rg("lt load partition (H2D)");
+  if (ctx->cfg.timing) CK(ctx->load_ev.begin(o.load_stream));
   CK(cudaMemcpyAsync(base, o.h_row_ptr + v0, 8ull * (v1 - v0 + 1), cudaMemcpyHostToDevice, o.load_stream));
   if (e1 > e0)
     CK(cudaMemcpyAsync(base + o.rp_bytes, o.h_col + e0, 4ull * (e1 - e0), cudaMemcpyHostToDevice, o.load_stream));
+  if (ctx->cfg.timing) CK(ctx->load_ev.end(o.load_stream));
   CK(cudaEventRecord(o.ev_ready[b], o.load_stream));
   if (o.part_in[b] >= 0) o.block_of[o.part_in[b]] = -1;
   o.part_in[b] = (int)k;
@@ -230,7 +475,7 @@ lt_status compute_block(lt_ctx* ctx, uint32_t k) {
   CK(cudaStreamWaitEvent(ctx->stream, o.ev_ready[b], 0));
   lt_status st = table_publish(ctx, (int)k);
   if (st != LT_OK) return st;
-  st = launch_update_timed(ctx, view_block(ctx, k, b), k, pending(ctx, k));
+  st = launch_partition(ctx, view_block(ctx, k, b), k, pending(ctx, k));
   if (st != LT_OK) return st;
   CK(cudaEventRecord(o.ev_used[b], ctx->stream));
   return LT_OK;
@@ -280,6 +525,7 @@ lt_status prefetch(lt_ctx* ctx, uint32_t i, bool selective, uint64_t alpha, uint
 }  // namespace
 
 lt_status run_out_of_core(lt_ctx* ctx) {
+  Range rg("lt run (out-of-core scheduler)");
   OutOfCore& o = ctx->ooc;
   const uint32_t P = ctx->P;
   const uint32_t pol = ctx->cfg.policy;
@@ -327,7 +573,7 @@ lt_status run_out_of_core(lt_ctx* ctx) {
       ctx->stats.zero_copy_launches++;
       st = table_publish(ctx, -1);
       if (st != LT_OK) return st;
-      st = launch_update_timed(ctx, view_zero_copy(ctx), i, pending(ctx, i));
+      st = launch_partition(ctx, view_zero_copy(ctx), i, pending(ctx, i));
       if (st != LT_OK) return st;
       continue;
     }

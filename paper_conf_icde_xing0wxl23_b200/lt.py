@@ -64,7 +64,7 @@ class Config(ctypes.Structure):
         ("refill", ctypes.c_uint32),
         ("visit_counts", ctypes.c_uint32),
         ("continue_resident", ctypes.c_uint32),
-        ("reserved0", ctypes.c_uint32),
+        ("walk_spill", ctypes.c_uint32),
         ("walk_pool_walks", ctypes.c_uint64),
         ("direct_start", ctypes.c_uint32),
         ("l2_persist", ctypes.c_uint32),
@@ -79,11 +79,13 @@ class Stats(ctypes.Structure):
         ("graph_prep_ms", ctypes.c_double), ("layout", ctypes.c_uint32), ("out_of_core", ctypes.c_uint32)] + [
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
-            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes", "prefetches")]
+            "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes", "prefetches",
+            "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak")] + [
+        ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64)]
 
 
 class PoolState(ctypes.Structure):
-    _fields_ = [("free_chunks", ctypes.c_int64), ("ring_chunks", ctypes.c_uint64), ("reserved0", ctypes.c_uint64),
+    _fields_ = [("free_chunks", ctypes.c_int64), ("ring_chunks", ctypes.c_uint64), ("host_chunks", ctypes.c_uint64),
                 ("total_chunks", ctypes.c_uint64), ("pending", ctypes.c_uint64), ("finished", ctypes.c_uint64),
                 ("device_err", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
@@ -187,7 +189,8 @@ class Engine:
                  path_mode: int = 0, graph_pool_bytes: int = 0, zero_copy: bool = False,
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
                  visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
-                 direct_start: bool = True, l2_persist: int = 0, ooc_prefetch: bool = False):
+                 direct_start: bool = True, l2_persist: int = 0, ooc_prefetch: bool = False,
+                 walk_spill: bool = False):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -211,6 +214,7 @@ class Engine:
         cfg.refill = refill
         cfg.continue_resident = int(bool(continue_resident))
         cfg.walk_pool_walks = int(walk_pool_walks)
+        cfg.walk_spill = int(bool(walk_spill))
         cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
         cfg.l2_persist = int(l2_persist)
         cfg.ooc_prefetch = int(bool(ooc_prefetch))

@@ -62,3 +62,20 @@ def test_cuda_arm_line():
     assert d["gpu_launches"] > 0
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
     assert d["parity_sample"]["mismatched_walks"] == 0
+
+
+def test_gpus_n_without_torchrun_launches_ranks():
+    """`bench.py --gpus 2` outside torchrun re-launches itself with one process per GPU (the driver's
+    launch line): one JSON line from rank 0 with n_gpus == 2, not a silent single-GPU run."""
+    lines = _run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--config", "1", "--steps", "1",
+                  "--warmup", "3"])
+    assert len(lines) == 1 and lines[0]["n_gpus"] == 2
+
+
+def test_world_size_must_match_gpus():
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29533", "bench.py", "--impl", "reference",
+                        "--gpus", "3", "--config", "1", "--steps", "1", "--warmup", "3"],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode != 0 and "WORLD_SIZE" in r.stderr

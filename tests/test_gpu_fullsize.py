@@ -1,7 +1,8 @@
 """Full-size parity: BASELINE.json configs[3] (FS-shaped, the bench workload) and configs[2]
 (TW-shaped PPR) at their full sizes, in the launch configuration bench.py times (library defaults,
-P = 1, layout auto). The oracle recomputes a spread sample of walks one by one; properties that hold
-at any size are checked on every walk."""
+P = 1, layout auto). The oracle recomputes a spread sample of >= 1M walks one by one (plus, for PPR,
+every walk of length >= 40: the tail of the geometric law); properties that hold at any
+size are checked on every walk."""
 import numpy as np
 import pytest
 
@@ -17,7 +18,7 @@ def _host(g):
                            g.max_deg, g.argmax_deg)
 
 
-def _sample(W, k=40_000, seed=0):
+def _sample(W, k=1_000_000, seed=0):
     rng = np.random.default_rng(seed)
     idx = np.unique(np.concatenate([np.arange(min(W, 1000)), np.arange(max(0, W - 1000), W),
                                     rng.integers(0, W, size=k)]))
@@ -59,7 +60,7 @@ def test_cfg4_partitioned_csr_sampled(fs_graph):
     g = fs_graph
     W = g.n
     starts = lt_inputs.deepwalk_starts(W, g.n)
-    ids = _sample(W, k=10_000, seed=3)
+    ids = _sample(W, k=1_000_000, seed=3)
     with LT.Engine(layout=LT.LAYOUT_CSR) as e:
         e.graph_load(g.row_ptr, g.col, 16)
         e.walks_init(torch.from_numpy(starts.view(np.int32)).cuda(), LT.DEEPWALK, 80, 1)
@@ -83,9 +84,12 @@ def test_cfg3_tw_shaped_ppr_full_size(gpu):
         e.walks_init(torch.from_numpy(starts.view(np.int32)).cuda(), LT.PPR, 0.15, 1)
         e.run()
         st = e.stats()
-        ids = _sample(W)
-        gp, gl = e.get_paths_rows(ids)
         _, lengths = e.get_paths(paths=False)
+        # a spread sample plus the whole tail: every walk with >= 40 path vertices (about 0.85^39 of W)
+        tail = np.nonzero(lengths >= 40)[0].astype(np.uint64)
+        assert len(tail) > 10_000
+        ids = np.union1d(_sample(W), tail).astype(np.uint64)
+        gp, gl = e.get_paths_rows(ids)
     # geometric length law at full size: mean within 4 sigma of 1/alpha
     N = lengths.astype(np.float64)
     assert abs(N.mean() - 1 / 0.15) < 4 * np.sqrt(0.85 / 0.15 ** 2 / W)

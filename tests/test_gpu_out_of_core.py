@@ -163,3 +163,29 @@ def test_continue_resident_ppr_and_pagerank(gpu, g14, app, param):
     np.testing.assert_array_equal(lengths, ol)
     np.testing.assert_array_equal(paths, op)
     np.testing.assert_array_equal(counts, O.visit_counts(op, ol, g14.n))
+
+
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 20), (LT.PPR, 0.15)])
+def test_continue_zero_copy_small_chunks(gpu, g14, app, param):
+    """Continuation during zero-copy launches with tiny chunks (C = 64): a walk going i -> resident q -> i
+    is appended to bucket i while i's launch still consumes it, so the bucket's ring must hold twice the
+    walks (the ring was sized for one pass and an install could overwrite a live slot)."""
+    starts = (lt_inputs.deepwalk_starts(g14.n, g14.n) if app == LT.DEEPWALK
+              else lt_inputs.ppr_starts(20_000, g14.argmax_deg))
+    paths, lengths, st = run(g14, starts, app, param, 3, 16, 3, zero_copy=True, continue_resident=True,
+                             chunk_walks=64)
+    op, ol, osteps, _ = oracle_of(g14, starts, app, param, 3)
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)
+    assert st["zero_copy_launches"] > 0
+
+
+@pytest.mark.parametrize("zero_copy", [False, True])
+def test_out_of_core_warp_specialised_kernel(gpu, g14, zero_copy):
+    """Out of core without continuation on the warp-specialised kernel (refill 3): graph-pool block views
+    and the zero-copy view of the mapped host CSR (CSR layout, V records)."""
+    starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
+    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, 16, 3, zero_copy=zero_copy, refill=3, chunk_walks=512)
+    op, ol, _, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
+    np.testing.assert_array_equal(paths, op)
+    np.testing.assert_array_equal(lengths, ol)

@@ -325,6 +325,12 @@ def test_fused_superstep_exact(gpu, g13, world, layout, app, param):
             np.testing.assert_array_equal(paths, op)
         assert sum(out[r][i][3]["steps"] for r in range(world)) == osteps
         assert sum(out[r][i][2]["records_sent"] for r in range(world)) > 0
+        # per-epoch statistics accumulate over the supersteps (one update launch each; the final
+        # lt_run over the empty buckets launches none), so bytes / update_ms is the epoch's rate
+        for r in range(world):
+            st, cnt = out[r][i][3], out[r][i][2]
+            assert st["update_launches"] == cnt["supersteps"]
+            assert st["update_ms"] > 0 and st["run_ms"] > 0
 
 
 def test_fused_superstep_preconditions(gpu, g13):
@@ -368,3 +374,96 @@ def test_fused_superstep_overflow_is_an_error(gpu, g13):
     for t in th:
         t.join()
     assert errors and all("overflow" in str(x) for x in errors)
+
+
+@pytest.mark.parametrize("p2p", [False, True])
+def test_ownership_paths_off_visit_counts(gpu, g13, p2p):
+    """path_mode 2 (no path matrix, the paper's accounting) with range ownership: no path rows are
+    pre-filled or merged, the visit counts summed over ranks equal the oracle's (the
+    0xFF pre-fill once ran over the 8-entry placeholder)."""
+    import torch
+    world = 2
+    starts = lt_inputs.deepwalk_starts(2 * g13.n, g13.n)
+    hub = ltdist.ThreadComm.Hub(world)
+    out, errors = [None] * world, []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world, path_mode=2, visit_counts=True, chunk_walks=512) as e:
+                e.graph_load(g13.row_ptr, g13.col, 8)
+                e.walks_init_pagerank(starts, 12, 0.15, 9)
+                comm = ltdist.ThreadComm(hub, r)
+                if p2p:
+                    ltdist.attach_peers(e, comm, len(starts))
+                    cnt = ltdist.run_supersteps_p2p(e, comm, "cuda")
+                else:
+                    cnt = ltdist.run_supersteps(e, comm, "cuda")
+                counts = ltdist.merge_visit_counts(e, comm, "cuda")
+                torch.cuda.synchronize()
+                assert e.pool_state()["device_err"] == 0
+                out[r] = (counts.cpu().numpy().view(np.uint64), cnt, e.stats())
+        except Exception as ex:
+            errors.append(ex)
+            hub.barrier.abort()
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errors:
+        raise errors[0]
+    op, ol, osteps, _ = O.walks(g13.row_ptr, g13.col, starts, app=O.PAGERANK, length=12, alpha=0.15, seed=9)
+    expect = O.visit_counts(op, ol, g13.n)
+    for counts, cnt, st in out:
+        np.testing.assert_array_equal(counts, expect)
+    assert sum(st["steps"] for _, _, st in out) == osteps
+    assert all(st["update_launches"] >= 1 and st["update_ms"] > 0 for _, _, st in out)
+
+
+@pytest.mark.parametrize("exchange", ["alltoall", "p2p", "fused"])
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
+def test_ownership_warp_specialised_kernel(gpu, g13, exchange, layout):
+    """Range ownership on the warp-specialised kernel (refill 3): walks for other ranks leave as V
+    records (a receiver needs the vertex), through send buckets or straight into peer buffers."""
+    world = 3
+    starts = lt_inputs.deepwalk_starts(3 * g13.n, g13.n)
+    P = world if exchange == "fused" else 12
+    kw = dict(layout=layout, refill=3, chunk_walks=512)
+    if exchange == "alltoall":
+        res = run_owned(g13, starts, LT.DEEPWALK, 16, 2, P, world, **kw)
+    else:
+        res = run_owned_p2p(g13, starts, LT.DEEPWALK, 16, 2, P, world, **kw) if exchange == "p2p" else None
+    if exchange == "fused":
+        import torch
+        hub = ltdist.ThreadComm.Hub(world)
+        res, errors = [None] * world, []
+
+        def rank_main(r):
+            try:
+                with LT.Engine(rank=r, world=world, **kw) as e:
+                    e.graph_load(g13.row_ptr, g13.col, P)
+                    e.walks_init(starts, LT.DEEPWALK, 16, 2)
+                    comm = ltdist.ThreadComm(hub, r)
+                    ltdist.attach_peers(e, comm, len(starts))
+                    cnt = ltdist.run_supersteps_p2p_fused(e, comm, "cuda")
+                    paths, lengths = ltdist.merge_paths(e, comm)
+                    torch.cuda.synchronize()
+                    res[r] = (paths.cpu().numpy().view(np.uint32), lengths.cpu().numpy().view(np.uint32), cnt,
+                              e.stats())
+            except Exception as ex:
+                errors.append(ex)
+                hub.barrier.abort()
+
+        th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        if errors:
+            raise errors[0]
+    op, ol, osteps, _ = oracle_of(g13, starts, LT.DEEPWALK, 16, 2)
+    for paths, lengths, _, _ in res:
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+    assert sum(r[3]["steps"] for r in res) == osteps

@@ -228,12 +228,13 @@ def _cfg2():
     return _CFG2["g"]
 
 
-@pytest.mark.parametrize("P,chunk", [(1, 8192), (4, 64), (16, 256), (64, 64)])
-def test_pool_invariants(gpu, cfg1, P, chunk):
+@pytest.mark.parametrize("P,chunk,refill", [(1, 8192, 0), (4, 64, 0), (16, 256, 0), (64, 64, 0), (16, 256, 3),
+                                            (4, 1024, 3), (64, 512, 3)])
+def test_pool_invariants(gpu, cfg1, P, chunk, refill):
     """Conservation of walks and chunks (a6): after init every walk is pending in some bucket and
     every chunk is either free or installed; after the run nothing is pending and nothing leaked."""
     starts = lt_inputs.deepwalk_starts(4096, cfg1.n)
-    with LT.Engine(chunk_walks=chunk) as e:
+    with LT.Engine(chunk_walks=chunk, refill=refill) as e:
         e.graph_load(cfg1.row_ptr, cfg1.col, P)
         e.walks_init(starts, LT.DEEPWALK, 10, 1)
         s0 = e.pool_state()
@@ -249,7 +250,7 @@ def test_pool_invariants(gpu, cfg1, P, chunk):
 
 
 @pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
-@pytest.mark.parametrize("ilp,refill", [(1, 1), (2, 1), (4, 1), (1, 2)])
+@pytest.mark.parametrize("ilp,refill", [(1, 1), (2, 1), (4, 1), (1, 2), (1, 3)])
 @pytest.mark.parametrize("gather_mode", [0, 3])
 @pytest.mark.parametrize("P", [1, 8])
 def test_kernel_variants_exact(gpu, cfg1, layout, ilp, refill, gather_mode, P):
@@ -309,7 +310,7 @@ def test_layouts_memory_and_limits(gpu, cfg1):
 @pytest.mark.parametrize("path_mode", [0, 1])
 @pytest.mark.parametrize("P", [1, 3, 16])
 @pytest.mark.parametrize("length", [0, 1, 7, 8, 9, 15, 16, 17, 80])
-@pytest.mark.parametrize("refill", [1, 2])
+@pytest.mark.parametrize("refill", [1, 2, 3])
 def test_path_store_modes_and_sector_edges(gpu, cfg1, path_mode, P, length, refill):
     """Buffered full-sector path stores vs one store per step, at lengths around the 8-entry sector
     boundaries, with visits that start mid-sector (P > 1), with and without lane refill."""
@@ -472,3 +473,33 @@ def test_lemire_rejection_chain_at_degree_2_31_plus_1(gpu, layout):
     starts = np.zeros(20_000, dtype=np.uint32)
     assert_parity(g, starts, LT.DEEPWALK, 12, 3, P=1, layout=layout)
     assert_parity(g, starts, LT.PPR, 0.1, 4, P=3, layout=layout)
+
+
+@pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
+@pytest.mark.parametrize("P", [2, 16, 300])
+@pytest.mark.parametrize("chunk", [256, 8192])
+def test_warp_specialised_kernel_exact(gpu, layout, P, chunk):
+    """k_update_ws (refill 3): stepping warps with prefetched records, offset-carrying O records and a
+    CTA inserter warp draining a shared-memory departure ring. More walks than one CTA's ring holds
+    (the ring wraps, producers wait for the inserter), partitions from 2 to 300, chunk sizes at and
+    far above the 256-position claim, DeepWalk / PPR / PageRank; paths equal the oracle."""
+    g = lt_inputs.rmat_cpu(15, 16 * 2 ** 15, seed=4)
+    kw = dict(layout=layout, refill=3, chunk_walks=chunk)
+    st = assert_parity(g, lt_inputs.deepwalk_starts(3 * g.n, g.n), LT.DEEPWALK, 23, 5, P=P, **kw)
+    assert st["visits"] > 3 * g.n
+    assert_parity(g, lt_inputs.ppr_starts(50_000, g.argmax_deg), LT.PPR, 0.1, 6, P=P, **kw)
+    with LT.Engine(visit_counts=True, **kw) as e:
+        starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+        e.graph_load(g.row_ptr, g.col, P)
+        e.walks_init_pagerank(starts, 19, 0.2, 8)
+        e.run()
+        paths, lengths = e.get_paths()
+        counts = e.visit_counts()
+    op, ol, _, _ = O.walks(g.row_ptr, g.col, starts, app=O.PAGERANK, length=19, alpha=0.2, seed=8)
+    np.testing.assert_array_equal(paths, op)
+    np.testing.assert_array_equal(counts, O.visit_counts(op, ol, g.n))
+
+
+def test_warp_specialised_kernel_small_chunks_fall_back(gpu, cfg1):
+    """chunk_walks < 256 cannot hold a 256-position claim: refill 3 falls back to the batch kernel."""
+    assert_parity(cfg1, lt_inputs.deepwalk_starts(4096, cfg1.n), LT.DEEPWALK, 10, 1, P=4, refill=3, chunk_walks=64)

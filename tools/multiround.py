@@ -1,7 +1,11 @@
 #!/usr/bin/env python3
-"""SURVEY.md §8(f) f3 / PAPER.md:353-363 (Fig. 16): massive walk counts under a walk-pool cap, walk
-admission (lt_config.walk_pool_walks) against the multi-round baseline (the same walks in R sequential
-rounds of W/R, each a separate lt_walks_init + lt_run) with the same memory cap.
+"""SURVEY.md §8(f) f3 / PAPER.md:353-363 (Fig. 16): massive walk counts under a walk-pool cap. Three arms
+with the same device memory cap m_w on the walk pool:
+  * spill (lt_config.walk_spill, the paper's mechanism): every walk exists
+    from the start; full chunks of the buckets with the fewest walks are evicted to pinned host memory
+    and loaded back before their partition is computed;
+  * admission (lt_config.walk_pool_walks alone): walks are created in index order as walks end;
+  * multi-round baseline: the same walks in R sequential rounds of m_w (separate lt_walks_init + lt_run).
 
 Graph: BASELINE configs[3] (FS-shaped R-MAT s26), out of core (pinned host CSR, capped graph pool,
 adaptive zero copy, continuation into resident partitions). Walks: DeepWalk l = 10 (the paper's Fig. 15
@@ -29,6 +33,7 @@ def main():
     ap.add_argument("--partitions", type=int, default=64)
     ap.add_argument("--graph-pool-gb", type=float, default=8.0)
     ap.add_argument("--reps", type=int, default=1)
+    ap.add_argument("--arms", default="spill,admission,multi")
     a = ap.parse_args()
     import torch
     import paper_conf_icde_xing0wxl23_b200 as LT
@@ -39,9 +44,11 @@ def main():
     starts = torch.from_numpy(lt_inputs.deepwalk_starts(W, g.n).view(np.int32)).cuda()
     ooc = a.graph_pool_gb > 0
 
-    def engine(cap):
+    arms = a.arms.split(",")
+
+    def engine(cap, spill=False):
         return LT.Engine(path_mode=2, walk_pool_walks=cap, graph_pool_bytes=int(a.graph_pool_gb * 2 ** 30),
-                         zero_copy=True, continue_resident=True, timing=True)
+                         zero_copy=ooc, continue_resident=ooc, timing=True, walk_spill=spill)
 
     def timed(fn):
         torch.cuda.synchronize()
@@ -54,19 +61,41 @@ def main():
 
     for cap in [int(x) for x in a.caps.split(",")]:
         rounds = -(-W // cap)
-        # (1) walk admission: all W walks, at most `cap` live
-        with engine(cap) as e:
-            t0 = time.time()
-            e.graph_load(g.row_ptr, g.col, a.partitions)
-            load_s = time.time() - t0
+        line = {"what": "walk spill vs walk admission vs multi-round (PAPER.md:353-363, Fig. 16 shape)",
+                "graph": f"{c['name']} out-of-core P={a.partitions} pool={a.graph_pool_gb} GiB" if ooc
+                else f"{c['name']} HBM-resident P={a.partitions}",
+                "walks": W, "cap_walks": cap, "rounds": rounds, "length": a.length}
 
-            def adm():
-                e.walks_init(starts, LT.DEEPWALK, a.length, 1)
-                e.run()
-                return e.stats()
-            adm()  # warm-up
-            ms_adm, st = min((timed(adm) for _ in range(a.reps)), key=lambda x: x[0])
-        # (2) multi-round baseline: R rounds of `cap` walks (walk IDs continue across rounds)
+        def capped(spill):
+            with engine(cap, spill) as e:
+                e.graph_load(g.row_ptr, g.col, a.partitions)
+
+                def go():
+                    e.walks_init(starts, LT.DEEPWALK, a.length, 1)
+                    e.run()
+                    return e.stats()
+                go()  # warm-up
+                ms, st = min((timed(go) for _ in range(a.reps)), key=lambda x: x[0])
+            assert st["steps"] == W * a.length
+            out = {"ms": ms, "steps_per_s": st["steps"] / (ms / 1000), "admissions": st["admissions"],
+                   "peak_live": st["peak_live"], "graph_h2d_gb": st["graph_h2d_bytes"] / 1e9,
+                   "explicit_copies": st["explicit_copies"], "iterations": st["iterations"],
+                   "chunks_total": st["chunks_total"], "update_launches": st["update_launches"]}
+            if spill:
+                out.update(spilled_chunks=st["spilled_chunks"], reloaded_chunks=st["reloaded_chunks"],
+                           spill_d2h_gb=st["spill_d2h_bytes"] / 1e9, spill_h2d_gb=st["spill_h2d_bytes"] / 1e9,
+                           host_chunks_peak=st["host_chunks_peak"])
+            return out
+
+        # (1) walk spill (every walk exists; the pool evicts to host memory) and (2) walk admission
+        if "spill" in arms:
+            line["spill"] = capped(True)
+        if "admission" in arms:
+            line["admission"] = capped(False)
+        if "multi" not in arms:
+            print(json.dumps(line), flush=True)
+            continue
+        # (3) multi-round baseline: R rounds of `cap` walks (walk IDs continue across rounds)
         with engine(0) as e:
             e.graph_load(g.row_ptr, g.col, a.partitions)
 
@@ -82,18 +111,13 @@ def main():
                 return tot
             multi()
             ms_mr, mt = min((timed(multi) for _ in range(a.reps)), key=lambda x: x[0])
-        line = {"what": "walk admission vs multi-round (PAPER.md:353-363, Fig. 16 shape)",
-                "graph": f"{c['name']} out-of-core P={a.partitions} pool={a.graph_pool_gb} GiB" if ooc else c["name"],
-                "walks": W, "cap_walks": cap, "rounds": rounds, "length": a.length,
-                "admission": {"ms": ms_adm, "steps_per_s": st["steps"] / (ms_adm / 1000),
-                              "admissions": st["admissions"], "peak_live": st["peak_live"],
-                              "graph_h2d_gb": st["graph_h2d_bytes"] / 1e9, "explicit_copies": st["explicit_copies"],
-                              "iterations": st["iterations"], "chunks_total": st["chunks_total"]},
-                "multi_round": {"ms": ms_mr, "steps_per_s": mt["steps"] / (ms_mr / 1000),
-                                "graph_h2d_gb": mt["graph_h2d_bytes"] / 1e9, "explicit_copies": mt["explicit_copies"],
-                                "iterations": mt["iterations"]},
-                "multi_round_slowdown": ms_mr / ms_adm, "graph_load_s": round(load_s, 1)}
-        assert st["steps"] == mt["steps"] == W * a.length
+        line["multi_round"] = {"ms": ms_mr, "steps_per_s": mt["steps"] / (ms_mr / 1000),
+                               "graph_h2d_gb": mt["graph_h2d_bytes"] / 1e9, "explicit_copies": mt["explicit_copies"],
+                               "iterations": mt["iterations"]}
+        for arm in ("spill", "admission"):
+            if arm in line:
+                line[f"multi_round_slowdown_vs_{arm}"] = ms_mr / line[arm]["ms"]
+        assert mt["steps"] == W * a.length
         print(json.dumps(line), flush=True)
 
 
