@@ -50,7 +50,7 @@ $(PKG)/liblt.so: $(LT_CU:.cu=.o) $(LT_CPP:.cpp=.o)
 variant: $(LT_CPP:.cpp=.o)
 	mkdir -p tools/variants
 	$(NVCC) $(NVFLAGS) $(VDEFS) -Iinclude -c $(CSRC)/lt_kernels.cu -o tools/variants/lt_kernels_$(VTAG).o
-	$(NVCC) $(ARCH) -shared tools/variants/lt_kernels_$(VTAG).o $(LT_CPP:.cpp=.o) -o tools/variants/liblt_$(VTAG).so
+	$(NVCC) $(ARCH) -shared tools/variants/lt_kernels_$(VTAG).o $(LT_CPP:.cpp=.o) -o tools/variants/liblt_$(VTAG).so -ldl
 
 clean:
 	rm -f tools/gather_bench lt_inputs/*.o lt_inputs/*.so oracle/*.so $(CSRC)/*.o $(CSRC)/*.ptxas.txt $(PKG)/*.so

@@ -429,8 +429,10 @@ def main():
     def one_step():
         init_walks(eng, c, starts_d, args.seed, first)
         if p2p:
-            if not attached:  # receive buffers for every walk, shared once through CUDA IPC
-                ltdist.attach_peers(eng, comm, W)
+            if not attached:  # receive buffers for every walk, shared once through CUDA IPC; every rank
+                ltdist.attach_peers(eng, comm, W)  # writes its path entries into rank 0's matrix (no merge)
+                if args.path_mode == 0:
+                    ltdist.attach_paths(eng, comm)
                 attached.append(True)
             # one owned partition per rank, HBM-resident: the fused superstep (one host round trip each)
             fused = P == world and not ooc

@@ -120,10 +120,8 @@ typedef struct lt_config {
                                  partitions. Every partition must fit one block
                                  (block = the largest partition's CSR slice). */
   uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
-  uint32_t refill;            /* update kernel: 0 auto (lane refill when P == 1, the measured best),
-                                 1 the batch kernel, 2 lane refill, 3 the warp-specialised kernel (7
-                                 stepping warps with prefetched records + 1 inserting warp per CTA;
-                                 needs chunk_walks >= 256, else the batch kernel) */
+  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P <= 4, the measured
+                                 best), 1 off (the batch kernel), 2 on */
   uint32_t visit_counts;      /* 1 -> count per-vertex visit frequency ("the visit
                                  frequency of each vertex is recorded") into a u64[n] device array
                                  reserved at lt_walks_init* and zeroed there: every path entry (start
@@ -366,6 +364,23 @@ lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received);
  * lt_superstep_p2p -> sum of d_sent over ranks (a device all-reduce; 0 ends it) -> ..., then one
  * lt_run to finalise statistics and visit counts. */
 lt_status lt_superstep_p2p(lt_ctx* ctx, unsigned long long* d_sent);
+/* Paths on one rank (range ownership; "the merged result lands on rank 0"): every rank
+ * writes its path entries and lengths straight into the HOME rank's path matrix and length array over
+ * peer memory (NVLink; stores buffered into 32-B sectors as usual), so when the last superstep ends the
+ * home rank holds every walk's path — no cross-rank merge, and the other ranks keep no path matrix of
+ * their own from their next lt_walks_init on (the home's capacity is checked there).
+ * lt_paths_buffers (home rank, after its lt_walks_init): its matrix, length array and the matrix capacity
+ * in u32 entries, for sharing (CUDA IPC through lt_ipc_handle / lt_ipc_open across processes, the
+ * pointers themselves between threads). lt_paths_attach (every other rank): install the home's buffers,
+ * or NULL, NULL to write locally again; with path_mode 1 it must precede lt_walks_init (which stores
+ * path[w][0]), with path_mode 0 it may follow it. In the epoch of the first lt_paths_buffers call the
+ * home's lt_walks_init has pre-filled its matrix: every rank's writes must start after it (dist.py
+ * synchronises and barriers once). From then on the home's lt_walks_init neither pre-fills nor zeroes
+ * its matrix and lengths (every length is written once per epoch where the walk ends; rows are padded
+ * lazily by the first copy-out), so later epochs need no barrier. lt_get_paths* on an attached rank:
+ * LT_ERR_STATE. */
+lt_status lt_paths_buffers(lt_ctx* ctx, void** d_paths, void** d_lengths, uint64_t* capacity_entries);
+lt_status lt_paths_attach(lt_ctx* ctx, void* d_paths, void* d_lengths, uint64_t capacity_entries);
 /* CUDA IPC of a device allocation's base pointer (handle: 64 bytes), and opening another process's
  * handle on this context's device (closed at lt_destroy). */
 lt_status lt_ipc_handle(const void* dptr, void* handle);

@@ -55,7 +55,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.world == 0) c.world = 1;
   if (c.rank >= c.world || c.world > 65535) return fail(LT_ERR_INVALID, "need rank < world <= 65535");
   if (c.path_mode > 2) return fail(LT_ERR_INVALID, "bad path_mode");
-  if (c.refill > 3) return fail(LT_ERR_INVALID, "bad refill");
+  if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
   if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
   if (c.direct_start > 1) return fail(LT_ERR_INVALID, "direct_start must be 0 (auto) or 1 (off)");
   if (c.walk_spill > 1) return fail(LT_ERR_INVALID, "walk_spill must be 0 or 1");
@@ -559,8 +559,12 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const uint64_t num_chunks = 2 * wc + 2 * (uint64_t)ctx->nb + 64;
   if (num_chunks >= 0x7FFFFFFFull) return fail(LT_ERR_INVALID, "pool too large; raise chunk_walks");
   const uint32_t pitch = (stride + 7u) & ~7u;  // rows start on 32-B sectors
-  // path_mode 2 stores no path entries (the paper's accounting): no path matrix
-  CK(ensure(ctx->d_paths, ctx->paths_cap, ctx->cfg.path_mode == 2 ? 8 : std::max<uint64_t>(W, 1) * pitch));
+  // path_mode 2 stores no path entries (the paper's accounting): no path matrix. A rank
+  // whose paths go to a home rank (lt_paths_attach) keeps no matrix of its own either.
+  const bool home = ctx->home_paths != nullptr && ctx->world > 1 && ctx->cfg.path_mode != 2;
+  if (home && (uint64_t)W * pitch > ctx->home_cap)
+    return fail(LT_ERR_INVALID, "the home rank's path matrix is smaller than W x pitch; attach again");
+  CK(ensure(ctx->d_paths, ctx->paths_cap, (ctx->cfg.path_mode == 2 || home) ? 8 : std::max<uint64_t>(W, 1) * pitch));
   CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
   CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
   CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
@@ -586,11 +590,12 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.wk.adj12 = ctx->ooc.on ? nullptr : ctx->d_adj12;
   p.wk.bounds = ctx->d_bounds;
   p.wk.P = ctx->P;
-  p.wk.paths = ctx->d_paths;
+  p.wk.paths = home ? ctx->home_paths : ctx->d_paths;
+  p.sys_fence = home ? 1u : 0u;
   p.wk.stride = stride;
   p.wk.pitch = pitch;
   p.wk.path_mode = ctx->cfg.path_mode;
-  p.wk.lengths = ctx->d_lengths;
+  p.wk.lengths = home ? ctx->home_lengths : ctx->d_lengths;
   p.wk.first_walk_id = first_walk_id;
   p.wk.seed_lo = (uint32_t)seed;
   p.wk.seed_hi = (uint32_t)(seed >> 32);
@@ -626,10 +631,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // measured best: 1 walk per lane with the one-gather-per-step ADJ layout, 2 with CSR
   p.ilp = ctx->cfg.ilp ? ctx->cfg.ilp : ((p.wk.adj || p.wk.adj12) ? 1u : 2u);
   // lane refill (k_update_rf): measured faster with one partition (DeepWalk 65.5 vs 81.7 ms, PPR 6.2
-  // vs 7.7 ms on cfg 4 / cfg 3) and slower with several (P=4: 275 vs 208 ms), DESIGN.md §8
-  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P == 1) ? 1u : 0u;
-  // warp-specialised kernel (refill 3): claims kWsMinChunk positions at a time, so it needs C >= that
-  if (ctx->cfg.refill == 3) p.refill = C >= lt::kWsMinChunk ? 3u : 0u;
+  // vs 7.7 ms on cfg 4 / cfg 3); with O records (round 2) also at P = 4 (15.7 vs 14.4·10^9 steps/s on
+  // cfg 4), even at P = 16 and mixed beyond (P = 8: 11.1 vs 11.8; P = 256: 3.8 vs 4.0), DESIGN.md §8
+  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P <= 4) ? 1u : 0u;
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm
@@ -710,13 +714,16 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->snap_valid = false;
   CK(lt::launch_pool_reset(p, s));
   ctx->stats.kernel_launches++;
-  if (W) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
+  // The home rank's matrix and lengths are written by every rank without a per-epoch barrier: after the
+  // first epoch it neither pre-fills nor zeroes them (every length is written once per epoch by the rank
+  // where the walk ends; the rows are padded lazily by the first copy-out, R24).
+  if (W && !home && !ctx->is_home) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
   if (narrow) CK(cudaMemsetAsync(ctx->d_visits32, 0, (size_t)ctx->n * sizeof(uint32_t), s));
   else if (ctx->cfg.visit_counts) CK(cudaMemsetAsync(ctx->d_visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
   // (path_mode 2 stores no rows: d_paths is a placeholder of 8 entries and there is nothing to merge)
-  if (W && ctx->world > 1 && ctx->cfg.path_mode != 2)
+  if (W && ctx->world > 1 && ctx->cfg.path_mode != 2 && !home && !ctx->is_home)
     CK(cudaMemsetAsync(ctx->d_paths, 0xFF, W * (uint64_t)pitch * sizeof(uint32_t), s));
   ctx->adm_starts = d_starts;
   ctx->cap_walks = cap;
@@ -763,7 +770,7 @@ lt_status lt_run(lt_ctx* ctx) {
   }
   // Path rows hold entries 0..length-1; the 0xFFFFFFFF padding of the rest is output formatting and is
   // written lazily by the first copy-out (ensure_padded). With ownership the rows were pre-filled.
-  ctx->padded = ctx->world > 1;
+  ctx->padded = ctx->world > 1 && !ctx->is_home;
   if (ctx->params.wk.visits32) {  // the result is u64[n]
     CK(lt::launch_widen(ctx->params.wk.visits32, ctx->params.wk.visits, ctx->n, s));
     ctx->stats.kernel_launches++;
@@ -813,6 +820,9 @@ lt_status lt_path_stride(lt_ctx* ctx, uint32_t* stride) {
 static lt_status need_ran(lt_ctx* ctx) {
   if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
   if (!ctx->ran) return fail(LT_ERR_STATE, "paths requested before lt_run");
+  if (ctx->cfg.path_mode != 2 && ctx->params.wk.paths != ctx->d_paths)
+    return fail(LT_ERR_STATE, "this rank's paths and lengths were written into the home rank's matrix "
+                              "(lt_paths_attach): read them there");
   CK(cudaSetDevice(ctx->cfg.device));
   if (!ctx->padded && ctx->cfg.path_mode != 2) {  // pad unused path slots with 0xFFFFFFFF once, before the first copy-out
     CK(lt::launch_finalize_paths(ctx->params, ctx->W, ctx->stream));
@@ -823,6 +833,8 @@ static lt_status need_ran(lt_ctx* ctx) {
 
 static lt_status need_paths(lt_ctx* ctx) {
   if (ctx->cfg.path_mode == 2) return fail(LT_ERR_STATE, "paths are not stored (path_mode 2)");
+  if (ctx->params.wk.paths != ctx->d_paths)
+    return fail(LT_ERR_STATE, "this rank's paths were written into the home rank's matrix (lt_paths_attach)");
   return LT_OK;
 }
 
@@ -1135,6 +1147,57 @@ lt_status lt_superstep_p2p(lt_ctx* ctx, unsigned long long* d_sent) {
   ctx->snap_valid = false;
   ctx->peer_epoch ^= 1u;
   ctx->params.peer.epoch = ctx->peer_epoch;
+  return LT_OK;
+}
+
+// ---- paths on the home rank (range ownership): every rank's path entries and lengths are written into
+// one rank's matrix over peer memory, so no cross-rank merge is needed
+lt_status lt_paths_buffers(lt_ctx* ctx, void** d_paths, void** d_lengths, uint64_t* capacity) {
+  if (!ctx || !d_paths || !d_lengths || !capacity) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!ctx->walks_ready) return fail(LT_ERR_STATE, "lt_paths_buffers before lt_walks_init");
+  if (ctx->cfg.path_mode == 2) return fail(LT_ERR_STATE, "paths are not stored (path_mode 2)");
+  if (ctx->home_paths) return fail(LT_ERR_STATE, "this rank writes into another rank's matrix");
+  ctx->is_home = true;
+  *d_paths = ctx->d_paths;
+  *d_lengths = ctx->d_lengths;
+  *capacity = ctx->paths_cap;
+  return LT_OK;
+}
+
+lt_status lt_paths_attach(lt_ctx* ctx, void* d_paths, void* d_lengths, uint64_t capacity) {
+  if (!ctx) return fail(LT_ERR_INVALID, "NULL ctx");
+  if ((d_paths == nullptr) != (d_lengths == nullptr)) return fail(LT_ERR_INVALID, "pass both buffers or neither");
+  if (d_paths && ctx->world < 2) return fail(LT_ERR_INVALID, "lt_paths_attach needs world > 1");
+  if (d_paths && ctx->cfg.path_mode == 2) return fail(LT_ERR_STATE, "paths are not stored (path_mode 2)");
+  if (d_paths && ctx->walks_ready && ctx->cfg.path_mode == 1)
+    return fail(LT_ERR_STATE, "path_mode 1 writes path[w][0] in lt_walks_init: attach before it");
+  CK(cudaSetDevice(ctx->cfg.device));
+  if (d_paths) {
+    for (const void* q : {static_cast<const void*>(d_paths), static_cast<const void*>(d_lengths)}) {
+      cudaPointerAttributes a{};
+      CK(cudaPointerGetAttributes(&a, q));
+      if (a.type != cudaMemoryTypeDevice) return fail(LT_ERR_INVALID, "home buffers must be device memory");
+      if (a.device != ctx->cfg.device) {
+        int can = 0;
+        CK(cudaDeviceCanAccessPeer(&can, ctx->cfg.device, a.device));
+        if (!can) return fail(LT_ERR_INVALID, "no peer access to the home rank's device");
+        const cudaError_t e = cudaDeviceEnablePeerAccess(a.device, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) (void)cudaGetLastError();
+        else CK(e);
+      }
+    }
+  }
+  ctx->home_paths = (uint32_t*)d_paths;
+  ctx->home_lengths = (uint32_t*)d_lengths;
+  ctx->home_cap = d_paths ? capacity : 0;
+  if (ctx->walks_ready) {  // the current epoch writes there from the next launch on
+    const bool home = d_paths != nullptr;
+    if (home && ctx->W * (uint64_t)ctx->pitch > capacity)
+      return fail(LT_ERR_INVALID, "the home rank's path matrix is smaller than W x pitch");
+    ctx->params.wk.paths = home ? ctx->home_paths : ctx->d_paths;
+    ctx->params.wk.lengths = home ? ctx->home_lengths : ctx->d_lengths;
+    ctx->params.sys_fence = home ? 1u : 0u;
+  }
   return LT_OK;
 }
 

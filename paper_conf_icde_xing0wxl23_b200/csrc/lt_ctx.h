@@ -142,6 +142,12 @@ struct lt_ctx {
   lt::OutOfCore ooc;
   lt::Spill spill;
   lt::PhaseEvents load_ev, xfer_ev;  // graph loads (load stream), walk-spill transfers (spill stream)
+  // paths on the home rank (lt_paths_attach): this rank's path entries and lengths go straight into the
+  // home rank's matrix over peer memory
+  uint32_t* home_paths = nullptr;
+  uint32_t* home_lengths = nullptr;
+  uint64_t home_cap = 0;  // u32 entries of home_paths
+  bool is_home = false;   // other ranks write into this rank's matrix (lt_paths_buffers was called)
   // walks
   bool walks_ready = false;
   bool ran = false;

@@ -118,8 +118,9 @@ struct Params {
   uint32_t insert_mode;
   uint32_t gather_mode;
   uint32_t ilp;
-  uint32_t refill;  // 0: batch kernel (k_update), 1: lane refill (k_update_rf), 3: warp-specialised (k_update_ws)
+  uint32_t refill;  // 0: batch kernel (k_update), 1: lane refill (k_update_rf)
   unsigned long long tail_cap;  // an update launch consumes [head, min(cursor, tail_cap)) (walk spill); ~0 otherwise
+  uint32_t sys_fence;           // kernels end with a system-scope fence: they wrote peer memory (paths on the home rank)
 };
 
 // Walk spill (lt_config.walk_spill): chunks moved between the device pool and host memory per launch.
@@ -167,9 +168,8 @@ cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* 
                              cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
                                cudaStream_t s);
-// resident blocks per SM of the update kernel the launch uses (refill: 0 batch, 1 lane refill, 3 warp-specialised)
+// resident blocks per SM of the update kernel the launch uses (refill: 0 batch, 1 lane refill)
 int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill, uint32_t app, uint32_t P);
-constexpr uint32_t kWsMinChunk = 256;  // the warp-specialised kernel claims 256 positions at a time (<= C)
 uint32_t update_smem_bounds_cap();             // max P whose bounds are staged in shared memory
 
 }  // namespace lt

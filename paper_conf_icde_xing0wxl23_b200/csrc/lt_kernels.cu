@@ -197,7 +197,8 @@ __device__ void last_cta_retire(const Params& p, int k, unsigned long long head,
   __shared__ bool s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
-    if (p.peer.recv) __threadfence_system();  // peer-memory appends performed before the grid ends
+    // peer-memory appends (walks for other ranks) and remote path entries performed before the grid ends
+    if (p.peer.recv || p.sys_fence) __threadfence_system();
     else __threadfence();
     const uint32_t ticket = atomicAdd(&p.ctr->done_ctas, 1u);
     s_last = (ticket == gridDim.x - 1);
@@ -727,6 +728,7 @@ __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, c
   __syncwarp();
 }
 
+
 // CONT (out-of-core, CSR layout only): resident-neighbour continuation (the
 // paper's preemptive idea taken inside the kernel). Each lane carries its own graph
 // view (row_ptr / col pointers pre-offset by the view's first vertex / first edge, and the range it
@@ -945,369 +947,6 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   }
   __syncwarp();
   flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
-  my_steps = warp_sum(my_steps);
-  my_trunc = warp_sum(my_trunc);
-  if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
-  if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
-  last_cta_retire(p, (int)k, head, tail);
-}
-
-// ------------------------------------------------------ a3 + a4 + a5, warp-specialised CTA (P > 1)
-// With several partitions a walk leaves its partition after about one step (R-MAT, W = |V|: 0.8-1.0
-// visits per step at P = 4-16), so a visit's fixed costs — reading its record, its first vertex's
-// offset and degree, and inserting it into the next bucket — are paid about once per step. The batch
-// kernel pays them in every stepping warp's critical path (the record load, a dependent row_ptr read,
-// the cursor atomics of the insertion) and idles lanes until a warp's longest walk ends (12 of 32
-// lanes active at P = 4). This kernel takes them off that path:
-//   * 7 stepping warps per CTA run lane refill; each lane keeps its NEXT record prefetched in registers
-//     (loaded while its current walk steps), so a lane whose walk ends starts the next one at once;
-//   * records carry the current vertex's offset and degree (O records, rec_make_o), so a visit starts
-//     with the neighbour gather, not with a dependent row_ptr read;
-//   * a departing walk is pushed into a CTA-wide shared-memory ring (one shared atomic per warp and
-//     departure batch), and the 8th warp drains the ring into the destination buckets, up to 128
-//     records per round with the cursor atomics of all rounds in flight together (the paper's
-//     two-level "local index", with a warp as the inserter);
-//   * the chunk ids of the launched bucket are staged in shared memory (no ring reads per claim).
-// Same step, RNG, path stores and exits as k_update_rf (Alg. 1 l.4-5).
-constexpr uint32_t kWsWarps = 8;                 // 7 stepping warps + 1 inserting warp
-constexpr uint32_t kWsSteppers = kWsWarps - 1;
-constexpr uint32_t kWsDep = 1024;                // departure ring entries (power of two)
-constexpr uint32_t kWsClaim = 256;               // bucket positions a stepping warp claims at a time (<= C)
-constexpr uint32_t kWsRingCache = 2048;          // chunk ids of the launched bucket staged in smem
-constexpr int kWsRounds = 4;                     // inserter: rounds of 32 records per batch
-#ifndef LT_WS_MINB
-#define LT_WS_MINB 3
-#endif
-
-// Warp-collective insertion of R rounds of (up to) 32 records: the cursor atomics of all rounds are
-// issued before any result is used, so one batch costs about one atomic and one ring round trip.
-template <int R>
-__device__ __forceinline__ void insert_warp_rounds(const Params& p, const bool (&act)[R], const uint32_t (&dest)[R],
-                                                   const uint4 (&rec)[R]) {
-  if (p.peer.recv || p.insert_mode == 1) {  // peer buffers / the direct-write ablation: one round at a time
-#pragma unroll
-    for (int r = 0; r < R; ++r) insert_warp(p, act[r], dest[r], rec[r]);
-    return;
-  }
-  const Pool& pl = p.pool;
-  const uint32_t lane = threadIdx.x & 31u;
-  const unsigned long long cmask = pl.C - 1;
-  uint32_t grp[R], leader[R];
-  unsigned long long base[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    const uint32_t a = __ballot_sync(kFull, act[r]);
-    grp[r] = 0;
-    leader[r] = 0;
-    base[r] = 0;
-    if (act[r]) {
-      grp[r] = __match_any_sync(a, dest[r]);
-      leader[r] = __ffs(grp[r]) - 1;
-      if (lane == leader[r]) base[r] = atomicAdd(pl.cursor + dest[r], (unsigned long long)__popc(grp[r]));
-    }
-  }
-  uint32_t c0[R], c1[R];
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    c0[r] = c1[r] = 0;
-    if (act[r] && lane == leader[r]) {
-      const uint32_t cnt = __popc(grp[r]);
-      const unsigned long long ci0 = base[r] >> pl.c_shift, ci1 = (base[r] + cnt - 1) >> pl.c_shift;
-      if (ci1 != ci0) c1[r] = install_chunk(p, dest[r], ci1);
-      c0[r] = (base[r] & cmask) == 0 ? install_chunk(p, dest[r], ci0) : wait_chunk(p, dest[r], ci0);
-      if (ci1 == ci0) c1[r] = c0[r];
-    }
-  }
-#pragma unroll
-  for (int r = 0; r < R; ++r) {
-    if (act[r]) {
-      const unsigned long long b = __shfl_sync(grp[r], base[r], leader[r]);
-      const uint32_t x0 = __shfl_sync(grp[r], c0[r], leader[r]);
-      const uint32_t x1 = __shfl_sync(grp[r], c1[r], leader[r]);
-      const unsigned long long pos = b + __popc(grp[r] & lanemask_lt());
-      const uint32_t c = ((pos >> pl.c_shift) == (b >> pl.c_shift)) ? x0 : x1;
-      pl.slots[((uint64_t)c << pl.c_shift) | (pos & cmask)] = rec[r];
-    }
-  }
-}
-
-template <int APP, int GM, int LAY, int VIS>
-__global__ void __launch_bounds__(kWsWarps * 32, LT_WS_MINB) k_update_ws(Params p, uint32_t k) {
-  extern __shared__ uint32_t s_bounds[];
-  __shared__ uint4 s_dq[kWsDep];       // departure ring: records (final format)
-  __shared__ uint32_t s_dd[kWsDep];    // their destination buckets
-  // slot sequence numbers (a bounded MPSC queue): s_df[slot] == j when the slot is free for departure j,
-  // j + 1 once departure j is written; the inserter frees it for departure j + kWsDep. (Several claims can
-  // wait on one slot — departures j and j + kWsDep — so "free" must name the generation.)
-  __shared__ uint32_t s_df[kWsDep];
-  __shared__ uint32_t s_ring[kWsRingCache];
-  __shared__ uint32_t s_dprod;         // departures claimed by the stepping warps
-  __shared__ uint32_t s_live;          // stepping warps still running
-  const Walk& wk = p.wk;
-  const Pool& pl = p.pool;
-  const unsigned long long head = pl.head[k];
-  // no appends to bucket k during its own launch; a spill-limited launch stops at tail_cap (the first
-  // position of the bucket's first chunk still in host memory)
-  const unsigned long long tail = pl.cursor[k] < p.tail_cap ? pl.cursor[k] : p.tail_cap;
-  const uint32_t lo = wk.bounds[k];
-  const uint32_t span = wk.bounds[k + 1] - lo;
-  const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-  const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
-  const unsigned long long cb = head >> pl.c_shift;
-  const unsigned long long ncb = tail > head ? ((tail - 1) >> pl.c_shift) - cb + 1 : 0;
-  const bool ring_cached = ncb <= kWsRingCache;
-  for (uint32_t i = threadIdx.x; i < kWsDep; i += blockDim.x) s_df[i] = i;
-  if (ring_cached)
-    for (uint32_t i = threadIdx.x; i < ncb; i += blockDim.x) s_ring[i] = ring_k[(cb + i) % pl.ring_len];
-  if (threadIdx.x == 0) {
-    s_dprod = 0;
-    s_live = kWsSteppers;
-  }
-  const uint32_t* B = stage_bounds(wk, s_bounds);
-  __syncthreads();
-  unsigned long long my_steps = 0, my_trunc = 0;
-
-  if (warp < kWsSteppers) {
-    // ------------------------------------------------------------------ stepping warps
-    const Policies pol = make_policies();
-    const uint64_t pol_last = VIS ? make_evict_last() : 0;
-    unsigned long long* claim = pl.claim + k;
-    bool has = false, nxt_ok = false, drained = false;
-    uint4 rec = make_uint4(0, 0, 0, 0), nxt = make_uint4(0, 0, 0, 0);
-    uint32_t* prow = wk.paths;
-    uint32_t pb[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) pb[q] = 0;
-    uint32_t nb = 0, d = 0;
-    unsigned long long off = 0;
-    bool kn = false;
-    // the warp's claimed positions [q_cur, q_end), and the next claim (issued one range ahead)
-    unsigned long long q_cur = 0, q_end = 0, q_next = 0;
-    if (lane == 0) {
-      q_cur = atomicAdd(claim, (unsigned long long)kWsClaim);
-      q_next = atomicAdd(claim, (unsigned long long)kWsClaim);
-    }
-    q_cur = __shfl_sync(kFull, q_cur, 0);
-    q_end = q_cur + kWsClaim < tail ? q_cur + kWsClaim : tail;
-    if (q_cur >= tail) drained = true;
-
-    for (;;) {
-      // ---- a lane whose walk ended takes its prefetched record
-      if (!has && nxt_ok) {
-        rec = nxt;
-        nxt_ok = false;
-        has = true;
-        const bool o = LAY != 0 && rec_decode(rec, off, d);
-        kn = LAY != 0;
-        prow = wk.paths + (uint64_t)rec.x * wk.pitch;
-        pb[7] = rec.y;
-        nb = (!o && (rec.z & 7u) == 0) ? 1u : 0u;
-        if (LAY != 0 && !o) {
-          off = __ldg(wk.row_ptr + rec.y);
-          d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
-        }
-      }
-      // ---- lanes with no prefetched record claim a position and issue its load (used next time)
-      uint32_t want = __ballot_sync(kFull, !nxt_ok);
-      while (want && !drained) {
-        if (q_cur >= q_end) {
-          q_cur = __shfl_sync(kFull, q_next, 0);
-          if (q_cur >= tail) {
-            drained = true;
-            break;
-          }
-          q_end = q_cur + kWsClaim < tail ? q_cur + kWsClaim : tail;
-          if (lane == 0) q_next = atomicAdd(claim, (unsigned long long)kWsClaim);  // result used one range later
-        }
-        const uint32_t avail = (q_end - q_cur < 32ull) ? (uint32_t)(q_end - q_cur) : 32u;
-        const uint32_t r = __popc(want & lanemask_lt());
-        if (!nxt_ok && r < avail) {
-          const unsigned long long pos = q_cur + r;
-          const uint32_t c = ring_cached ? s_ring[(pos >> pl.c_shift) - cb] : ring_k[(pos >> pl.c_shift) % pl.ring_len];
-          nxt = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
-          nxt_ok = true;
-        }
-        const uint32_t took = (uint32_t)__popc(want) < avail ? (uint32_t)__popc(want) : avail;
-        q_cur += took;
-        want = __ballot_sync(kFull, !nxt_ok);
-      }
-      if (!__any_sync(kFull, has || nxt_ok)) break;
-      // ---- one step of every lane that holds a walk
-      bool done = false, left = false, trunc = false;
-      if (has) {
-        if (APP != 1 && rec.z == wk.length) {
-          done = true;
-        } else if (APP == 1 && rec.z == wk.lmax) {
-          done = true;
-          trunc = true;
-        } else {
-          if (LAY == 0) {
-            const unsigned long long* rp = wk.row_ptr + (rec.y - wk.vbase);
-            const unsigned long long r0 = ld_rp(rp), r1 = ld_rp(rp + 1);
-            off = r0 - wk.ebase;
-            d = (uint32_t)(r1 - r0);
-          }
-          const uint64_t wid = wk.first_walk_id + rec.x;
-          const uint4 b = philox10(make_uint4(rec.z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
-          const bool restart = APP == 2 && b.x < wk.T;
-          if ((APP == 1 && b.x < wk.T) || (d == 0 && !restart)) {
-            done = true;
-          } else {
-            const uint32_t dd = restart ? wk.n : d;
-            const uint64_t m = (uint64_t)b.y * dd;
-            const uint32_t idx = ((uint32_t)m < dd) ? lemire_slow(dd, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
-                                                                 wk.seed_lo, wk.seed_hi)
-                                                    : (uint32_t)(m >> 32);
-            uint32_t nv;
-            if (restart) {
-              nv = idx;
-              kn = LAY != 0 && idx - lo < span;
-              if (kn) {
-                off = __ldg(wk.row_ptr + idx);
-                d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
-              }
-            } else if (LAY == 0) {
-              nv = ld_col<GM>(wk.col + off + idx, pol);
-            } else if (LAY == 1) {
-              const uint4 e = ld_adj<GM>(wk.adj + (off - wk.ebase) + idx, pol);
-              nv = e.x;
-              d = e.y;
-              off = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
-              kn = true;
-            } else {
-              const Adj e = ld_adj12<GM>(wk.adj12, off - wk.ebase + idx, pol);
-              nv = e.u;
-              d = e.deg;
-              off = e.off;
-              kn = true;
-            }
-            rec.y = nv;
-            rec.z += 1;
-            count_visit<VIS>(wk, nv, pol_last);
-            const uint32_t t = rec.z;
-            if (wk.path_mode == 0) {
-#pragma unroll
-              for (int q = 0; q < 7; ++q) pb[q] = pb[q + 1];
-              pb[7] = nv;
-              nb += 1;
-              if ((t & 7u) == 7u) {
-                if (nb == 8) {
-                  st_sector(prow + (t - 7), pb, pol);
-                } else {
-#pragma unroll
-                  for (int q = 0; q < 8; ++q)
-                    if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
-                }
-                nb = 0;
-              }
-            } else if (wk.path_mode == 1) {
-              prow[t] = nv;
-            }
-            // a walk that reached its end ends here rather than one visit later in the next bucket
-            if (APP != 1 && t == wk.length) {
-              done = true;
-            } else if (APP == 1 && t == wk.lmax) {
-              done = true;
-              trunc = true;
-            } else {
-              left = (nv - lo >= span);
-            }
-          }
-        }
-      }
-      // ---- retire the walks that ended this step
-      const bool ended = done || left;
-      if (ended && wk.path_mode == 0) {
-        const uint32_t t = rec.z;
-#pragma unroll
-        for (int q = 0; q < 8; ++q)
-          if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
-        nb = 0;
-      }
-      if (done) {
-        wk.lengths[rec.x] = rec.z + 1;
-        my_steps += rec.z;
-        my_trunc += trunc ? 1 : 0;
-      }
-      // ---- departures into the CTA's ring (one shared atomic per warp), drained by the inserting warp
-      const uint32_t lm = __ballot_sync(kFull, left);
-      if (lm) {
-        const uint32_t leader = __ffs(lm) - 1;
-        uint32_t base = 0;
-        if (lane == leader) base = atomicAdd(&s_dprod, (uint32_t)__popc(lm));
-        base = __shfl_sync(kFull, base, leader);
-        if (left) {
-          const uint32_t j = base + __popc(lm & lanemask_lt());
-          const uint32_t slot = j & (kWsDep - 1);
-          const uint32_t dest = bucket_of(p, find_partition(B, wk.P, rec.y));
-          const uint4 out = (LAY != 0 && kn && dest < wk.P && rec_fits_o(rec.z, off)) ? rec_make_o(rec.x, rec.z, off, d)
-                                                                                      : rec;
-          volatile uint32_t* f = s_df + slot;
-          while (*f != j) __nanosleep(32);  // the ring is full: wait for the inserter to free this generation
-          s_dq[slot] = out;
-          s_dd[slot] = dest;
-          __threadfence_block();
-          *f = j + 1;
-        }
-      }
-      if (ended) has = false;
-    }
-    __syncwarp();
-    if (lane == 0) {
-      __threadfence_block();
-      atomicSub(&s_live, 1u);
-    }
-  } else {
-    // ------------------------------------------------------------------ the inserting warp
-    uint32_t cons = 0;
-    uint32_t idle = 0;
-    for (;;) {
-      const uint32_t live = *(volatile uint32_t*)&s_live;
-      __threadfence_block();
-      const uint32_t prod = *(volatile uint32_t*)&s_dprod;
-      uint32_t n = prod - cons;
-      if (n == 0) {
-        if (live == 0) break;  // every stepping warp has pushed its last departure (prod read after live)
-        __nanosleep(128);
-        continue;
-      }
-      if (n < 32 && live != 0 && idle < 4) {  // let a batch build up (fewer atomics per record)
-        ++idle;
-        __nanosleep(256);
-        continue;
-      }
-      idle = 0;
-      if (n > 32u * kWsRounds) n = 32u * kWsRounds;
-      bool act[kWsRounds];
-      uint32_t dst[kWsRounds];
-      uint4 rc[kWsRounds];
-#pragma unroll
-      for (int r = 0; r < kWsRounds; ++r) {
-        const uint32_t i = (uint32_t)r * 32u + lane;
-        act[r] = i < n;
-        dst[r] = 0;
-        rc[r] = make_uint4(0, 0, 0, 0);
-        if (act[r]) {
-          const uint32_t j = cons + i;
-          const uint32_t slot = j & (kWsDep - 1);
-          volatile uint32_t* f = s_df + slot;
-          while (*f != j + 1) __nanosleep(16);  // claimed, not yet written
-          __threadfence_block();
-          rc[r] = s_dq[slot];
-          dst[r] = s_dd[slot];
-        }
-      }
-      __threadfence_block();
-#pragma unroll
-      for (int r = 0; r < kWsRounds; ++r)
-        if (act[r]) {
-          const uint32_t j = cons + (uint32_t)r * 32u + lane;
-          *(volatile uint32_t*)(s_df + (j & (kWsDep - 1))) = j + kWsDep;  // free for departure j + kWsDep
-        }
-      insert_warp_rounds<kWsRounds>(p, act, dst, rc);
-      cons += n;
-    }
-  }
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
   if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
@@ -1561,10 +1200,8 @@ uint32_t update_smem_bounds_cap() { return kSmemBoundsCap - 1; }
 int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill, uint32_t app, uint32_t P) {
   int nb = 0;
   const size_t dyn = (P + 1 <= kSmemBoundsCap) ? (size_t)(P + 1) * sizeof(uint32_t) : 0;
-  if (refill == 3) {
-    cudaFuncSetAttribute(k_update_ws<0, 3, 1, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_ws<0, 3, 1, 0>, (int)(kWsWarps * 32), dyn);
-  } else if (refill && app == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<1, 3, 1, 0, 0>, (int)block, 0);
+  (void)dyn;
+  if (refill && app == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<1, 3, 1, 0, 0>, (int)block, 0);
   else if (refill) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update_rf<0, 3, 1, 0, 0>, (int)block, 0);
   else if (ilp == 1) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 1, 1, 0>, (int)block, 0);
   else if (ilp == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_update<0, 3, 4, 1, 0>, (int)block, 0);
@@ -1677,21 +1314,7 @@ void launch_update_rf(const Params& p, uint32_t k, uint32_t grid, uint32_t block
 }
 
 template <int APP, int GM, int LAY, int VIS>
-void launch_update_ws(const Params& p, uint32_t k, uint32_t grid, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k_update_ws<APP, GM, LAY, VIS>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemBoundsCap * 4);
-    attr = true;
-  }
-  k_update_ws<APP, GM, LAY, VIS><<<grid, kWsWarps * 32, bounds_smem(p), s>>>(p, k);
-}
-
-template <int APP, int GM, int LAY, int VIS>
 void launch_update_ilp(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  if (p.refill == 3) {
-    launch_update_ws<APP, GM, LAY, VIS>(p, k, grid, s);
-    return;
-  }
   if (p.refill) {
     launch_update_rf<APP, GM, LAY, VIS>(p, k, grid, block, s);
     return;

@@ -113,8 +113,9 @@ inline uint64_t append_chunks(const lt_ctx* ctx, uint64_t n) {
 }
 
 // Evict up to `want` chunks of buckets other than `keep` (fewest pending walks first, highest chunk
-// index first). Uses the last snapshot's head/cursor. Returns the number evicted in *done.
-lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done) {
+// index first), or, with only >= 0, of bucket `only` from chunk index min_ci up. Uses the last snapshot's
+// head/cursor. Returns the number evicted in *done.
+lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done, int only = -1, uint64_t min_ci = 0) {
   Range rg("lt walk spill: evict");
   Spill& sp = ctx->spill;
   const uint64_t C = ctx->params.pool.C;
@@ -123,7 +124,7 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done) {
   if (!want) return LT_OK;
   std::vector<uint32_t> order;
   for (uint32_t q = 0; q < nb; ++q)
-    if ((int)q != keep && ctx->h_hc[nb + q] > ctx->h_hc[q]) order.push_back(q);
+    if ((int)q != keep && (only < 0 || (int)q == only) && ctx->h_hc[nb + q] > ctx->h_hc[q]) order.push_back(q);
   std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
     return ctx->h_hc[nb + a] - ctx->h_hc[a] < ctx->h_hc[nb + b] - ctx->h_hc[b];
   });
@@ -158,7 +159,7 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done) {
   };
   for (uint32_t q : order) {
     const uint64_t head = ctx->h_hc[q], cur = ctx->h_hc[nb + q];
-    const uint64_t lo = (head + C - 1) / C;  // first chunk wholly at or after head
+    const uint64_t lo = std::max<uint64_t>((head + C - 1) / C, min_ci);  // first chunk wholly at or after head
     const uint64_t hi = cur / C;             // chunks [lo, hi) end at or before cursor
     for (uint64_t ci = hi; ci-- > lo && *done < want;) {
       if (sp.spilled[q].count(ci)) continue;
@@ -241,6 +242,13 @@ lt_status ensure_walks(lt_ctx* ctx, uint32_t k, unsigned long long* tail_cap) {
   while (r > 0 && sp.free_chunks - (int64_t)r < (int64_t)append_chunks(ctx, covered(r))) --r;
   st = reload_chunks(ctx, k, r);
   if (st != LT_OK) return st;
+  // If the pool is so full that even one chunk of k's walks cannot absorb its appends (k itself holds
+  // most chunks), k's own top chunks are evicted: the launch takes only the first one.
+  if (sp.free_chunks - (int64_t)ctx->nb - 1 < 1) {
+    uint64_t done = 0;
+    st = evict_chunks(ctx, -1, (uint64_t)((int64_t)ctx->nb + 2 - sp.free_chunks), &done, (int)k, (head + C - 1) / C + 1);
+    if (st != LT_OK) return st;
+  }
   // the launch stops at k's first chunk still on the host, or earlier if the free chunks cannot absorb
   // the appends of every device-resident walk before it
   unsigned long long cap = sk.empty() ? ~0ull : sk.begin()->first * C;

@@ -250,6 +250,43 @@ def run_supersteps_p2p_fused(engine, comm, device, max_supersteps: int = 1 << 20
             raise RuntimeError("ownership supersteps did not converge")
 
 
+def attach_paths(engine, comm, home: int = 0):
+    """Paths on the home rank (lt_paths_buffers / lt_paths_attach): every rank writes its path entries and
+    lengths straight into the home rank's matrix over peer memory, so no merge is needed (SURVEY.md §8(b):
+    the merged result lands on rank 0). Call once, after every rank's walks_init of the first epoch
+    (path_mode 0) and before its superstep loop: it synchronises the device and barriers so that no rank
+    writes into the home matrix before the home's walks_init (which pre-fills it that once) has run; later
+    epochs stay attached and need no call (include/lt.h). Calling it again is harmless. Handles are
+    exchanged once and cached on the engine."""
+    import torch
+    me = comm.rank
+    key = getattr(engine, "_home_key", None)
+    if me == home:
+        p, l, cap = engine.paths_buffers()
+        mine = (p, l, cap) if comm.same_process else (lt_ipc(p), lt_ipc(l), cap, p, l)
+    else:
+        mine = None
+    allv = comm.allgather_obj(mine)
+    hv = allv[home]
+    if me != home:
+        if comm.same_process:
+            p, l, cap = hv
+        else:
+            if key != (hv[3], hv[4]):  # open the home's IPC handles once per allocation
+                engine._home_ptrs = (engine.ipc_open(hv[0]), engine.ipc_open(hv[1]))
+                engine._home_key = (hv[3], hv[4])
+            p, l = engine._home_ptrs
+            cap = hv[2]
+        engine.paths_attach(p, l, cap)
+    torch.cuda.synchronize()
+    comm.allgather_obj(None)  # barrier: the home's pre-fill is complete before anyone writes into it
+
+
+def lt_ipc(dptr: int) -> bytes:
+    from .lt import ipc_handle
+    return ipc_handle(dptr)
+
+
 def merge_paths(engine, comm):
     """Cross-rank merge of the partial path matrices: unsigned min of entries, max of lengths.
     Returns CUDA/CPU int32 tensors (paths [W, stride], lengths [W]) identical on every rank."""

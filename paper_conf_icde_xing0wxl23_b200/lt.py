@@ -35,7 +35,7 @@ EXPORTED = [
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
     "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
     "lt_exchange_buffers", "lt_exchange_attach", "lt_exchange_sent", "lt_exchange_take", "lt_ipc_handle",
-    "lt_ipc_open", "lt_superstep_p2p",
+    "lt_ipc_open", "lt_superstep_p2p", "lt_paths_buffers", "lt_paths_attach",
 ]
 
 
@@ -123,6 +123,8 @@ _lib.lt_exchange_take.argtypes = [_vp, ctypes.POINTER(_u64)]
 _lib.lt_ipc_handle.argtypes = [_vp, _vp]
 _lib.lt_ipc_open.argtypes = [_vp, _vp, ctypes.POINTER(_vp)]
 _lib.lt_superstep_p2p.argtypes = [_vp, _vp]
+_lib.lt_paths_buffers.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_u64)]
+_lib.lt_paths_attach.argtypes = [_vp, _vp, _vp, _u64]
 _lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
 _lib.lt_run_to_host_compact.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u64, _u32]
 _lib.lt_get_paths_compact.argtypes = [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]
@@ -441,6 +443,22 @@ class Engine:
         if not dev:
             raise ValueError("superstep_p2p needs a CUDA tensor")
         _check(_lib.lt_superstep_p2p(self._h, pp))
+
+    def paths_buffers(self):
+        """Home rank: (path matrix, length array, capacity in u32 entries) device addresses (lt_paths_buffers)."""
+        p, l, c = _vp(), _vp(), _u64()
+        _check(_lib.lt_paths_buffers(self._h, ctypes.byref(p), ctypes.byref(l), ctypes.byref(c)))
+        return int(p.value), int(l.value), int(c.value)
+
+    def paths_attach(self, d_paths, d_lengths, capacity: int):
+        """Write this rank's path entries and lengths into the home rank's buffers (lt_paths_attach);
+        (None, None, 0) writes locally again."""
+        _check(_lib.lt_paths_attach(self._h, _vp(d_paths) if d_paths else None, _vp(d_lengths) if d_lengths else None,
+                                    int(capacity)))
+
+    def home_paths(self):
+        """Home rank after the epoch: (paths [W, stride], lengths [W]) CUDA int32 tensors (all ranks' entries)."""
+        return self.partial_paths()
 
     def export_buffers(self):
         """CUDA IPC handles of this rank's receive buffers (parity 0, 1) and of its cursor pair."""

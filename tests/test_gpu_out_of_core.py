@@ -181,11 +181,11 @@ def test_continue_zero_copy_small_chunks(gpu, g14, app, param):
 
 
 @pytest.mark.parametrize("zero_copy", [False, True])
-def test_out_of_core_warp_specialised_kernel(gpu, g14, zero_copy):
-    """Out of core without continuation on the warp-specialised kernel (refill 3): graph-pool block views
-    and the zero-copy view of the mapped host CSR (CSR layout, V records)."""
+def test_out_of_core_lane_refill_without_continuation(gpu, g14, zero_copy):
+    """Out of core without continuation on the lane-refill kernel (refill 2): graph-pool block views and
+    the zero-copy view of the mapped host CSR (CSR layout, V records)."""
     starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
-    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, 16, 3, zero_copy=zero_copy, refill=3, chunk_walks=512)
+    paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, 16, 3, zero_copy=zero_copy, refill=2, chunk_walks=512)
     op, ol, _, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
     np.testing.assert_array_equal(paths, op)
     np.testing.assert_array_equal(lengths, ol)

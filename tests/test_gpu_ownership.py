@@ -292,7 +292,7 @@ def test_fused_superstep_exact(gpu, g13, world, layout, app, param):
 
     def rank_main(r):
         try:
-            with LT.Engine(rank=r, world=world, layout=layout, chunk_walks=512) as e:
+            with LT.Engine(rank=r, world=world, layout=layout, chunk_walks=512, timing=True) as e:
                 e.graph_load(g13.row_ptr, g13.col, world)
                 comm = ltdist.ThreadComm(hub, r)
                 res = []
@@ -389,7 +389,7 @@ def test_ownership_paths_off_visit_counts(gpu, g13, p2p):
 
     def rank_main(r):
         try:
-            with LT.Engine(rank=r, world=world, path_mode=2, visit_counts=True, chunk_walks=512) as e:
+            with LT.Engine(rank=r, world=world, path_mode=2, visit_counts=True, chunk_walks=512, timing=True) as e:
                 e.graph_load(g13.row_ptr, g13.col, 8)
                 e.walks_init_pagerank(starts, 12, 0.15, 9)
                 comm = ltdist.ThreadComm(hub, r)
@@ -423,13 +423,14 @@ def test_ownership_paths_off_visit_counts(gpu, g13, p2p):
 
 @pytest.mark.parametrize("exchange", ["alltoall", "p2p", "fused"])
 @pytest.mark.parametrize("layout", [LT.LAYOUT_CSR, LT.LAYOUT_ADJ])
-def test_ownership_warp_specialised_kernel(gpu, g13, exchange, layout):
-    """Range ownership on the warp-specialised kernel (refill 3): walks for other ranks leave as V
-    records (a receiver needs the vertex), through send buckets or straight into peer buffers."""
+def test_ownership_lane_refill_offset_records(gpu, g13, exchange, layout):
+    """Range ownership on the lane-refill kernel at P > 1 (refill 2): walks for a local bucket leave as O
+    records, walks for other ranks as V records (a receiver needs the vertex), through send buckets or
+    straight into peer buffers."""
     world = 3
     starts = lt_inputs.deepwalk_starts(3 * g13.n, g13.n)
     P = world if exchange == "fused" else 12
-    kw = dict(layout=layout, refill=3, chunk_walks=512)
+    kw = dict(layout=layout, refill=2, chunk_walks=512)
     if exchange == "alltoall":
         res = run_owned(g13, starts, LT.DEEPWALK, 16, 2, P, world, **kw)
     else:
@@ -467,3 +468,113 @@ def test_ownership_warp_specialised_kernel(gpu, g13, exchange, layout):
         np.testing.assert_array_equal(lengths, ol)
         np.testing.assert_array_equal(paths, op)
     assert sum(r[3]["steps"] for r in res) == osteps
+
+
+# ---- paths on the home rank (lt_paths_buffers / lt_paths_attach): every rank writes its path entries and
+# lengths straight into rank 0's matrix, so the paths are complete there without a merge
+
+@pytest.mark.parametrize("exchange", ["alltoall", "p2p", "fused"])
+@pytest.mark.parametrize("app,param", [(LT.DEEPWALK, 16), (LT.PPR, 0.15)])
+def test_paths_on_home_rank(gpu, g13, exchange, app, param):
+    import torch
+    world = 3
+    starts = (lt_inputs.deepwalk_starts(3 * g13.n, g13.n) if app == LT.DEEPWALK
+              else lt_inputs.ppr_starts(20_000, g13.argmax_deg))
+    P = world if exchange == "fused" else 12
+    hub = ltdist.ThreadComm.Hub(world)
+    out, errors = [None] * world, []
+
+    def rank_main(r):
+        try:
+            with LT.Engine(rank=r, world=world, layout=LT.LAYOUT_ADJ, chunk_walks=512, refill=2) as e:
+                e.graph_load(g13.row_ptr, g13.col, P)
+                comm = ltdist.ThreadComm(hub, r)
+                res = []
+                for seed in (2, 3):  # two epochs: the second reuses the attachment
+                    e.walks_init(starts, app, param, seed)
+                    ltdist.attach_paths(e, comm)
+                    if exchange == "alltoall":
+                        ltdist.run_supersteps(e, comm, "cuda")
+                    else:
+                        if seed == 2:
+                            ltdist.attach_peers(e, comm, len(starts))
+                        run = ltdist.run_supersteps_p2p_fused if exchange == "fused" else ltdist.run_supersteps_p2p
+                        run(e, comm, "cuda")
+                    torch.cuda.synchronize()
+                    comm.allgather_obj(None)  # every rank's kernels are done
+                    if r == 0:
+                        paths, lengths = e.home_paths()
+                        res.append((paths.cpu().numpy().view(np.uint32), lengths.cpu().numpy().view(np.uint32)))
+                    else:
+                        with pytest.raises(LT.LTError):
+                            e.get_paths()  # the paths live on the home rank
+                    assert e.stats()["steps"] >= 0
+                out[r] = res
+        except Exception as ex:
+            errors.append(ex)
+            hub.barrier.abort()
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    if errors:
+        raise errors[0]
+    for i, seed in enumerate((2, 3)):
+        op, ol, _, _ = oracle_of(g13, starts, app, param, seed)
+        paths, lengths = out[0][i]
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+
+
+def _home_proc(rank, world, port, out_q):
+    import os
+
+    import torch
+    import torch.distributed as tdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    tdist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        g = lt_inputs.rmat_cpu(13, 8 * 2 ** 13, seed=3)
+        starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+        with LT.Engine(rank=rank, world=world) as e:
+            e.graph_load(g.row_ptr, g.col, world)
+            e.walks_init(starts, LT.DEEPWALK, 12, 7)
+            comm = ltdist.TorchComm()
+            ltdist.attach_paths(e, comm)  # CUDA IPC of rank 0's path matrix and length array
+            ltdist.attach_peers(e, comm, len(starts))
+            ltdist.run_supersteps_p2p_fused(e, comm, "cuda:0")
+            torch.cuda.synchronize()
+            tdist.barrier()
+            if rank == 0:
+                paths, lengths = e.home_paths()
+                out_q.put((paths.cpu().numpy().view(np.uint32).copy(), lengths.cpu().numpy().view(np.uint32).copy()))
+    finally:
+        tdist.destroy_process_group()
+
+
+def test_paths_on_home_rank_processes_cuda_ipc(gpu):
+    import socket
+
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_home_proc, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    paths, lengths = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    g = lt_inputs.rmat_cpu(13, 8 * 2 ** 13, seed=3)
+    starts = lt_inputs.deepwalk_starts(2 * g.n, g.n)
+    op, ol, _, _ = oracle_of(g, starts, LT.DEEPWALK, 12, 7)
+    np.testing.assert_array_equal(lengths, ol)
+    np.testing.assert_array_equal(paths, op)

@@ -51,7 +51,7 @@ def run_spill(g, starts, app, param, seed, P, cap, length=15, **cfg):
 
 @pytest.mark.parametrize("cap_div", [3, 8])
 @pytest.mark.parametrize("P", [4, 16, 64])
-@pytest.mark.parametrize("refill", [0, 2, 3])
+@pytest.mark.parametrize("refill", [0, 2])
 def test_spill_deepwalk_exact(gpu, g14, cap_div, P, refill):
     W = 4 * g14.n
     C = 256

@@ -2,7 +2,7 @@
 """Partition-count sweep of the update kernels on one GPU (DESIGN.md §8 "P > 1"): BASELINE configs[3]
 (FS-shaped R-MAT s26, |V| DeepWalk walks of length 80; --config picks another), one JSON line per
 (kernel, P): steps/s device-timed over --steps walks after --warmup, visits per step, sweeps, launches.
-  refill 0 = batch kernel (k_update), 2 = lane refill (k_update_rf), 3 = warp-specialised (k_update_ws)."""
+  refill 0 = batch kernel (k_update), 2 = lane refill (k_update_rf)."""
 import argparse
 import json
 import os
@@ -20,7 +20,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", type=int, default=4)
     ap.add_argument("--P", default="4,8,16,64")
-    ap.add_argument("--refill", default="0,3")
+    ap.add_argument("--refill", default="0,2")
     ap.add_argument("--layout", type=int, default=0)
     ap.add_argument("--app", default="config")
     ap.add_argument("--steps", type=int, default=3)
@@ -65,7 +65,7 @@ def main():
                     ms = ev0.elapsed_time(ev1)
                     steps = sum(s["steps"] for s in sts)
                     line = {"config": a.config, "app": app, "P": P, "refill": rf, "insert_mode": im,
-                            "kernel": {0: "k_update", 1: "k_update", 2: "k_update_rf", 3: "k_update_ws"}[rf],
+                            "kernel": {0: "k_update", 1: "k_update", 2: "k_update_rf"}[rf],
                             "layout": sts[-1]["layout"], "steps_per_s": steps / (ms / 1e3), "ms_per_step": ms / a.steps,
                             "update_ms_per_step": sum(s["update_ms"] for s in sts) / a.steps,
                             "visits_per_step": sum(s["visits"] for s in sts) / max(1, steps),

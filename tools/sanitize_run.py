@@ -4,7 +4,9 @@ initcheck): resident P=1 (refill), P=4 (batch kernel, CSR and ADJ), PPR, out-of-
 two-rank ownership, streamed run_to_host (dense and ragged), ragged copy-out, PageRank with u32 / u64
 visit counters, out-of-core continuation, walk admission, paths off, the direct start (P = 1, both
 path modes, device starts), the compact ADJ12 layout, slice-only ownership (CSR / ADJ / ADJ12, host and
-borrowed device graphs), the peer exchange (CSR / ADJ)."""
+borrowed device graphs), the peer exchange (CSR / ADJ); round 2: O records through the lane-refill kernel at
+P > 1 and the walk spill
+(evict / reload kernels, tail-capped launches)."""
 import os
 import sys
 import threading
@@ -22,7 +24,7 @@ starts = lt_inputs.deepwalk_starts(4096, g.n)
 pstarts = lt_inputs.ppr_starts(4096, g.argmax_deg)
 for kw in [dict(P=1), dict(P=4, layout=LT.LAYOUT_CSR), dict(P=4, layout=LT.LAYOUT_ADJ), dict(P=4, refill=2),
            dict(P=1, layout=LT.LAYOUT_ADJ12), dict(P=4, layout=LT.LAYOUT_ADJ12), dict(P=1, path_mode=1),
-           dict(P=1, direct_start=False)]:
+           dict(P=1, direct_start=False), dict(P=4, refill=2, layout=LT.LAYOUT_CSR)]:
     P = kw.pop("P")
     with LT.Engine(chunk_walks=256, **kw) as e:
         e.graph_load(g.row_ptr, g.col, P)
@@ -110,4 +112,19 @@ for layout in (LT.LAYOUT_CSR, LT.LAYOUT_ADJ):
         t.start()
     for t in th:
         t.join()
+print("sanitize_run done")
+
+# round 2: O records at P > 1 (lane refill) and walk spill
+g14 = lt_inputs.rmat_cpu(14, 16 * 2 ** 14, seed=2)
+s14 = lt_inputs.deepwalk_starts(4 * g14.n, g14.n)
+with LT.Engine(chunk_walks=256, refill=2) as e:
+    e.graph_load(g14.row_ptr, g14.col, 8)
+    e.walks_init(s14, LT.DEEPWALK, 12, 1)
+    e.run()
+    e.get_paths()
+with LT.Engine(chunk_walks=256, walk_pool_walks=len(s14) // 5, walk_spill=True) as e:
+    e.graph_load(g14.row_ptr, g14.col, 8)
+    e.walks_init(s14, LT.DEEPWALK, 12, 1)
+    e.run()
+    e.get_paths()
 print("sanitize_run done")
