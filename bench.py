@@ -403,7 +403,7 @@ def main():
         and free the device one (room for the e2e buffers)."""
         nonlocal g, g_host
         if args.release_col and not ooc and eng.stats()["layout"] != LT.LAYOUT_CSR and \
-                not isinstance(g.col, np.ndarray) and g.col is not None and not args.sweep:
+                not isinstance(g.col, np.ndarray) and g.col is not None and not args.sweep and not own:
             if rank == 0 and world == 1 and not args.no_cpu_baseline:
                 g_host = host_graph(g)
             g = lt_inputs.Graph(g.n, g.m, g.row_ptr, None, g.max_deg, g.argmax_deg)

@@ -47,7 +47,8 @@ typedef enum {
   LT_ERR_STATE = 2,   /* call out of order */
   LT_ERR_OOM = 3,     /* device memory reservation failed (create / graph_load / walks_init) */
   LT_ERR_CUDA = 4,    /* a CUDA runtime error, or a device-side invariant violation */
-  LT_ERR_NCCL = 5     /* reserved for the multi-GPU exchange */
+  LT_ERR_NCCL = 5     /* reserved: the library issues no collective itself (the caller's torch.distributed
+                         does, dist.py), so it never returns this */
 } lt_status;
 
 typedef enum {
@@ -154,6 +155,15 @@ typedef struct lt_config {
   uint32_t l2_persist;        /* L2 set-aside for the lines the kernels tag evict_last (visit counters,
                                  row_ptr): 0 -> leave cudaLimitPersistingL2CacheSize as it is; 1 -> set
                                  it to the device maximum at lt_create (process-wide device state) */
+  void* arena;                /* caller-owned device memory (e.g. a torch tensor) on cfg->device, or NULL
+                                 (SURVEY.md §8(b)): when given, every pool the library reserves — graph,
+                                 augmented adjacency, walk pool, paths, lengths, counters, staging — is
+                                 sub-allocated from it (256-B aligned bump allocation; LT_ERR_OOM when it
+                                 runs out), nothing is freed back, and each lt_graph_load* starts it over.
+                                 It stays owned by the caller and must outlive the context. Not used for
+                                 buffers shared through CUDA IPC (lt_exchange_buffers; lt_paths_buffers is
+                                 refused) nor for the temporaries of lt_get_paths_rows. */
+  uint64_t arena_bytes;
 } lt_config;
 
 typedef struct lt_stats {
@@ -204,6 +214,7 @@ typedef struct lt_stats {
   double load_ms;              /* graph-partition H2D copies on the load stream (out-of-core) */
   double spill_xfer_ms;        /* walk-spill D2H + H2D copies on the transfer stream */
   uint64_t host_syncs;         /* scheduler round trips: count reads that wait for the device */
+  uint64_t arena_bytes_used;   /* high-water mark of the caller arena (lt_config.arena), 0 without one */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,
@@ -385,6 +396,11 @@ lt_status lt_paths_attach(lt_ctx* ctx, void* d_paths, void* d_lengths, uint64_t 
  * handle on this context's device (closed at lt_destroy). */
 lt_status lt_ipc_handle(const void* dptr, void* handle);
 lt_status lt_ipc_open(lt_ctx* ctx, const void* handle, void** dptr);
+
+/* Diagnostic (SURVEY.md §4 pin P2): the update kernels' Philox4x32-10 (reading R3) evaluated on the
+ * device for n counters ctr[4i..4i+3] and keys key[2i..2i+1] (host arrays), out[4i..4i+3] = the block.
+ * Lets tests compare the device RNG with cuRAND's curand_Philox4x32_10. Synchronous. */
+lt_status lt_philox_device(int device, uint64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out);
 
 /* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:
  * pending + finished == num_walks; free_chunks + ring_chunks == total_chunks. */

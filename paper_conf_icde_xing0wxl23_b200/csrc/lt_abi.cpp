@@ -21,9 +21,57 @@ lt_status fail(lt_status s, const std::string& msg) {
   g_err = msg;
   return s;
 }
+
+cudaError_t dmalloc(lt_ctx* ctx, void** p, size_t bytes) {
+  if (!ctx->arena) return cudaMalloc(p, bytes);
+  const size_t at = (ctx->arena_top + 255) & ~size_t(255);
+  if (at + bytes > ctx->arena_size) return cudaErrorMemoryAllocation;  // -> LT_ERR_OOM
+  *p = ctx->arena + at;
+  ctx->arena_top = at + bytes;
+  ctx->arena_peak = std::max(ctx->arena_peak, ctx->arena_top);
+  return cudaSuccess;
+}
+
+void dfree(lt_ctx* ctx, void* p) {
+  if (!p) return;
+  if (ctx->arena && (char*)p >= ctx->arena && (char*)p < ctx->arena + ctx->arena_size) return;  // caller-owned
+  cudaFree(p);
+}
+
+void arena_track(lt_ctx* ctx, void** p, size_t* cap) {
+  if (!ctx->arena) return;
+  for (const auto& b : ctx->arena_bufs)
+    if (b.first == p) return;
+  ctx->arena_bufs.emplace_back(p, cap);
+}
+
+// A graph load starts the arena over (every pool buffer is reserved again, graph first): the buffers of
+// the previous graph and walks are dropped.
+static void arena_reset(lt_ctx* ctx) {
+  if (!ctx->arena) return;
+  for (const auto& b : ctx->arena_bufs) {
+    *b.first = nullptr;
+    *b.second = 0;
+  }
+  for (int i = 0; i < 2; ++i) {
+    ctx->d_paths2[i] = nullptr;
+    ctx->paths2_cap[i] = 0;
+    ctx->d_lengths2[i] = nullptr;
+    ctx->lengths2_cap[i] = 0;
+  }
+  if (ctx->own_graph) {
+    ctx->d_row_ptr = nullptr;
+    ctx->d_col = nullptr;
+  }
+  ctx->d_owner = nullptr;
+  ctx->walks_ready = false;
+  ctx->arena_top = ctx->arena_mark;
+}
 }  // namespace lt
 using lt::fail;
 using lt::ensure;
+using lt::dfree;
+using lt::dmalloc;
 
 extern "C" {
 
@@ -91,8 +139,20 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
     if (e == cudaSuccess) e = cudaDeviceGetLimit(&got, cudaLimitPersistingL2CacheSize);
     ctx->stats.l2_persist_bytes = got;
   }
-  if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_small, 4 * sizeof(uint32_t));
-  if (e == cudaSuccess) e = cudaMalloc((void**)&ctx->d_ctr, sizeof(lt::Counters));
+  if (c.arena || c.arena_bytes) {  // caller-owned device memory for every pool
+    cudaPointerAttributes a{};
+    if (!c.arena || c.arena_bytes < 4096 || cudaPointerGetAttributes(&a, c.arena) != cudaSuccess ||
+        a.type != cudaMemoryTypeDevice || a.device != c.device) {
+      (void)cudaGetLastError();
+      lt_destroy(ctx);
+      return fail(LT_ERR_INVALID, "arena must be device memory of cfg->device, >= 4096 bytes");
+    }
+    ctx->arena = (char*)c.arena;
+    ctx->arena_size = c.arena_bytes;
+  }
+  if (e == cudaSuccess) e = dmalloc(ctx, (void**)&ctx->d_small, 4 * sizeof(uint32_t));
+  if (e == cudaSuccess) e = dmalloc(ctx, (void**)&ctx->d_ctr, sizeof(lt::Counters));
+  ctx->arena_mark = ctx->arena_top;
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_ctr, sizeof(lt::Counters), cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&ctx->h_free, sizeof(int), cudaHostAllocMapped);
   if (e == cudaSuccess) e = cudaEventCreate(&ctx->ev_a);
@@ -111,8 +171,8 @@ static void free_ooc(lt_ctx* ctx) {
   for (auto e : o.ev_ready) cudaEventDestroy(e);
   for (auto e : o.ev_used) cudaEventDestroy(e);
   if (o.load_stream) cudaStreamDestroy(o.load_stream);
-  if (o.d_gpool) cudaFree(o.d_gpool);
-  if (o.d_table) cudaFree(o.d_table);
+  if (o.d_gpool) dfree(ctx, o.d_gpool);
+  if (o.d_table) dfree(ctx, o.d_table);
   if (o.h_row_ptr) cudaFreeHost(o.h_row_ptr);
   if (o.h_col) cudaFreeHost(o.h_col);
   ctx->ooc = lt::OutOfCore();
@@ -126,19 +186,19 @@ void lt_destroy(lt_ctx* ctx) {
   lt::free_spill(ctx);
   ctx->load_ev.destroy();
   ctx->xfer_ev.destroy();
-  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
-  cudaFree(ctx->d_adj);
-  cudaFree(ctx->d_adj12);
-  cudaFree(ctx->d_bounds);
-  cudaFree(ctx->d_owner);
-  cudaFree(ctx->d_paths);
-  cudaFree(ctx->d_lengths);
+  if (ctx->own_graph) { dfree(ctx, ctx->d_row_ptr); dfree(ctx, ctx->d_col); }
+  dfree(ctx, ctx->d_adj);
+  dfree(ctx, ctx->d_adj12);
+  dfree(ctx, ctx->d_bounds);
+  dfree(ctx, ctx->d_owner);
+  dfree(ctx, ctx->d_paths);
+  dfree(ctx, ctx->d_lengths);
   for (int i = 0; i < 2; ++i) {
-    if (ctx->d_paths2[i] && ctx->d_paths2[i] != ctx->d_paths) cudaFree(ctx->d_paths2[i]);
-    if (ctx->d_lengths2[i] && ctx->d_lengths2[i] != ctx->d_lengths) cudaFree(ctx->d_lengths2[i]);
-    if (ctx->d_dense2[i]) cudaFree(ctx->d_dense2[i]);
-    if (ctx->d_off2[i]) cudaFree(ctx->d_off2[i]);
-    if (ctx->d_vert2[i]) cudaFree(ctx->d_vert2[i]);
+    if (ctx->d_paths2[i] && ctx->d_paths2[i] != ctx->d_paths) dfree(ctx, ctx->d_paths2[i]);
+    if (ctx->d_lengths2[i] && ctx->d_lengths2[i] != ctx->d_lengths) dfree(ctx, ctx->d_lengths2[i]);
+    if (ctx->d_dense2[i]) dfree(ctx, ctx->d_dense2[i]);
+    if (ctx->d_off2[i]) dfree(ctx, ctx->d_off2[i]);
+    if (ctx->d_vert2[i]) dfree(ctx, ctx->d_vert2[i]);
     if (ctx->ev_computed[i]) cudaEventDestroy(ctx->ev_computed[i]);
     if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
   }
@@ -149,18 +209,18 @@ void lt_destroy(lt_ctx* ctx) {
   cudaFree(ctx->d_xcur);
   cudaFree(ctx->d_peer_recv);
   cudaFree(ctx->d_peer_cur);
-  cudaFree(ctx->d_starts);
-  cudaFree(ctx->d_starts_all);
-  cudaFree(ctx->d_visits);
-  cudaFree(ctx->d_visits32);
-  cudaFree(ctx->d_slots);
-  cudaFree(ctx->d_ring);
-  cudaFree(ctx->d_hc);
-  cudaFree(ctx->d_free);
-  cudaFree(ctx->d_small);
-  cudaFree(ctx->d_tiles);
+  dfree(ctx, ctx->d_starts);
+  dfree(ctx, ctx->d_starts_all);
+  dfree(ctx, ctx->d_visits);
+  dfree(ctx, ctx->d_visits32);
+  dfree(ctx, ctx->d_slots);
+  dfree(ctx, ctx->d_ring);
+  dfree(ctx, ctx->d_hc);
+  dfree(ctx, ctx->d_free);
+  dfree(ctx, ctx->d_small);
+  dfree(ctx, ctx->d_tiles);
   if (ctx->h_total) cudaFreeHost(ctx->h_total);
-  cudaFree(ctx->d_ctr);
+  dfree(ctx, ctx->d_ctr);
   if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
   if (ctx->h_ctr) cudaFreeHost(ctx->h_ctr);
   if (ctx->h_free) cudaFreeHost(ctx->h_free);
@@ -256,18 +316,18 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     }
   }
   if (lay == LT_LAYOUT_ADJ) {
-    CK(ensure(ctx->d_adj, ctx->adj_cap, ml));
+    CK(ensure(ctx, ctx->d_adj, ctx->adj_cap, ml));
     CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj, ctx->stream));
   } else if (ctx->d_adj) {
-    cudaFree(ctx->d_adj);
+    dfree(ctx, ctx->d_adj);
     ctx->d_adj = nullptr;
     ctx->adj_cap = 0;
   }
   if (lay == LT_LAYOUT_ADJ12) {
-    CK(ensure(ctx->d_adj12, ctx->adj12_cap, 3 * ml));
+    CK(ensure(ctx, ctx->d_adj12, ctx->adj12_cap, 3 * ml));
     CK(lt::launch_build_adj12(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj12, ctx->stream));
   } else if (ctx->d_adj12) {
-    cudaFree(ctx->d_adj12);
+    dfree(ctx, ctx->d_adj12);
     ctx->d_adj12 = nullptr;
     ctx->adj12_cap = 0;
   }
@@ -275,7 +335,7 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   // one may be released by the caller, include/lt.h)
   if (lay != LT_LAYOUT_CSR && ctx->own_graph && ctx->d_col) {
     CK(cudaStreamSynchronize(ctx->stream));
-    cudaFree(ctx->d_col);
+    dfree(ctx, ctx->d_col);
     ctx->d_col = nullptr;
   }
   ctx->stats.layout = (uint32_t)lay;
@@ -285,7 +345,7 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   std::vector<uint32_t> b(P + 1);
   lt_status s = lt_partition_bounds(n, h_row_ptr, P, b.data());
   if (s != LT_OK) return s;
-  CK(ensure(ctx->d_bounds, ctx->bounds_cap, P + 1));
+  CK(ensure(ctx, ctx->d_bounds, ctx->bounds_cap, P + 1));
   CK(cudaMemcpy(ctx->d_bounds, b.data(), (P + 1) * sizeof(uint32_t), cudaMemcpyHostToDevice));
   // range ownership: rank r owns partitions [floor(P r / R), floor(P (r+1) / R))
   const uint32_t R = ctx->world;
@@ -293,17 +353,17 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   ctx->own_lo = (uint32_t)((uint64_t)P * ctx->rank / R);
   ctx->own_hi = (uint32_t)((uint64_t)P * (ctx->rank + 1) / R);
   ctx->nb = P + (R > 1 ? R : 0);
-  if (ctx->d_owner) cudaFree(ctx->d_owner);
+  if (ctx->d_owner) dfree(ctx, ctx->d_owner);
   ctx->d_owner = nullptr;
   if (R > 1) {
     std::vector<uint16_t> own(P);
     for (uint32_t r = 0; r < R; ++r)
       for (uint64_t q = (uint64_t)P * r / R; q < (uint64_t)P * (r + 1) / R; ++q) own[q] = (uint16_t)r;
-    CK(cudaMalloc((void**)&ctx->d_owner, P * sizeof(uint16_t)));
+    CK(dmalloc(ctx, (void**)&ctx->d_owner, P * sizeof(uint16_t)));
     CK(cudaMemcpy(ctx->d_owner, own.data(), P * sizeof(uint16_t), cudaMemcpyHostToDevice));
   }
   const size_t nb = ctx->nb;
-  CK(ensure(ctx->d_hc, ctx->hc_cap, 3 * nb));  // head, cursor, refill claim
+  CK(ensure(ctx, ctx->d_hc, ctx->hc_cap, 3 * nb));  // head, cursor, refill claim
   if (ctx->h_hc_cap < 2 * nb) {
     if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
     ctx->h_hc = nullptr;
@@ -368,7 +428,7 @@ static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     return fail(LT_ERR_INVALID, "graph pool smaller than one partition (" + std::to_string(o.block_bytes) +
                                     " B): raise num_partitions or graph_pool_bytes");
   o.m_g = (uint32_t)std::min<uint64_t>(mg, P);
-  CK(cudaMalloc((void**)&o.d_gpool, (size_t)o.m_g * o.block_bytes));
+  CK(dmalloc(ctx, (void**)&o.d_gpool, (size_t)o.m_g * o.block_bytes));
   o.block_of.assign(P, -1);
   o.part_in.assign(o.m_g, -1);
   o.loaded_at.assign(o.m_g, 0);
@@ -379,7 +439,7 @@ static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     CK(cudaEventCreateWithFlags(&o.ev_used[q], cudaEventDisableTiming));
   }
   CK(cudaStreamCreateWithFlags(&o.load_stream, cudaStreamNonBlocking));
-  CK(cudaMalloc((void**)&o.d_table, (size_t)P * sizeof(uint32_t)));
+  CK(dmalloc(ctx, (void**)&o.d_table, (size_t)P * sizeof(uint32_t)));
   CK(cudaMemset(o.d_table, 0xFF, (size_t)P * sizeof(uint32_t)));
   o.table.assign(P, lt::kEmpty);
   o.on = true;
@@ -397,7 +457,9 @@ lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row
   for (uint64_t i = 0; i < m; ++i)
     if (col[i] >= n) return fail(LT_ERR_INVALID, "col[" + std::to_string(i) + "] >= n");
   if (P == 0 || P > n) return fail(LT_ERR_INVALID, "need 1 <= num_partitions <= n");
-  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  CK(cudaDeviceSynchronize());  // nothing in flight reads the buffers the load replaces
+  if (ctx->own_graph) { dfree(ctx, ctx->d_row_ptr); dfree(ctx, ctx->d_col); }
+  lt::arena_reset(ctx);
   ctx->d_row_ptr = nullptr;
   ctx->d_col = nullptr;
   ctx->graph_loaded = false;
@@ -414,8 +476,8 @@ lt_status lt_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64_t* row
   s = owned_edges(ctx, n, m, row_ptr, P, &e_lo, &e_hi);
   if (s != LT_OK) return s;
   ctx->own_graph = true;
-  CK(cudaMalloc((void**)&ctx->d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t)));
-  CK(cudaMalloc((void**)&ctx->d_col, std::max<uint64_t>(e_hi - e_lo, 1) * sizeof(uint32_t)));
+  CK(dmalloc(ctx, (void**)&ctx->d_row_ptr, ((size_t)n + 1) * sizeof(uint64_t)));
+  CK(dmalloc(ctx, (void**)&ctx->d_col, std::max<uint64_t>(e_hi - e_lo, 1) * sizeof(uint32_t)));
   CK(cudaMemcpy(ctx->d_row_ptr, row_ptr, ((size_t)n + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice));
   if (e_hi > e_lo) CK(cudaMemcpy(ctx->d_col, col + e_lo, (e_hi - e_lo) * sizeof(uint32_t), cudaMemcpyHostToDevice));
   ctx->e_lo = e_lo;
@@ -439,7 +501,9 @@ lt_status lt_graph_load_device(lt_ctx* ctx, uint32_t n, uint64_t m, const uint64
   CK(cudaMemcpyAsync(&bad, ctx->d_small + 2, sizeof(uint32_t), cudaMemcpyDeviceToHost, ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
   if (bad) return fail(LT_ERR_INVALID, "col entry >= n");
-  if (ctx->own_graph) { cudaFree(ctx->d_row_ptr); cudaFree(ctx->d_col); }
+  CK(cudaDeviceSynchronize());
+  if (ctx->own_graph) { dfree(ctx, ctx->d_row_ptr); dfree(ctx, ctx->d_col); }
+  lt::arena_reset(ctx);
   ctx->own_graph = false;
   ctx->graph_loaded = false;
   free_ooc(ctx);
@@ -529,7 +593,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   if (!on_device) {
     for (uint64_t i = 0; i < W; ++i)
       if (starts[i] >= ctx->n) return fail(LT_ERR_INVALID, "starts[" + std::to_string(i) + "] >= n");
-    CK(ensure(ctx->d_starts, ctx->starts_cap, W));
+    CK(ensure(ctx, ctx->d_starts, ctx->starts_cap, W));
     if (W) CK(cudaMemcpyAsync(ctx->d_starts, starts, W * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
     ctx->stats.h2d_bytes += W * 4;
     d_starts = ctx->d_starts;
@@ -564,15 +628,15 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const bool home = ctx->home_paths != nullptr && ctx->world > 1 && ctx->cfg.path_mode != 2;
   if (home && (uint64_t)W * pitch > ctx->home_cap)
     return fail(LT_ERR_INVALID, "the home rank's path matrix is smaller than W x pitch; attach again");
-  CK(ensure(ctx->d_paths, ctx->paths_cap, (ctx->cfg.path_mode == 2 || home) ? 8 : std::max<uint64_t>(W, 1) * pitch));
-  CK(ensure(ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
-  CK(ensure(ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
-  CK(ensure(ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
-  CK(ensure(ctx->d_free, ctx->free_cap, num_chunks));
+  CK(ensure(ctx, ctx->d_paths, ctx->paths_cap, (ctx->cfg.path_mode == 2 || home) ? 8 : std::max<uint64_t>(W, 1) * pitch));
+  CK(ensure(ctx, ctx->d_lengths, ctx->lengths_cap, std::max<uint64_t>(W, 1)));
+  CK(ensure(ctx, ctx->d_slots, ctx->slots_cap, (num_chunks + 1) * C));
+  CK(ensure(ctx, ctx->d_ring, ctx->ring_cap, (uint64_t)ctx->nb * ring_len));
+  CK(ensure(ctx, ctx->d_free, ctx->free_cap, num_chunks));
   // visit counters: u32 while no count can reach 2^32 (at most W * stride path entries in total)
   const bool narrow = ctx->cfg.visit_counts == 1 && (uint64_t)W * stride < 0xFFFFFFFFull;
-  if (ctx->cfg.visit_counts) CK(ensure(ctx->d_visits, ctx->visits_cap, ctx->n));
-  if (narrow) CK(ensure(ctx->d_visits32, ctx->visits32_cap, ctx->n));
+  if (ctx->cfg.visit_counts) CK(ensure(ctx, ctx->d_visits, ctx->visits_cap, ctx->n));
+  if (narrow) CK(ensure(ctx, ctx->d_visits32, ctx->visits32_cap, ctx->n));
   if (on_device == 1 && W) {
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
     CK(lt::launch_check_starts(d_starts, W, ctx->n, ctx->d_small + 2, s));
@@ -695,7 +759,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
         sp.host_cap = host_cap;
       }
       for (int b = 0; b < 2; ++b) {
-        CK(ensure(sp.d_stage[b], sp.stage_cap[b], (size_t)lt::kSpillBatch * C));
+        CK(ensure(ctx, sp.d_stage[b], sp.stage_cap[b], (size_t)lt::kSpillBatch * C));
         if (!sp.ev_ready[b]) CK(cudaEventCreateWithFlags(&sp.ev_ready[b], cudaEventDisableTiming));
         if (!sp.ev_free[b]) CK(cudaEventCreateWithFlags(&sp.ev_free[b], cudaEventDisableTiming));
       }
@@ -908,13 +972,13 @@ static lt_status pack_compact(lt_ctx* ctx, const uint32_t* d_paths, const uint32
   if (!ctx->h_total) CK(cudaHostAlloc((void**)&ctx->h_total, sizeof(unsigned long long), cudaHostAllocMapped));
   unsigned long long* d_total = nullptr;
   CK(cudaHostGetDevicePointer((void**)&d_total, ctx->h_total, 0));
-  CK(ensure(ctx->d_tiles, ctx->tiles_cap, std::max<uint64_t>(lt::paths_scan_tiles(n), 1)));
-  CK(ensure(ctx->d_off2[b], ctx->off2_cap[b], std::max<uint64_t>(n, 1)));
+  CK(ensure(ctx, ctx->d_tiles, ctx->tiles_cap, std::max<uint64_t>(lt::paths_scan_tiles(n), 1)));
+  CK(ensure(ctx, ctx->d_off2[b], ctx->off2_cap[b], std::max<uint64_t>(n, 1)));
   *ctx->h_total = 0;
   CK(lt::launch_paths_scan(d_lengths, n, ctx->d_tiles, d_total, s));
   CK(cudaStreamSynchronize(s));
   const uint64_t tot = *(volatile unsigned long long*)ctx->h_total;
-  CK(ensure(ctx->d_vert2[b], ctx->vert2_cap[b], std::max<uint64_t>(tot, 1)));
+  CK(ensure(ctx, ctx->d_vert2[b], ctx->vert2_cap[b], std::max<uint64_t>(tot, 1)));
   CK(lt::launch_paths_pack(d_lengths, n, ctx->d_tiles, base, ctx->d_off2[b], d_paths, ctx->pitch, ctx->d_vert2[b], s));
   *total = tot;
   return LT_OK;
@@ -1157,6 +1221,8 @@ lt_status lt_paths_buffers(lt_ctx* ctx, void** d_paths, void** d_lengths, uint64
   if (!ctx->walks_ready) return fail(LT_ERR_STATE, "lt_paths_buffers before lt_walks_init");
   if (ctx->cfg.path_mode == 2) return fail(LT_ERR_STATE, "paths are not stored (path_mode 2)");
   if (ctx->home_paths) return fail(LT_ERR_STATE, "this rank writes into another rank's matrix");
+  if (ctx->arena)
+    return fail(LT_ERR_STATE, "with a caller arena the path matrix is a sub-allocation: CUDA IPC needs its own");
   ctx->is_home = true;
   *d_paths = ctx->d_paths;
   *d_lengths = ctx->d_lengths;
@@ -1250,7 +1316,7 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
   // All starts go H2D once (pinned host memory: at the link rate) and are range-checked on the device,
   // instead of a host loop over W starts in front of every range's walk: each range then starts from
   // its slice of the validated device array.
-  CK(ensure(ctx->d_starts_all, ctx->starts_all_cap, std::max<uint64_t>(W, 1)));
+  CK(ensure(ctx, ctx->d_starts_all, ctx->starts_all_cap, std::max<uint64_t>(W, 1)));
   if (W) {
     CK(cudaMemcpyAsync(ctx->d_starts_all, starts, W * sizeof(uint32_t), cudaMemcpyHostToDevice, ctx->stream));
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), ctx->stream));
@@ -1315,7 +1381,7 @@ static lt_status run_to_host_impl(lt_ctx* ctx, uint64_t W, const uint32_t* start
       d2h += n * 8 + tot * 4;
     } else if (n) {  // stream chunk c out while chunk c+1 computes
       // dense rows first (a 2-D copy of 324-B rows runs well below the link rate)
-      CK(ensure(ctx->d_dense2[b], ctx->dense2_cap[b], n * ctx->stride));
+      CK(ensure(ctx, ctx->d_dense2[b], ctx->dense2_cap[b], n * ctx->stride));
       CK(lt::launch_compact_rows(ctx->d_paths2[b], ctx->d_lengths2[b], ctx->pitch, ctx->stride, n, ctx->d_dense2[b],
                                  ctx->stream));
       CK(cudaEventRecord(ctx->ev_computed[b], ctx->stream));
@@ -1383,8 +1449,30 @@ lt_status lt_get_visit_counts_device(lt_ctx* ctx, uint64_t* d_counts) {
   return copy_visits(ctx, d_counts, cudaMemcpyDeviceToDevice);
 }
 
+lt_status lt_philox_device(int device, uint64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out) {
+  if (n && (!ctr || !key || !out)) return fail(LT_ERR_INVALID, "NULL argument");
+  if (!n) return LT_OK;
+  CK(cudaSetDevice(device));
+  uint4* d_ctr = nullptr;
+  uint2* d_key = nullptr;
+  uint4* d_out = nullptr;
+  cudaError_t e = cudaMalloc((void**)&d_ctr, n * sizeof(uint4));
+  if (e == cudaSuccess) e = cudaMalloc((void**)&d_key, n * sizeof(uint2));
+  if (e == cudaSuccess) e = cudaMalloc((void**)&d_out, n * sizeof(uint4));
+  if (e == cudaSuccess) e = cudaMemcpy(d_ctr, ctr, n * sizeof(uint4), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = cudaMemcpy(d_key, key, n * sizeof(uint2), cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) e = lt::launch_philox_blocks(d_ctr, d_key, d_out, n, nullptr);
+  if (e == cudaSuccess) e = cudaMemcpy(out, d_out, n * sizeof(uint4), cudaMemcpyDeviceToHost);
+  cudaFree(d_ctr);
+  cudaFree(d_key);
+  cudaFree(d_out);
+  if (e != cudaSuccess) return fail(LT_ERR_CUDA, std::string("lt_philox_device: ") + cudaGetErrorString(e));
+  return LT_OK;
+}
+
 lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out) {
   if (!ctx || !out) return fail(LT_ERR_INVALID, "NULL argument");
+  ctx->stats.arena_bytes_used = ctx->arena ? ctx->arena_peak : 0;
   *out = ctx->stats;
   return LT_OK;
 }

@@ -8,18 +8,30 @@
 #include <string>
 #include <vector>
 
+struct lt_ctx;
+
 namespace lt {
 
 lt_status fail(lt_status s, const std::string& msg);
 
+// Device memory of the library's pools ("the library sub-allocates all pools from it
+// once"): from the caller-owned arena (lt_config.arena) when one is given — a bump allocator, 256-B
+// aligned; freeing inside the arena is a no-op and lt_graph_load* resets it — else cudaMalloc.
+cudaError_t dmalloc(lt_ctx* ctx, void** p, size_t bytes);
+void dfree(lt_ctx* ctx, void* p);
+void arena_track(lt_ctx* ctx, void** p, size_t* cap);  // ensure() buffers: nulled when the arena resets
+
 template <class T>
-cudaError_t ensure(T*& p, size_t& cap, size_t count) {
+cudaError_t ensure(lt_ctx* ctx, T*& p, size_t& cap, size_t count) {
   if (count <= cap && p) return cudaSuccess;
-  if (p) cudaFree(p);
+  if (p) dfree(ctx, p);
   p = nullptr;
   cap = 0;
-  cudaError_t e = cudaMalloc((void**)&p, std::max<size_t>(count, 1) * sizeof(T));
-  if (e == cudaSuccess) cap = count;
+  cudaError_t e = dmalloc(ctx, (void**)&p, std::max<size_t>(count, 1) * sizeof(T));
+  if (e == cudaSuccess) {
+    cap = count;
+    arena_track(ctx, (void**)&p, &cap);
+  }
   return e;
 }
 
@@ -142,6 +154,11 @@ struct lt_ctx {
   lt::OutOfCore ooc;
   lt::Spill spill;
   lt::PhaseEvents load_ev, xfer_ev;  // graph loads (load stream), walk-spill transfers (spill stream)
+  // caller-owned arena (lt_config.arena): [arena, arena + arena_size), bump pointer arena_top; buffers
+  // from ensure() registered in arena_bufs are dropped when a graph load resets the arena to arena_mark
+  char* arena = nullptr;
+  size_t arena_size = 0, arena_top = 0, arena_mark = 0, arena_peak = 0;
+  std::vector<std::pair<void**, size_t*>> arena_bufs;
   // paths on the home rank (lt_paths_attach): this rank's path entries and lengths go straight into the
   // home rank's matrix over peer memory
   uint32_t* home_paths = nullptr;

@@ -149,6 +149,7 @@ cudaError_t launch_compact_rows(const uint32_t* paths, const uint32_t* lengths, 
 cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
+cudaError_t launch_philox_blocks(const uint4* ctr, const uint2* key, uint4* out, uint64_t n, cudaStream_t s);
 // walk spill: chunks list[0..count) -> stage (ring slots marked kSpilled, chunks freed) / stage -> fresh chunks
 cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* stage, cudaStream_t s);
 cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* stage, cudaStream_t s);

@@ -1437,6 +1437,20 @@ cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count
   return cudaGetLastError();
 }
 
+// Diagnostic (tests/test_gpu_philox.py, SURVEY.md §4 pin P2): the update kernels' own Philox4x32-10 on
+// given counters and keys, so the device RNG can be compared with cuRAND's curand_Philox4x32_10.
+__global__ void k_philox_blocks(const uint4* __restrict__ ctr, const uint2* __restrict__ key, uint4* __restrict__ out,
+                                uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    out[i] = philox10(ctr[i], key[i].x, key[i].y);
+}
+
+cudaError_t launch_philox_blocks(const uint4* ctr, const uint2* key, uint4* out, uint64_t n, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_philox_blocks<<<num_sms() * 4, 256, 0, s>>>(ctr, key, out, n);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s) {
   k_pool_reset<<<num_sms() * 4, 256, 0, s>>>(p);
   return cudaGetLastError();

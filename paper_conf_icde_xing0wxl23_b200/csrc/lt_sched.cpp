@@ -224,33 +224,35 @@ lt_status ensure_walks(lt_ctx* ctx, uint32_t k, unsigned long long* tail_cap) {
   const uint64_t C = ctx->params.pool.C;
   const uint64_t head = ctx->h_hc[k], cur = ctx->h_hc[ctx->nb + k];
   auto& sk = sp.spilled[k];
-  // walks a launch would cover after reloading the first r evicted chunks of k
-  auto covered = [&](uint64_t r) -> uint64_t {
-    if (r >= sk.size()) return cur - head;
-    auto it = sk.begin();
-    std::advance(it, (long)r);
-    return it->first * C - head;
-  };
-  const uint64_t all = sk.size();
-  const int64_t want_free = (int64_t)(all + append_chunks(ctx, cur - head));
+  // (1) room for k's evicted chunks and every append of its launch: other buckets' chunks go first
+  const int64_t want_free = (int64_t)(sk.size() + append_chunks(ctx, cur - head));
   if (sp.free_chunks < want_free) {
     uint64_t done = 0;
     st = evict_chunks(ctx, (int)k, (uint64_t)(want_free - sp.free_chunks), &done);
     if (st != LT_OK) return st;
   }
-  uint64_t r = all;
-  while (r > 0 && sp.free_chunks - (int64_t)r < (int64_t)append_chunks(ctx, covered(r))) --r;
-  st = reload_chunks(ctx, k, r);
-  if (st != LT_OK) return st;
-  // If the pool is so full that even one chunk of k's walks cannot absorb its appends (k itself holds
-  // most chunks), k's own top chunks are evicted: the launch takes only the first one.
-  if (sp.free_chunks - (int64_t)ctx->nb - 1 < 1) {
+  // (2) the launch must make progress: room for one chunk of appends, plus k's first evicted chunk when
+  // it starts at head. If the pool is still that full (k itself holds most chunks), k's own top chunks
+  // above its first full chunk are evicted.
+  const bool head_spilled = !sk.empty() && sk.begin()->first * C <= head;
+  const int64_t min_free = (head_spilled ? 1 : 0) + (int64_t)ctx->nb + 2;
+  if (sp.free_chunks < min_free) {
     uint64_t done = 0;
-    st = evict_chunks(ctx, -1, (uint64_t)((int64_t)ctx->nb + 2 - sp.free_chunks), &done, (int)k, (head + C - 1) / C + 1);
+    st = evict_chunks(ctx, -1, (uint64_t)(min_free - sp.free_chunks), &done, (int)k, (head + C - 1) / C + 1);
     if (st != LT_OK) return st;
   }
-  // the launch stops at k's first chunk still on the host, or earlier if the free chunks cannot absorb
-  // the appends of every device-resident walk before it
+  // (3) reload k's evicted chunks, lowest first, while the free chunks still absorb the appends of every
+  // walk up to the end of the reloaded chunk
+  uint64_t r = 0;
+  for (auto it = sk.begin(); it != sk.end(); ++it) {
+    const uint64_t walks_to = (it->first + 1) * C - head;
+    if (sp.free_chunks < (int64_t)(r + 1 + append_chunks(ctx, walks_to))) break;
+    ++r;
+  }
+  st = reload_chunks(ctx, k, r);
+  if (st != LT_OK) return st;
+  // (4) the launch stops at k's first chunk still on the host, or earlier if the free chunks cannot
+  // absorb the appends of every device-resident walk before it
   unsigned long long cap = sk.empty() ? ~0ull : sk.begin()->first * C;
   const int64_t room = sp.free_chunks - (int64_t)ctx->nb - 1;  // chunks left for full chunks of appends
   if (room < 1) return fail(LT_ERR_OOM, "walk spill: the walk pool cannot hold one chunk of appends; raise walk_pool_walks");
@@ -295,7 +297,7 @@ void free_spill(lt_ctx* ctx) {
   if (sp.xfer) cudaStreamSynchronize(sp.xfer);
   if (sp.h_store) cudaFreeHost(sp.h_store);
   for (int b = 0; b < 2; ++b) {
-    if (sp.d_stage[b]) cudaFree(sp.d_stage[b]);
+    if (sp.d_stage[b]) dfree(ctx, sp.d_stage[b]);
     if (sp.ev_ready[b]) cudaEventDestroy(sp.ev_ready[b]);
     if (sp.ev_free[b]) cudaEventDestroy(sp.ev_free[b]);
   }

@@ -35,7 +35,7 @@ EXPORTED = [
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
     "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
     "lt_exchange_buffers", "lt_exchange_attach", "lt_exchange_sent", "lt_exchange_take", "lt_ipc_handle",
-    "lt_ipc_open", "lt_superstep_p2p", "lt_paths_buffers", "lt_paths_attach",
+    "lt_ipc_open", "lt_superstep_p2p", "lt_paths_buffers", "lt_paths_attach", "lt_philox_device",
 ]
 
 
@@ -68,6 +68,8 @@ class Config(ctypes.Structure):
         ("walk_pool_walks", ctypes.c_uint64),
         ("direct_start", ctypes.c_uint32),
         ("l2_persist", ctypes.c_uint32),
+        ("arena", ctypes.c_void_p),
+        ("arena_bytes", ctypes.c_uint64),
     ]
 
 
@@ -81,7 +83,8 @@ class Stats(ctypes.Structure):
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
             "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes", "prefetches",
             "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak")] + [
-        ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64)]
+        ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64),
+        ("arena_bytes_used", ctypes.c_uint64)]
 
 
 class PoolState(ctypes.Structure):
@@ -125,6 +128,17 @@ _lib.lt_ipc_open.argtypes = [_vp, _vp, ctypes.POINTER(_vp)]
 _lib.lt_superstep_p2p.argtypes = [_vp, _vp]
 _lib.lt_paths_buffers.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_u64)]
 _lib.lt_paths_attach.argtypes = [_vp, _vp, _vp, _u64]
+_lib.lt_philox_device.argtypes = [ctypes.c_int, _u64, _vp, _vp, _vp]
+
+
+def philox_device(ctr, key, device: int = 0) -> np.ndarray:
+    """The update kernels' Philox4x32-10 on the device (lt_philox_device): ctr u32[n, 4], key u32[n, 2]."""
+    ctr = np.ascontiguousarray(ctr, dtype=np.uint32).reshape(-1, 4)
+    key = np.ascontiguousarray(key, dtype=np.uint32).reshape(-1, 2)
+    assert len(ctr) == len(key)
+    out = np.zeros_like(ctr)
+    _check(_lib.lt_philox_device(device, len(ctr), ctr.ctypes.data, key.ctypes.data, out.ctypes.data))
+    return out
 _lib.lt_run_to_host.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u32]
 _lib.lt_run_to_host_compact.argtypes = [_vp, _u64, _vp, _u64, ctypes.c_int, ctypes.c_double, _u64, _vp, _vp, _u64, _u32]
 _lib.lt_get_paths_compact.argtypes = [_vp, _vp, _vp, _u64, ctypes.POINTER(_u64)]
@@ -192,7 +206,7 @@ class Engine:
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
                  visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
                  direct_start: bool = True, l2_persist: int = 0, ooc_prefetch: bool = False,
-                 walk_spill: bool = False):
+                 walk_spill: bool = False, arena=None):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -217,6 +231,12 @@ class Engine:
         cfg.continue_resident = int(bool(continue_resident))
         cfg.walk_pool_walks = int(walk_pool_walks)
         cfg.walk_spill = int(bool(walk_spill))
+        if arena is not None:  # caller-owned device memory (a CUDA tensor) for every pool
+            if not (_is_torch(arena) and arena.is_cuda and arena.is_contiguous()):
+                raise ValueError("arena must be a contiguous CUDA tensor")
+            cfg.arena = arena.data_ptr()
+            cfg.arena_bytes = arena.numel() * arena.element_size()
+        self._arena_keep = arena
         cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
         cfg.l2_persist = int(l2_persist)
         cfg.ooc_prefetch = int(bool(ooc_prefetch))
