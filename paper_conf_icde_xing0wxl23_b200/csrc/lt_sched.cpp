@@ -125,7 +125,11 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done, int
   std::vector<uint32_t> order;
   for (uint32_t q = 0; q < nb; ++q)
     if ((int)q != keep && (only < 0 || (int)q == only) && ctx->h_hc[nb + q] > ctx->h_hc[q]) order.push_back(q);
+  // reading R17: out of core, the buckets of partitions whose graph is NOT in the graph pool go first (a
+  // resident partition is likely computed soon); then the fewest pending walks
+  auto resident = [&](uint32_t q) { return ctx->ooc.on && q < ctx->P && ctx->ooc.block_of[q] >= 0; };
   std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) {
+    if (resident(a) != resident(b)) return !resident(a);
     return ctx->h_hc[nb + a] - ctx->h_hc[a] < ctx->h_hc[nb + b] - ctx->h_hc[b];
   });
   SpillList list;
@@ -137,16 +141,31 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done, int
     CK(launch_spill(ctx->params, list, cnt, sp.d_stage[b], s));
     CK(cudaEventRecord(sp.ev_ready[b], s));
     CK(cudaStreamWaitEvent(sp.xfer, sp.ev_ready[b], 0));
+    uint32_t slots[kSpillBatch];
+    uint64_t waited = 0;  // bitmask of transfer events already waited for (64 = kXferEvents)
+    for (uint32_t i = 0; i < cnt; ++i) {
+      slots[i] = sp.host_free.back();
+      sp.host_free.pop_back();
+      const int e = sp.slot_ev[slots[i]];  // the reload that last read this slot must be done
+      if (e >= 0 && !(waited >> e & 1)) {
+        CK(cudaStreamWaitEvent(sp.xfer, sp.xev[e], 0));
+        waited |= 1ull << e;
+      }
+    }
     if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer));
     for (uint32_t i = 0; i < cnt; ++i) {
-      const uint32_t slot = sp.host_free.back();
-      sp.host_free.pop_back();
-      CK(cudaMemcpyAsync(sp.h_store + (uint64_t)slot * C, sp.d_stage[b] + (uint64_t)i * C, C * sizeof(uint4),
+      CK(cudaMemcpyAsync(sp.h_store + (uint64_t)slots[i] * C, sp.d_stage[b] + (uint64_t)i * C, C * sizeof(uint4),
                          cudaMemcpyDeviceToHost, sp.xfer));
-      sp.spilled[list.bucket[i]][list.chunk[i]] = slot;
+      sp.spilled[list.bucket[i]][list.chunk[i]] = slots[i];
     }
     if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer));
     CK(cudaEventRecord(sp.ev_free[b], sp.xfer));
+    {
+      const int e = sp.xev_next;
+      sp.xev_next = (sp.xev_next + 1) % Spill::kXferEvents;
+      CK(cudaEventRecord(sp.xev[e], sp.xfer));
+      for (uint32_t i = 0; i < cnt; ++i) sp.slot_ev[slots[i]] = e;
+    }
     sp.host_used += cnt;
     sp.free_chunks += cnt;
     ctx->stats.spilled_chunks += cnt;
@@ -186,19 +205,36 @@ lt_status reload_chunks(lt_ctx* ctx, uint32_t k, uint64_t r) {
   while (r) {
     SpillList list;
     uint32_t cnt = 0;
-    const int b = stage_take(ctx, sp.xfer);
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer));
+    const int b = stage_take(ctx, sp.xfer_in);
+    uint32_t slots[kSpillBatch];
+    uint64_t waited = 0;
     for (auto it = sk.begin(); it != sk.end() && cnt < kSpillBatch && cnt < r;) {
       list.bucket[cnt] = k;
       list.chunk[cnt] = it->first;
-      CK(cudaMemcpyAsync(sp.d_stage[b] + (uint64_t)cnt * C, sp.h_store + (uint64_t)it->second * C, C * sizeof(uint4),
-                         cudaMemcpyHostToDevice, sp.xfer));
-      sp.host_free.push_back(it->second);  // later D2H into this slot are ordered after this H2D (same stream)
+      slots[cnt] = it->second;
+      const int e = sp.slot_ev[it->second];  // the eviction that wrote this slot must be done
+      if (e >= 0 && !(waited >> e & 1)) {
+        CK(cudaStreamWaitEvent(sp.xfer_in, sp.xev[e], 0));
+        waited |= 1ull << e;
+      }
       it = sk.erase(it);
       ++cnt;
     }
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer));
-    CK(cudaEventRecord(sp.ev_ready[b], sp.xfer));
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer_in));
+    for (uint32_t i = 0; i < cnt; ++i)
+      CK(cudaMemcpyAsync(sp.d_stage[b] + (uint64_t)i * C, sp.h_store + (uint64_t)slots[i] * C, C * sizeof(uint4),
+                         cudaMemcpyHostToDevice, sp.xfer_in));
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer_in));
+    CK(cudaEventRecord(sp.ev_ready[b], sp.xfer_in));
+    {
+      const int e = sp.xev_next;
+      sp.xev_next = (sp.xev_next + 1) % Spill::kXferEvents;
+      CK(cudaEventRecord(sp.xev[e], sp.xfer_in));
+      for (uint32_t i = 0; i < cnt; ++i) {
+        sp.slot_ev[slots[i]] = e;
+        sp.host_free.push_back(slots[i]);  // a later eviction into this slot waits for this H2D
+      }
+    }
     CK(cudaStreamWaitEvent(ctx->stream, sp.ev_ready[b], 0));
     CK(launch_reload(ctx->params, list, cnt, sp.d_stage[b], ctx->stream));
     CK(cudaEventRecord(sp.ev_free[b], ctx->stream));
@@ -295,6 +331,7 @@ lt_status spill_admit_all(lt_ctx* ctx) {
 void free_spill(lt_ctx* ctx) {
   Spill& sp = ctx->spill;
   if (sp.xfer) cudaStreamSynchronize(sp.xfer);
+  if (sp.xfer_in) cudaStreamSynchronize(sp.xfer_in);
   if (sp.h_store) cudaFreeHost(sp.h_store);
   for (int b = 0; b < 2; ++b) {
     if (sp.d_stage[b]) dfree(ctx, sp.d_stage[b]);
@@ -302,6 +339,8 @@ void free_spill(lt_ctx* ctx) {
     if (sp.ev_free[b]) cudaEventDestroy(sp.ev_free[b]);
   }
   if (sp.xfer) cudaStreamDestroy(sp.xfer);
+  if (sp.xfer_in) cudaStreamDestroy(sp.xfer_in);
+  for (auto e : sp.xev) cudaEventDestroy(e);
   sp = Spill();
 }
 

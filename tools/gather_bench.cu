@@ -4,7 +4,8 @@
 // value, like a walk step). Reports loads/s and useful GB/s; pair with ncu dram__bytes_read.sum to
 // get the DRAM bytes actually moved per load (the DRAM access atom).
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o tools/gather_bench tools/gather_bench.cu
-//   tools/gather_bench <bytes> <width 4|8|16|32|64> <U> <dependent 0|1> [iters] [blocks_per_sm] [mode]
+//   tools/gather_bench <bytes> <width 4|8|16|32|64> <U 1|2|4|8|16|32> <dependent 0|1> [iters] [blocks_per_sm] [mode]
+// mode (width 16): 0 plain __ldg, 1 L2::64B, 3 L2 evict_first + L2::64B (the walk kernel's gather)
 #include <cstdio>
 #include <cstdlib>
 #include <cuda_runtime.h>
@@ -57,7 +58,21 @@ __global__ void __launch_bounds__(256) k_gather(const uint4* __restrict__ buf, u
       uint32_t v;
       if (WIDTH == 4) v = ld4((const uint32_t*)p, g_mode);
       else if (WIDTH == 8) { uint2 t = __ldg((const uint2*)p); v = t.x ^ t.y; }
-      else if (WIDTH == 16) { uint4 t = __ldg((const uint4*)p); v = t.x ^ t.y ^ t.z ^ t.w; }
+      else if (WIDTH == 16) {
+        uint4 t;
+        if (g_mode == 3) {  // the walk kernel's neighbour gather: L2 evict_first + 64-B fill
+          uint64_t pol;
+          asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+          asm volatile("ld.global.nc.L2::cache_hint.L2::64B.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+                       : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w) : "l"(p), "l"(pol));
+        } else if (g_mode == 1) {
+          asm volatile("ld.global.nc.L2::64B.v4.u32 {%0, %1, %2, %3}, [%4];"
+                       : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w) : "l"(p));
+        } else {
+          t = __ldg((const uint4*)p);
+        }
+        v = t.x ^ t.y ^ t.z ^ t.w;
+      }
       else {
         v = 0;
 #pragma unroll
@@ -100,6 +115,8 @@ float dispatch_u(int U, bool dep, const uint4* buf, uint64_t bytes, int iters, i
     case 5: return run<WIDTH, 2, true>(buf, bytes, iters, grid, s);
     case 8: return run<WIDTH, 4, false>(buf, bytes, iters, grid, s);
     case 9: return run<WIDTH, 4, true>(buf, bytes, iters, grid, s);
+    case 32: return run<WIDTH, 16, false>(buf, bytes, iters, grid, s);
+    case 64: return run<WIDTH, 32, false>(buf, bytes, iters, grid, s);
     default: return run<WIDTH, 8, false>(buf, bytes, iters, grid, s);
   }
 }
