@@ -137,9 +137,9 @@ typedef struct lt_config {
                                  walk exists from the start and the walk pool EVICTS whole chunks of the
                                  buckets with the fewest pending walks to pinned host memory when it is
                                  full, and loads a partition's evicted chunks back before the partition
-                                 is computed (reading R17). Eviction (D2H)
-                                 and loading (H2D) run on their own stream through double-buffered
-                                 staging. Single-rank contexts only. Paths are unchanged. */
+                                 is computed (reading R17). The copies are
+                                 kernels reading / writing a pinned, mapped host store (no per-chunk
+                                 cudaMemcpy). Single-rank contexts only. Paths are unchanged. */
   uint64_t walk_pool_walks;   /* m_w, the walk pool's capacity in walks (D4; SURVEY.md
                                  8(f) f3): 0 -> sized for all W walks. When W > m_w the walks are
                                  admitted in index order as the pool drains: lt_walks_init creates the
@@ -208,11 +208,12 @@ typedef struct lt_stats {
   uint64_t spill_d2h_bytes;    /* walk records moved device -> host by evictions */
   uint64_t spill_h2d_bytes;    /* walk records moved host -> device by reloads */
   uint64_t host_chunks_peak;   /* most chunks held in host memory at once */
+  uint64_t spill_prefetched_chunks; /* reloads started during the previous partition's launch (overlapped) */
   /* per-phase breakdown of the last lt_run (update vs reshuffle vs loading). The
      reshuffle (bucket insertion, a5) is fused into the update kernels, so update_ms covers both. With
      lt_config.timing: */
   double load_ms;              /* graph-partition H2D copies on the load stream (out-of-core) */
-  double spill_xfer_ms;        /* walk-spill D2H + H2D copies on the transfer stream */
+  double spill_xfer_ms;        /* walk-spill copy kernels (evictions + reloads over PCIe) */
   uint64_t host_syncs;         /* scheduler round trips: count reads that wait for the device */
   uint64_t arena_bytes_used;   /* high-water mark of the caller arena (lt_config.arena), 0 without one */
 } lt_stats;

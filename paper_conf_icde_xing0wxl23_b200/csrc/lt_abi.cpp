@@ -738,6 +738,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.spill_d2h_bytes = 0;
   ctx->stats.spill_h2d_bytes = 0;
   ctx->stats.host_chunks_peak = 0;
+  ctx->stats.spill_prefetched_chunks = 0;
   ctx->stats.load_ms = 0;
   ctx->stats.spill_xfer_ms = 0;
   ctx->stats.host_syncs = 0;
@@ -752,36 +753,18 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
     if (sp.on) {
       const uint64_t host_cap = (W + C - 1) / C + ctx->nb + 2;
       if (sp.host_cap < host_cap) {
-        if (sp.xfer) CK(cudaStreamSynchronize(sp.xfer));
-        if (sp.xfer_in) CK(cudaStreamSynchronize(sp.xfer_in));
+        CK(cudaStreamSynchronize(ctx->stream));
         if (sp.h_store) cudaFreeHost(sp.h_store);
         sp.h_store = nullptr;
+        sp.d_store = nullptr;
         sp.host_cap = 0;
-        CK(cudaHostAlloc((void**)&sp.h_store, host_cap * C * sizeof(uint4), cudaHostAllocPortable));
+        CK(cudaHostAlloc((void**)&sp.h_store, host_cap * C * sizeof(uint4), cudaHostAllocPortable | cudaHostAllocMapped));
+        CK(cudaHostGetDevicePointer((void**)&sp.d_store, sp.h_store, 0));
         sp.host_cap = host_cap;
       }
-      for (int b = 0; b < 2; ++b) {
-        CK(ensure(ctx, sp.d_stage[b], sp.stage_cap[b], (size_t)lt::kSpillBatch * C));
-        if (!sp.ev_ready[b]) CK(cudaEventCreateWithFlags(&sp.ev_ready[b], cudaEventDisableTiming));
-        if (!sp.ev_free[b]) CK(cudaEventCreateWithFlags(&sp.ev_free[b], cudaEventDisableTiming));
-      }
-      if (!sp.xfer) CK(cudaStreamCreateWithFlags(&sp.xfer, cudaStreamNonBlocking));
-      if (!sp.xfer_in) CK(cudaStreamCreateWithFlags(&sp.xfer_in, cudaStreamNonBlocking));
-      while (sp.xev.size() < (size_t)lt::Spill::kXferEvents) {
-        cudaEvent_t ev;
-        CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-        sp.xev.push_back(ev);
-      }
-      if (sp.used[0] || sp.used[1]) {  // the previous epoch's transfers
-        CK(cudaStreamSynchronize(sp.xfer));
-        CK(cudaStreamSynchronize(sp.xfer_in));
-      }
-      sp.used[0] = sp.used[1] = false;
-      sp.next = 0;
       sp.spilled.assign(ctx->nb, {});
       sp.host_free.resize(sp.host_cap);
       for (uint64_t i = 0; i < sp.host_cap; ++i) sp.host_free[i] = (uint32_t)(sp.host_cap - 1 - i);
-      sp.slot_ev.assign(sp.host_cap, -1);
       sp.host_used = 0;
       sp.free_chunks = (int64_t)num_chunks;
     }
@@ -870,8 +853,6 @@ lt_status lt_run(lt_ctx* ctx) {
     if (ctx->ooc.load_stream) CK(cudaStreamSynchronize(ctx->ooc.load_stream));
     CK(ctx->load_ev.total_ms(&t));
     ctx->stats.load_ms += t;
-    if (ctx->spill.xfer) CK(cudaStreamSynchronize(ctx->spill.xfer));
-    if (ctx->spill.xfer_in) CK(cudaStreamSynchronize(ctx->spill.xfer_in));
     CK(ctx->xfer_ev.total_ms(&t));
     ctx->stats.spill_xfer_ms += t;
   }

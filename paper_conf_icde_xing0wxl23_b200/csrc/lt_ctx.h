@@ -61,31 +61,18 @@ struct OutOfCore {
 
 // Walk spill (lt_config.walk_spill): the walk pool keeps at most its
 // num_chunks chunks on the device; full chunks of buckets with the fewest pending walks are evicted to a
-// pinned host store (PAPER.md:118 "evict a batch when full", :202 "the same way") and loaded back before
-// their partition is computed. Evictions (D2H) run on `xfer`, reloads (H2D) on `xfer_in` — full duplex over
-// PCIe — through two staging buffers of kSpillBatch chunks.
+// pinned, MAPPED host store (PAPER.md:118 "evict a batch when full", :202 "the same way") and loaded back
+// before their partition is computed. The copies are kernels (k_spill / k_reload, a block per chunk)
+// that read and write the host store through its device mapping: no staging buffers and no per-chunk
+// cudaMemcpy calls (a 128-KB memcpy ran at ~40 % of the link, measured).
 struct Spill {
   bool on = false;
-  uint4* h_store = nullptr;                 // pinned host chunk slots (host_cap x C records)
+  uint4* h_store = nullptr;                 // pinned + mapped host chunk slots (host_cap x C records)
+  uint4* d_store = nullptr;                 // its device view
   uint64_t host_cap = 0;
   std::vector<uint32_t> host_free;          // free host slots
   std::vector<std::map<uint64_t, uint32_t>> spilled;  // per bucket: chunk index -> host slot
   uint64_t host_used = 0;
-  uint4* d_stage[2] = {nullptr, nullptr};
-  size_t stage_cap[2] = {0, 0};
-  cudaStream_t xfer = nullptr;     // evictions: D2H of staged chunks into host slots
-  cudaStream_t xfer_in = nullptr;  // reloads: H2D of host slots into staging (full duplex with evictions, :190)
-  // ordering of the two transfer streams per host slot: slot_ev[s] = the event (ring of kXferEvents, reused
-  // round robin: a reused event only makes a waiter wait longer) of the last transfer that wrote (D2H) or
-  // read (H2D) host slot s; the next transfer of that slot on the other stream waits for it
-  static constexpr int kXferEvents = 64;
-  std::vector<cudaEvent_t> xev;
-  int xev_next = 0;
-  std::vector<int> slot_ev;
-  cudaEvent_t ev_ready[2] = {nullptr, nullptr};  // stage b's contents are complete (recorded by its producer)
-  cudaEvent_t ev_free[2] = {nullptr, nullptr};   // stage b may be overwritten (recorded by its consumer)
-  bool used[2] = {false, false};
-  int next = 0;
   int64_t free_chunks = 0;                  // host mirror of the device free stack, kept exact between snapshots
 };
 
@@ -162,7 +149,7 @@ struct lt_ctx {
   size_t bounds_cap = 0;
   lt::OutOfCore ooc;
   lt::Spill spill;
-  lt::PhaseEvents load_ev, xfer_ev;  // graph loads (load stream), walk-spill transfers (spill stream)
+  lt::PhaseEvents load_ev, xfer_ev;  // graph loads (load stream), walk-spill copy kernels (compute stream)
   // caller-owned arena (lt_config.arena): [arena, arena + arena_size), bump pointer arena_top; buffers
   // from ensure() registered in arena_bufs are dropped when a graph load resets the arena to arena_mark
   char* arena = nullptr;

@@ -127,6 +127,7 @@ struct Params {
 constexpr uint32_t kSpillBatch = 64;
 struct SpillList {
   uint32_t bucket[kSpillBatch];
+  uint32_t slot[kSpillBatch];             // host store slot
   unsigned long long chunk[kSpillBatch];  // chunk index within the bucket (position / C)
 };
 
@@ -150,9 +151,10 @@ cudaError_t launch_check_col(const uint32_t* col, uint64_t m, uint32_t n, uint32
 cudaError_t launch_check_starts(const uint32_t* starts, uint64_t W, uint32_t n, uint32_t* bad, cudaStream_t s);
 cudaError_t launch_pool_reset(const Params& p, cudaStream_t s);
 cudaError_t launch_philox_blocks(const uint4* ctr, const uint2* key, uint4* out, uint64_t n, cudaStream_t s);
-// walk spill: chunks list[0..count) -> stage (ring slots marked kSpilled, chunks freed) / stage -> fresh chunks
-cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* stage, cudaStream_t s);
-cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* stage, cudaStream_t s);
+// walk spill: chunks list[0..count) -> their host slots of `store` (the mapped host store; ring slots marked
+// kSpilled, device chunks freed) / host slots -> fresh device chunks installed in the ring
+cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* store, cudaStream_t s);
+cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* store, cudaStream_t s);
 // compact path output: (1) tile sums + their exclusive scan (total -> *total); (2) offsets[i] = base +
 // exclusive prefix of lengths for i < n, rows packed into vertices (indexed from 0 for this range)
 uint64_t paths_scan_tiles(uint64_t n);  // tile_sum entries launch_paths_scan needs

@@ -955,11 +955,12 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
 }
 
 // ------------------------------------------------------------------------- walk spill (f3, a8)
-// Eviction: block i copies chunk list[i] = (bucket, chunk index) of the ring
-// into staging slot i (coalesced 16-B records), marks the ring slot kSpilled and returns the device chunk
-// to the free stack. Only full chunks strictly inside [head, cursor) of a bucket that is not being
-// launched are listed, so no kernel reads or writes them while they live in host memory.
-__global__ void __launch_bounds__(256) k_spill(Params p, SpillList list, uint4* __restrict__ stage) {
+// Eviction: block i copies chunk list[i] = (bucket, chunk index) into host slot
+// list.slot[i] of the mapped host store (16-B stores over PCIe, 4 per thread in flight), marks the ring
+// slot kSpilled and returns the device chunk to the free stack. Only full chunks strictly inside
+// [head, cursor) of a bucket that is not being launched are listed, so no kernel reads or writes them while
+// they live in host memory.
+__global__ void __launch_bounds__(256) k_spill(Params p, SpillList list, uint4* __restrict__ store) {
   const Pool& pl = p.pool;
   __shared__ uint32_t s_c;
   uint32_t* slot = pl.ring + (uint64_t)list.bucket[blockIdx.x] * pl.ring_len + (list.chunk[blockIdx.x] % pl.ring_len);
@@ -967,8 +968,17 @@ __global__ void __launch_bounds__(256) k_spill(Params p, SpillList list, uint4* 
   __syncthreads();
   const uint32_t c = s_c;
   const uint4* src = pl.slots + ((uint64_t)c << pl.c_shift);
-  uint4* dst = stage + ((uint64_t)blockIdx.x << pl.c_shift);
-  for (uint32_t i = threadIdx.x; i < pl.C; i += blockDim.x) dst[i] = __ldcs(src + i);
+  uint4* dst = store + ((uint64_t)list.slot[blockIdx.x] << pl.c_shift);
+  for (uint32_t i = threadIdx.x; i < pl.C; i += 4 * blockDim.x) {
+    uint4 v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (i + u * blockDim.x < pl.C) v[u] = __ldcs(src + i + u * blockDim.x);
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (i + u * blockDim.x < pl.C) dst[i + u * blockDim.x] = v[u];
+  }
+  __threadfence_system();  // the host copy is complete before the chunk can be reused
   __syncthreads();
   if (threadIdx.x == 0) {
     *slot = kSpilled;
@@ -977,9 +987,9 @@ __global__ void __launch_bounds__(256) k_spill(Params p, SpillList list, uint4* 
   }
 }
 
-// Reload: block i pops a free device chunk, copies staging slot i into it and installs it in the ring
-// slot of list[i] (which holds kSpilled).
-__global__ void __launch_bounds__(256) k_reload(Params p, SpillList list, const uint4* __restrict__ stage) {
+// Reload: block i pops a free device chunk, copies host slot list.slot[i] into it (reads over PCIe, 4 per
+// thread in flight) and installs it in the ring slot of list[i] (which holds kSpilled).
+__global__ void __launch_bounds__(256) k_reload(Params p, SpillList list, const uint4* __restrict__ store) {
   const Pool& pl = p.pool;
   __shared__ uint32_t s_c;
   uint32_t* slot = pl.ring + (uint64_t)list.bucket[blockIdx.x] * pl.ring_len + (list.chunk[blockIdx.x] % pl.ring_len);
@@ -994,8 +1004,16 @@ __global__ void __launch_bounds__(256) k_reload(Params p, SpillList list, const 
   __syncthreads();
   const uint32_t c = s_c;
   uint4* dst = pl.slots + ((uint64_t)c << pl.c_shift);
-  const uint4* src = stage + ((uint64_t)blockIdx.x << pl.c_shift);
-  for (uint32_t i = threadIdx.x; i < pl.C; i += blockDim.x) dst[i] = __ldcs(src + i);
+  const uint4* src = store + ((uint64_t)list.slot[blockIdx.x] << pl.c_shift);
+  for (uint32_t i = threadIdx.x; i < pl.C; i += 4 * blockDim.x) {
+    uint4 v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (i + u * blockDim.x < pl.C) v[u] = __ldcv(src + i + u * blockDim.x);  // not cached: host memory
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (i + u * blockDim.x < pl.C) dst[i + u * blockDim.x] = v[u];
+  }
   __syncthreads();
   if (threadIdx.x == 0) *slot = c;
 }
@@ -1425,15 +1443,15 @@ cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t 
   return cudaGetLastError();
 }
 
-cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* stage, cudaStream_t s) {
+cudaError_t launch_spill(const Params& p, const SpillList& list, uint32_t count, uint4* store, cudaStream_t s) {
   if (!count) return cudaSuccess;
-  k_spill<<<count, 256, 0, s>>>(p, list, stage);
+  k_spill<<<count, 256, 0, s>>>(p, list, store);
   return cudaGetLastError();
 }
 
-cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* stage, cudaStream_t s) {
+cudaError_t launch_reload(const Params& p, const SpillList& list, uint32_t count, const uint4* store, cudaStream_t s) {
   if (!count) return cudaSuccess;
-  k_reload<<<count, 256, 0, s>>>(p, list, stage);
+  k_reload<<<count, 256, 0, s>>>(p, list, store);
   return cudaGetLastError();
 }
 

@@ -90,20 +90,11 @@ lt_status admit_walks(lt_ctx* ctx, uint64_t live, bool* did) {
 // cursor's chunk or later) — and q is not being launched; its ring slot then holds kSpilled and its
 // device chunk is free. A launch of partition k consumes [head_k, tail_cap): every chunk there is on the
 // device (tail_cap = the start of k's first chunk still on the host, or the prefix the free chunks can
-// absorb). Eviction: k_spill (compute stream) copies the chunks into a staging buffer, the D2H to their
-// host slots runs on the transfer stream. Reload: H2D into a staging buffer on the transfer stream, then
-// k_reload installs fresh device chunks. Two staging buffers alternate; events order their reuse.
+// absorb). Eviction: k_spill copies the chunks into their host slots through the host store's device
+// mapping and frees them (ring slot -> kSpilled); reload: k_reload copies host slots into fresh device
+// chunks and installs them. Both run on the compute stream, so host slots and device chunks are reused in
+// stream order, with no staging buffers and no per-chunk cudaMemcpy calls.
 namespace {
-
-// The writer stream of stage b waits until its previous consumer is done with it.
-int stage_take(lt_ctx* ctx, cudaStream_t writer) {
-  Spill& sp = ctx->spill;
-  const int b = sp.next;
-  sp.next ^= 1;
-  if (sp.used[b]) cudaStreamWaitEvent(writer, sp.ev_free[b], 0);
-  sp.used[b] = true;
-  return b;
-}
 
 // chunks a launch over n walks may need for its appends: one per C walks plus a partial tail chunk
 // per destination bucket
@@ -137,35 +128,9 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done, int
   auto flush = [&]() -> lt_status {
     if (!cnt) return LT_OK;
     const cudaStream_t s = ctx->stream;
-    const int b = stage_take(ctx, s);
-    CK(launch_spill(ctx->params, list, cnt, sp.d_stage[b], s));
-    CK(cudaEventRecord(sp.ev_ready[b], s));
-    CK(cudaStreamWaitEvent(sp.xfer, sp.ev_ready[b], 0));
-    uint32_t slots[kSpillBatch];
-    uint64_t waited = 0;  // bitmask of transfer events already waited for (64 = kXferEvents)
-    for (uint32_t i = 0; i < cnt; ++i) {
-      slots[i] = sp.host_free.back();
-      sp.host_free.pop_back();
-      const int e = sp.slot_ev[slots[i]];  // the reload that last read this slot must be done
-      if (e >= 0 && !(waited >> e & 1)) {
-        CK(cudaStreamWaitEvent(sp.xfer, sp.xev[e], 0));
-        waited |= 1ull << e;
-      }
-    }
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer));
-    for (uint32_t i = 0; i < cnt; ++i) {
-      CK(cudaMemcpyAsync(sp.h_store + (uint64_t)slots[i] * C, sp.d_stage[b] + (uint64_t)i * C, C * sizeof(uint4),
-                         cudaMemcpyDeviceToHost, sp.xfer));
-      sp.spilled[list.bucket[i]][list.chunk[i]] = slots[i];
-    }
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer));
-    CK(cudaEventRecord(sp.ev_free[b], sp.xfer));
-    {
-      const int e = sp.xev_next;
-      sp.xev_next = (sp.xev_next + 1) % Spill::kXferEvents;
-      CK(cudaEventRecord(sp.xev[e], sp.xfer));
-      for (uint32_t i = 0; i < cnt; ++i) sp.slot_ev[slots[i]] = e;
-    }
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(s));
+    CK(launch_spill(ctx->params, list, cnt, sp.d_store, s));
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(s));
     sp.host_used += cnt;
     sp.free_chunks += cnt;
     ctx->stats.spilled_chunks += cnt;
@@ -183,8 +148,12 @@ lt_status evict_chunks(lt_ctx* ctx, int keep, uint64_t want, uint64_t* done, int
     for (uint64_t ci = hi; ci-- > lo && *done < want;) {
       if (sp.spilled[q].count(ci)) continue;
       if (sp.host_free.empty()) return fail(LT_ERR_OOM, "walk spill: host store full (invariant violated)");
+      const uint32_t hs = sp.host_free.back();  // host slots are reused in stream order (kernels only)
+      sp.host_free.pop_back();
+      sp.spilled[q][ci] = hs;
       list.bucket[cnt] = q;
       list.chunk[cnt] = ci;
+      list.slot[cnt] = hs;
       ++*done;
       if (++cnt == kSpillBatch) {
         lt_status st = flush();
@@ -202,42 +171,21 @@ lt_status reload_chunks(lt_ctx* ctx, uint32_t k, uint64_t r) {
   Spill& sp = ctx->spill;
   const uint64_t C = ctx->params.pool.C;
   auto& sk = sp.spilled[k];
-  while (r) {
+  while (r && !sk.empty()) {
     SpillList list;
     uint32_t cnt = 0;
-    const int b = stage_take(ctx, sp.xfer_in);
-    uint32_t slots[kSpillBatch];
-    uint64_t waited = 0;
     for (auto it = sk.begin(); it != sk.end() && cnt < kSpillBatch && cnt < r;) {
       list.bucket[cnt] = k;
       list.chunk[cnt] = it->first;
-      slots[cnt] = it->second;
-      const int e = sp.slot_ev[it->second];  // the eviction that wrote this slot must be done
-      if (e >= 0 && !(waited >> e & 1)) {
-        CK(cudaStreamWaitEvent(sp.xfer_in, sp.xev[e], 0));
-        waited |= 1ull << e;
-      }
+      list.slot[cnt] = it->second;
+      sp.host_free.push_back(it->second);  // an eviction into this slot is stream-ordered after this reload
       it = sk.erase(it);
       ++cnt;
     }
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(sp.xfer_in));
-    for (uint32_t i = 0; i < cnt; ++i)
-      CK(cudaMemcpyAsync(sp.d_stage[b] + (uint64_t)i * C, sp.h_store + (uint64_t)slots[i] * C, C * sizeof(uint4),
-                         cudaMemcpyHostToDevice, sp.xfer_in));
-    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(sp.xfer_in));
-    CK(cudaEventRecord(sp.ev_ready[b], sp.xfer_in));
-    {
-      const int e = sp.xev_next;
-      sp.xev_next = (sp.xev_next + 1) % Spill::kXferEvents;
-      CK(cudaEventRecord(sp.xev[e], sp.xfer_in));
-      for (uint32_t i = 0; i < cnt; ++i) {
-        sp.slot_ev[slots[i]] = e;
-        sp.host_free.push_back(slots[i]);  // a later eviction into this slot waits for this H2D
-      }
-    }
-    CK(cudaStreamWaitEvent(ctx->stream, sp.ev_ready[b], 0));
-    CK(launch_reload(ctx->params, list, cnt, sp.d_stage[b], ctx->stream));
-    CK(cudaEventRecord(sp.ev_free[b], ctx->stream));
+    const cudaStream_t s = ctx->stream;
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.begin(s));
+    CK(launch_reload(ctx->params, list, cnt, sp.d_store, s));
+    if (ctx->cfg.timing) CK(ctx->xfer_ev.end(s));
     sp.host_used -= cnt;
     sp.free_chunks -= cnt;
     ctx->stats.reloaded_chunks += cnt;
@@ -330,17 +278,7 @@ lt_status spill_admit_all(lt_ctx* ctx) {
 
 void free_spill(lt_ctx* ctx) {
   Spill& sp = ctx->spill;
-  if (sp.xfer) cudaStreamSynchronize(sp.xfer);
-  if (sp.xfer_in) cudaStreamSynchronize(sp.xfer_in);
   if (sp.h_store) cudaFreeHost(sp.h_store);
-  for (int b = 0; b < 2; ++b) {
-    if (sp.d_stage[b]) dfree(ctx, sp.d_stage[b]);
-    if (sp.ev_ready[b]) cudaEventDestroy(sp.ev_ready[b]);
-    if (sp.ev_free[b]) cudaEventDestroy(sp.ev_free[b]);
-  }
-  if (sp.xfer) cudaStreamDestroy(sp.xfer);
-  if (sp.xfer_in) cudaStreamDestroy(sp.xfer_in);
-  for (auto e : sp.xev) cudaEventDestroy(e);
   sp = Spill();
 }
 
@@ -369,6 +307,31 @@ lt_status launch_update_timed(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t
   return LT_OK;
 }
 
+// Walk-spill prefetch: while partition k's launch runs, load back the evicted chunks of the partition
+// most likely to be computed next (the most pending walks, as the selective policy picks),
+// so its reload H2D overlaps k's compute instead of sitting in front of its own launch. Only chunks the
+// free pool can spare beyond k's appends (up to ⌈launched/C⌉ + nb + 1 chunks) are loaded; the reload
+// kernel is stream-ordered after k's launch. Parity-neutral: only residency changes.
+static lt_status prefetch_walks(lt_ctx* ctx, uint32_t k, uint64_t launched) {
+  Spill& sp = ctx->spill;
+  int j = -1;
+  uint64_t best = 0;
+  for (uint32_t q = ctx->own_lo; q < ctx->own_hi; ++q) {
+    if (q == k || sp.spilled[q].empty()) continue;
+    const uint64_t pend = ctx->h_hc[ctx->nb + q] - ctx->h_hc[q];
+    if (pend > best) {
+      best = pend;
+      j = (int)q;
+    }
+  }
+  if (j < 0) return LT_OK;
+  const int64_t spare = sp.free_chunks - (int64_t)append_chunks(ctx, launched) - (int64_t)ctx->nb - 2;
+  if (spare <= 0) return LT_OK;
+  const uint64_t r = std::min<uint64_t>((uint64_t)spare, sp.spilled[(uint32_t)j].size());
+  ctx->stats.spill_prefetched_chunks += r;
+  return reload_chunks(ctx, (uint32_t)j, r);
+}
+
 // One partition's update launch; with walk spill, as many launches as it takes to consume every walk
 // that was in bucket k when the call began (each preceded by ensure_walks).
 lt_status launch_partition(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t walks_bound) {
@@ -383,9 +346,10 @@ lt_status launch_partition(lt_ctx* ctx, const Params& p, uint32_t k, uint64_t wa
     if (first) end = cur;
     if (head >= end || head >= cur) return LT_OK;
     pv.tail_cap = cap;
-    st = launch_update_timed(ctx, pv, k, std::min<unsigned long long>(cap, cur) - head);
+    const unsigned long long launched = std::min<unsigned long long>(cap, cur) - head;
+    st = launch_update_timed(ctx, pv, k, launched);
     if (st != LT_OK) return st;
-    if (cap >= cur) return LT_OK;
+    if (cap >= cur) return prefetch_walks(ctx, k, launched);
   }
 }
 

@@ -82,7 +82,8 @@ class Stats(ctypes.Structure):
         (name, ctypes.c_uint64) for name in (
             "iterations", "explicit_copies", "pool_hits", "zero_copy_launches", "preemptive_launches",
             "graph_h2d_bytes", "pool_blocks", "pool_block_bytes", "admissions", "peak_live", "direct_start", "graph_device_bytes", "l2_persist_bytes", "prefetches",
-            "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak")] + [
+            "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak",
+            "spill_prefetched_chunks")] + [
         ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64),
         ("arena_bytes_used", ctypes.c_uint64)]
 

@@ -62,6 +62,7 @@ def test_spill_deepwalk_exact(gpu, g14, cap_div, P, refill):
     assert st["spill_d2h_bytes"] == st["spilled_chunks"] * C * 16 == st["spill_h2d_bytes"]
     assert st["chunks_total"] <= 2 * -(-(W // cap_div) // C) + 2 * P + 64  # sized by the cap, not by W
     assert st["host_chunks_peak"] > 0
+    assert st["spill_prefetched_chunks"] <= st["reloaded_chunks"]
 
 
 @pytest.mark.parametrize("app,param", [(LT.PPR, 0.15), (LT.PAGERANK, 0.2)])

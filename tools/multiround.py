@@ -81,10 +81,13 @@ def main():
                    "peak_live": st["peak_live"], "graph_h2d_gb": st["graph_h2d_bytes"] / 1e9,
                    "explicit_copies": st["explicit_copies"], "iterations": st["iterations"],
                    "chunks_total": st["chunks_total"], "update_launches": st["update_launches"]}
+            out.update(update_ms=st["update_ms"], run_ms=st["run_ms"], load_ms=st["load_ms"],
+                       host_syncs=st["host_syncs"])
             if spill:
                 out.update(spilled_chunks=st["spilled_chunks"], reloaded_chunks=st["reloaded_chunks"],
                            spill_d2h_gb=st["spill_d2h_bytes"] / 1e9, spill_h2d_gb=st["spill_h2d_bytes"] / 1e9,
-                           host_chunks_peak=st["host_chunks_peak"])
+                           host_chunks_peak=st["host_chunks_peak"], spill_xfer_ms=st["spill_xfer_ms"],
+                           spill_prefetched_chunks=st["spill_prefetched_chunks"])
             return out
 
         # (1) walk spill (every walk exists; the pool evicts to host memory) and (2) walk admission
