@@ -718,6 +718,14 @@ template <int APP> struct RfMinBlocks {
 #endif
 };
 
+#ifndef LT_RF_RINGCACHE
+#define LT_RF_RINGCACHE 1
+#endif
+#ifndef LT_RF_PRECLAIM
+#define LT_RF_PRECLAIM 1
+#endif
+constexpr uint32_t kRfRingCache = 2048;  // chunk ids of the launched bucket staged in shared memory (8 KB)
+
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
   const uint32_t lane = threadIdx.x & 31u;
@@ -771,6 +779,22 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   uint32_t q_cnt = 0;
 #pragma unroll
   for (int q = 0; q < 8; ++q) pb[q] = 0;
+#if LT_RF_RINGCACHE
+  // the chunk ids of the launched bucket's positions [head, tail), staged once per CTA: a refill then
+  // finds its record's chunk in shared memory instead of an L2 read in front of the record load
+  __shared__ uint32_t s_ring[kRfRingCache];
+  const unsigned long long cb = head >> pl.c_shift;
+  const unsigned long long ncb = tail > head ? ((tail - 1) >> pl.c_shift) - cb + 1 : 0;
+  const bool ring_cached = p.direct.count == 0 && ncb <= kRfRingCache;
+  if (ring_cached)
+    for (uint32_t i = threadIdx.x; i < ncb; i += blockDim.x) s_ring[i] = ring_k[(cb + i) % pl.ring_len];
+  __syncthreads();
+#endif
+#if LT_RF_PRECLAIM
+  // the warp's next claim is issued one range ahead, so its atomic's latency overlaps the steps
+  unsigned long long q_next = 0;
+  if (lane == 0) q_next = atomicAdd(claim, (unsigned long long)kRefill);
+#endif
 
   for (;;) {
     // ---- refill idle lanes from the warp's claimed range (claim kRefill more when it runs out)
@@ -778,7 +802,14 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
     while (need && !drained) {
       if (q_cur >= q_end) {
         unsigned long long base = 0;
+#if LT_RF_PRECLAIM
+        if (lane == 0) {
+          base = q_next;
+          q_next = atomicAdd(claim, (unsigned long long)kRefill);  // used one range later
+        }
+#else
         if (lane == 0) base = atomicAdd(claim, (unsigned long long)kRefill);
+#endif
         base = __shfl_sync(kFull, base, 0);
         q_cur = base;
         q_end = (base + kRefill < tail) ? base + kRefill : tail;
@@ -793,7 +824,11 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           if (wk.path_mode == 1) wk.paths[pos * wk.pitch] = rec.y;
           count_visit<VIS>(wk, rec.y, pol_last);  // the start is the walk's first visit
         } else {
+#if LT_RF_RINGCACHE
+          const uint32_t c = ring_cached ? s_ring[(pos >> pl.c_shift) - cb] : ring_k[(pos >> pl.c_shift) % pl.ring_len];
+#else
           const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
+#endif
           rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
         }
         has = true;
