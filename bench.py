@@ -489,8 +489,9 @@ def main():
     sector_eff = None
     prof = os.path.join(ROOT, "profiles", "update_kernel_traffic.json")
     if os.path.exists(prof):
-        pj = json.load(open(prof))
-        if pj.get("config_key") == f"cfg{args.config}-P{P}-layout{args.layout}" and not own and not ooc:
+        key = f"cfg{args.config}-P{P}-layout{args.layout}-{c['app']}"
+        pj = next((e for e in json.load(open(prof))["entries"] if e.get("config_key") == key), {})
+        if pj and not own and not ooc:
             traffic = pj.get("dram_bytes_per_launch")
             traffic_source = (f"static: ncu --set full capture {pj.get('source', 'profiles/update_kernel_traffic.json')} "
                               f"of this configuration ({pj.get('captured', 'see file')}), not measured in this run")

@@ -128,7 +128,10 @@ typedef struct lt_config {
                                  reserved at lt_walks_init* and zeroed there: every path entry (start
                                  included) adds 1 to its vertex. Read with lt_get_visit_counts*. The
                                  kernels count in u32 while no count can reach 2^32 (W * stride <
-                                 2^32) and widen at the end of lt_run; 2 -> always count in u64. */
+                                 2^32) and widen at the end of lt_run — with an augmented layout in
+                                 16-bit halves for the vertices below a hub degree (lt_stats.hub_deg),
+                                 a wrap detected exactly and recounted from the paths (an error under
+                                 path_mode 2); 2 -> always count in u64. */
   uint32_t continue_resident; /* out-of-core: 1 -> a walk leaving the launched partition for another
                                  partition resident in the graph pool keeps stepping there instead of
                                  being appended to its bucket (parity-neutral);
@@ -216,6 +219,11 @@ typedef struct lt_stats {
   double spill_xfer_ms;        /* walk-spill copy kernels (evictions + reloads over PCIe) */
   uint64_t host_syncs;         /* scheduler round trips: count reads that wait for the device */
   uint64_t arena_bytes_used;   /* high-water mark of the caller arena (lt_config.arena), 0 without one */
+  /* visit counting (lt_config.visit_counts = 1) of the last lt_walks_init + lt_run */
+  uint64_t hub_deg;            /* 0: u32/u64 counters; > 0: paired 16-bit counters for vertices of degree
+                                  < hub_deg, u32 for the rest (chosen at lt_walks_init) */
+  uint64_t visit_recounts;     /* 1 if a 16-bit counter wrapped and the counts were recomputed from the
+                                  paths at the end of lt_run (exact either way) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

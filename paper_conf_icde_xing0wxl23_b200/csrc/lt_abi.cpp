@@ -213,6 +213,8 @@ void lt_destroy(lt_ctx* ctx) {
   dfree(ctx, ctx->d_starts_all);
   dfree(ctx, ctx->d_visits);
   dfree(ctx, ctx->d_visits32);
+  dfree(ctx, ctx->d_visits16);
+  dfree(ctx, ctx->d_vsum);
   dfree(ctx, ctx->d_slots);
   dfree(ctx, ctx->d_ring);
   dfree(ctx, ctx->d_hc);
@@ -363,7 +365,10 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     CK(cudaMemcpy(ctx->d_owner, own.data(), P * sizeof(uint16_t), cudaMemcpyHostToDevice));
   }
   const size_t nb = ctx->nb;
-  CK(ensure(ctx, ctx->d_hc, ctx->hc_cap, 3 * nb));  // head, cursor, refill claim
+  // head, cursor, refill claim of bucket b in block b of hs u64 (Pool::hs): 256 B per bucket while there
+  // are few buckets (each insertion cursor on its own L2 line), 32 B beyond
+  ctx->hs = nb <= 4096 ? 32 : 4;
+  CK(ensure(ctx, ctx->d_hc, ctx->hc_cap, ctx->hs * nb));
   if (ctx->h_hc_cap < 2 * nb) {
     if (ctx->h_hc) cudaFreeHost(ctx->h_hc);
     ctx->h_hc = nullptr;
@@ -637,6 +642,28 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   const bool narrow = ctx->cfg.visit_counts == 1 && (uint64_t)W * stride < 0xFFFFFFFFull;
   if (ctx->cfg.visit_counts) CK(ensure(ctx, ctx->d_visits, ctx->visits_cap, ctx->n));
   if (narrow) CK(ensure(ctx, ctx->d_visits32, ctx->visits32_cap, ctx->n));
+  // Paired 16-bit counters for the non-hub vertices (VIS 3, DESIGN.md §7 "PageRank and visit counts"):
+  // with an augmented layout (the step knows the visited vertex's degree), one rank, the graph resident.
+  // A hub is a vertex whose expected count could approach 2^16: with Nt = W * stride path entries at most
+  // and the walk's arrival rate at v about deg(v) / m per step (+ alpha / n per step for restarts, + the
+  // starts), deg >= hub_deg keeps every non-hub's expected count <= 4096 (16x below the wrap). A wrap is
+  // still possible (e.g. all starts on one low-degree vertex); it is detected exactly and recounted.
+  uint32_t hub_deg = 0;
+  bool half = false;
+  if (narrow && ctx->world == 1 && !ctx->ooc.on && (ctx->d_adj || ctx->d_adj12) && ctx->cfg.gather_mode == 3 &&
+      ctx->m && W) {
+    const double Nt = (double)W * stride;
+    const double rest = (app == LT_APP_PAGERANK ? Nt * alpha : 0.0) / ctx->n + (double)W / ctx->n;
+    const double h = (4096.0 - rest) * (double)ctx->m / Nt;
+    if (h >= 64.0) {
+      half = true;
+      hub_deg = h > 4e9 ? 0xFFFFFFFFu : (uint32_t)h;
+    }
+  }
+  if (half) {
+    CK(ensure(ctx, ctx->d_visits16, ctx->visits16_cap, (ctx->n + 1) / 2));
+    CK(ensure(ctx, ctx->d_vsum, ctx->vsum_cap, 1));
+  }
   if (on_device == 1 && W) {
     CK(cudaMemsetAsync(ctx->d_small + 2, 0, sizeof(uint32_t), s));
     CK(lt::launch_check_starts(d_starts, W, ctx->n, ctx->d_small + 2, s));
@@ -670,6 +697,10 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.wk.n = ctx->n;
   p.wk.visits = ctx->cfg.visit_counts ? ctx->d_visits : nullptr;
   p.wk.visits32 = narrow ? ctx->d_visits32 : nullptr;
+  p.wk.visits16 = half ? ctx->d_visits16 : nullptr;
+  p.wk.hub_deg = hub_deg;
+  ctx->stats.hub_deg = hub_deg;
+  ctx->stats.visit_recounts = 0;
   p.pool.slots = ctx->d_slots;
   p.pool.C = (uint32_t)C;
   p.pool.c_shift = c_shift;
@@ -678,8 +709,9 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.pool.ring_len = (uint32_t)ring_len;
   p.pool.nbuckets = ctx->nb;
   p.pool.head = ctx->d_hc;
-  p.pool.cursor = ctx->d_hc + ctx->nb;
-  p.pool.claim = ctx->d_hc + 2 * (size_t)ctx->nb;
+  p.pool.cursor = ctx->d_hc + 1;
+  p.pool.claim = ctx->d_hc + 2;
+  p.pool.hs = ctx->hs;
   p.own.own_lo = ctx->own_lo;
   p.own.own_hi = ctx->own_hi;
   p.own.owner = ctx->d_owner;
@@ -778,6 +810,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // where the walk ends; the rows are padded lazily by the first copy-out, R24).
   if (W && !home && !ctx->is_home) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
   if (narrow) CK(cudaMemsetAsync(ctx->d_visits32, 0, (size_t)ctx->n * sizeof(uint32_t), s));
+  if (half) CK(cudaMemsetAsync(ctx->d_visits16, 0, (size_t)((ctx->n + 1) / 2) * sizeof(uint32_t), s));
   else if (ctx->cfg.visit_counts) CK(cudaMemsetAsync(ctx->d_visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
@@ -830,7 +863,12 @@ lt_status lt_run(lt_ctx* ctx) {
   // Path rows hold entries 0..length-1; the 0xFFFFFFFF padding of the rest is output formatting and is
   // written lazily by the first copy-out (ensure_padded). With ownership the rows were pre-filled.
   ctx->padded = ctx->world > 1 && !ctx->is_home;
-  if (ctx->params.wk.visits32) {  // the result is u64[n]
+  if (ctx->params.wk.visits16) {  // the result is u64[n]; the sum of all counts checks for a 16-bit wrap
+    CK(cudaMemsetAsync(ctx->d_vsum, 0, sizeof(unsigned long long), s));
+    CK(lt::launch_widen16(ctx->params.wk.visits16, ctx->params.wk.visits32, ctx->d_row_ptr, ctx->params.wk.hub_deg,
+                          ctx->params.wk.visits, ctx->n, ctx->d_vsum, s));
+    ctx->stats.kernel_launches++;
+  } else if (ctx->params.wk.visits32) {  // the result is u64[n]
     CK(lt::launch_widen(ctx->params.wk.visits32, ctx->params.wk.visits, ctx->n, s));
     ctx->stats.kernel_launches++;
   }
@@ -859,6 +897,24 @@ lt_status lt_run(lt_ctx* ctx) {
   ctx->stats.steps = ctx->h_ctr->steps;
   ctx->stats.visits = ctx->h_ctr->visits;
   ctx->stats.truncated = ctx->h_ctr->truncated;
+  if (ctx->params.wk.visits16) {
+    // every walk has 1 + (its steps) path entries; a wrapped 16-bit half loses 2^16 (or 2^16 - 1 with the
+    // carry into its neighbour) from the sum, so sum == entries iff nothing wrapped
+    unsigned long long sum = 0;
+    CK(cudaMemcpy(&sum, ctx->d_vsum, sizeof(sum), cudaMemcpyDeviceToHost));
+    const unsigned long long entries = ctx->h_ctr->steps + ctx->W;
+    ctx->stats.visit_recounts = 0;
+    if (sum != entries) {
+      if (ctx->cfg.path_mode == 2)
+        return fail(LT_ERR_INVALID, "a 16-bit visit counter wrapped and path_mode 2 keeps no paths to recount "
+                                    "from; set visit_counts = 2 (u64 counters)");
+      CK(cudaMemsetAsync(ctx->params.wk.visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
+      CK(lt::launch_recount(ctx->params.wk.paths, ctx->params.wk.pitch, ctx->params.wk.lengths, ctx->W,
+                            ctx->params.wk.visits, s));
+      CK(cudaStreamSynchronize(s));
+      ctx->stats.visit_recounts = 1;
+    }
+  }
   ctx->ran = true;
   ctx->visits_ready = ctx->cfg.visit_counts != 0;
   if (ctx->h_ctr->err & lt::kErrOOM) return fail(LT_ERR_CUDA, "walk pool exhausted on the device (invariant violated)");
@@ -1015,8 +1071,12 @@ lt_status lt_get_pool_state(lt_ctx* ctx, lt_pool_state* out) {
   CK(cudaMemcpy(&c, ctx->d_ctr, sizeof(c), cudaMemcpyDeviceToHost));
   std::vector<uint32_t> ring((size_t)ctx->nb * p.pool.ring_len);
   CK(cudaMemcpy(ring.data(), ctx->d_ring, ring.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
-  std::vector<unsigned long long> hc(2 * (size_t)ctx->nb);
-  CK(cudaMemcpy(hc.data(), ctx->d_hc, hc.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+  std::vector<unsigned long long> hcs((size_t)ctx->nb * ctx->hs), hc(2 * (size_t)ctx->nb);
+  CK(cudaMemcpy(hcs.data(), ctx->d_hc, hcs.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+  for (size_t b = 0; b < ctx->nb; ++b) {
+    hc[b] = hcs[b * ctx->hs];
+    hc[ctx->nb + b] = hcs[b * ctx->hs + 1];
+  }
   std::vector<uint32_t> len(ctx->W);
   if (ctx->W) CK(cudaMemcpy(len.data(), ctx->d_lengths, ctx->W * sizeof(uint32_t), cudaMemcpyDeviceToHost));
   out->free_chunks = small[0];

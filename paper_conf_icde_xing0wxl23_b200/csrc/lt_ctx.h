@@ -177,6 +177,11 @@ struct lt_ctx {
   size_t visits_cap = 0;
   uint32_t* d_visits32 = nullptr;          // [n] narrow counters (while counts fit in u32)
   size_t visits32_cap = 0;
+  uint32_t* d_visits16 = nullptr;          // [ceil(n/2)] paired 16-bit counters (VIS 3)
+  size_t visits16_cap = 0;
+  unsigned long long* d_vsum = nullptr;    // [1] sum of the widened counts (VIS 3 wrap check)
+  size_t vsum_cap = 0;
+  uint64_t vis_entries = 0;                // path entries of the current walks (W + steps), for the check
   bool visits_ready = false;
   uint32_t* d_starts = nullptr;
   size_t starts_cap = 0;
@@ -193,6 +198,7 @@ struct lt_ctx {
   size_t ring_cap = 0;
   unsigned long long* d_hc = nullptr;  // head[P] then cursor[P]
   size_t hc_cap = 0;
+  uint32_t hs = 32;  // u64 per bucket block in d_hc (Pool::hs)
   uint32_t* d_free = nullptr;
   size_t free_cap = 0;
   uint32_t* d_small = nullptr;  // [0]=free_top [1]=unused [2..3]=scratch flags

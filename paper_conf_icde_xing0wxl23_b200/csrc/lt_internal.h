@@ -27,9 +27,13 @@ struct Pool {
   uint32_t* ring;
   uint32_t ring_len;
   uint32_t nbuckets;              // P partition buckets + one send bucket per other rank
-  unsigned long long* head;       // [nbuckets]
-  unsigned long long* cursor;     // [nbuckets]
-  unsigned long long* claim;      // [nbuckets] refill claims within a launch (== head between launches)
+  // Bucket b's head / cursor / claim are head[b * hs], cursor[b * hs], claim[b * hs] (one block of hs
+  // u64 per bucket: cursor = head + 1, claim = head + 2). hs = 32 (256 B) while the buckets are few, so
+  // every bucket's cursor — the target of every insertion atomic — has its own L2 line and slice.
+  unsigned long long* head;
+  unsigned long long* cursor;
+  unsigned long long* claim;      // refill claims within a launch (== head between launches)
+  uint32_t hs;
   uint32_t* free_list;            // [num_chunks]
   int* free_top;
 };
@@ -57,7 +61,10 @@ struct Walk {
   uint32_t n;                     // |V|: a PageRank restart draws its vertex from [0, n)
   unsigned long long* visits;     // [n] per-vertex visit counts or nullptr (off)
   uint32_t* visits32;             // [n] narrow counters used instead while every count fits in u32
-                                  // (W * stride < 2^32); widened into `visits` at the end of lt_run
+                                  // (W * stride < 2^32); widened into `visits` at the end of lt_run;
+                                  // with visits16: the hub counters (degree >= hub_deg)
+  uint32_t* visits16;             // [ceil(n/2)] paired 16-bit counters of the non-hub vertices, or nullptr
+  uint32_t hub_deg;               // degree from which a vertex counts in visits32 (visits16 on)
 };
 
 struct Counters {
@@ -143,7 +150,7 @@ cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t b
 cudaError_t launch_finalize_paths(const Params& p, uint64_t W, cudaStream_t s);
 cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, uint64_t count,
                                uint32_t* out_paths, uint32_t* out_lengths, cudaStream_t s);
-cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Counters* ctr, const int* free_top,
+cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t nb, uint32_t hs, const Counters* ctr, const int* free_top,
                             unsigned long long* out_hc, Counters* out_ctr, int* out_free, cudaStream_t s);
 cudaError_t launch_compact_rows(const uint32_t* paths, const uint32_t* lengths, uint64_t pitch, uint64_t stride,
                                 uint64_t n, uint32_t* out, cudaStream_t s);
@@ -167,6 +174,11 @@ cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_
                              cudaStream_t s);  // table[idx[i]] = val[i], count <= kTableSetMax
 constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
+cudaError_t launch_widen16(const uint32_t* v16, const uint32_t* v32, const unsigned long long* row_ptr,
+                           uint32_t hub_deg, unsigned long long* dst, uint64_t n, unsigned long long* sum,
+                           cudaStream_t s);
+cudaError_t launch_recount(const uint32_t* paths, uint64_t pitch, const uint32_t* lengths, uint64_t W,
+                           unsigned long long* dst, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
                              cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,

@@ -115,7 +115,7 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
   const uint32_t lane = threadIdx.x & 31u;
   const unsigned long long cmask = pl.C - 1;
   if (p.insert_mode == 1) {  // "direct write" ablation: one global atomic per walk
-    const unsigned long long pos = atomicAdd(pl.cursor + dest, 1ull);
+    const unsigned long long pos = atomicAdd(pl.cursor + (uint64_t)dest * pl.hs, 1ull);
     const uint32_t c = (pos & cmask) == 0 ? install_chunk(p, dest, pos >> pl.c_shift)
                                           : wait_chunk(p, dest, pos >> pl.c_shift);
     pl.slots[((uint64_t)c << pl.c_shift) | (pos & cmask)] = rec;
@@ -141,7 +141,7 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
   uint32_t c0 = 0, c1 = 0;
   if (lane == leader) {
     const uint32_t cnt = __popc(grp);  // cnt <= 32 <= C: the range touches at most two chunks
-    base = atomicAdd(pl.cursor + dest, (unsigned long long)cnt);
+    base = atomicAdd(pl.cursor + (uint64_t)dest * pl.hs, (unsigned long long)cnt);
     const unsigned long long ci0 = base >> pl.c_shift, ci1 = (base + cnt - 1) >> pl.c_shift;
     if (ci1 != ci0) c1 = install_chunk(p, dest, ci1);  // chunk ci1 starts inside our range
     c0 = (base & cmask) == 0 ? install_chunk(p, dest, ci0) : wait_chunk(p, dest, ci0);
@@ -221,8 +221,8 @@ __device__ void last_cta_retire(const Params& p, int k, unsigned long long head,
   __syncthreads();
   if (threadIdx.x == 0) {
     if (k >= 0) {
-      pl.head[k] = tail;
-      pl.claim[k] = tail;  // refill claims may have run past the snapshot
+      pl.head[(uint64_t)k * pl.hs] = tail;
+      pl.claim[(uint64_t)k * pl.hs] = tail;  // refill claims may have run past the snapshot
       atomicAdd(&p.ctr->visits, tail - head);
     }
     *(volatile uint32_t*)&p.ctr->done_ctas = 0;
@@ -270,7 +270,11 @@ __global__ void __launch_bounds__(256) k_init(Params p, const uint32_t* __restri
         // path[w][0]: with buffered path stores (path_mode 0) the update kernel writes the walk's first
         // sector, entry 0 included, on the walk's first visit, so only the per-step mode stores it here
         if (wk.path_mode == 1) wk.paths[i * wk.pitch] = v;
-        if (wk.visits32) atomicAdd(wk.visits32 + v, 1u);  // the start is the walk's first visit
+        if (wk.visits16) {  // the start is the walk's first visit (VIS 3: the counter by degree)
+          const uint32_t dg = (uint32_t)(__ldg(wk.row_ptr + v + 1) - __ldg(wk.row_ptr + v));
+          if (dg >= wk.hub_deg) atomicAdd(wk.visits32 + v, 1u);
+          else atomicAdd(wk.visits16 + (v >> 1), (v & 1u) ? 0x10000u : 1u);
+        } else if (wk.visits32) atomicAdd(wk.visits32 + v, 1u);
         else if (wk.visits) atomicAdd(wk.visits + v, 1ull);
         rec = make_uint4((uint32_t)i, v, 0u, 0u);
       }
@@ -311,7 +315,7 @@ __global__ void __launch_bounds__(256) k_insert_records(Params p, const uint4* _
 // and retire its chunks.
 __global__ void __launch_bounds__(256) k_pack(Params p, uint32_t bucket, uint4* __restrict__ out) {
   const Pool& pl = p.pool;
-  const unsigned long long head = pl.head[bucket], tail = pl.cursor[bucket];
+  const unsigned long long head = pl.head[(uint64_t)bucket * pl.hs], tail = pl.cursor[(uint64_t)bucket * pl.hs];
   const uint32_t* ring_b = pl.ring + (uint64_t)bucket * pl.ring_len;
   for (unsigned long long pos = head + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; pos < tail;
        pos += (uint64_t)gridDim.x * blockDim.x) {
@@ -481,8 +485,24 @@ template <> struct MinBlocks<4> { static constexpr int v = 2; };
 #ifndef LT_VIS_HINT
 #define LT_VIS_HINT 1
 #endif
+// VIS 3 (round 2): two 16-bit counters per 32-bit word (vertex v in half v & 1 of word v >> 1; the
+// n/2-word array is half the size of the u32 one, so far more of it stays in L2), except for hub vertices
+// (degree >= wk.hub_deg, whose expected count is too large for 16 bits), which count in the u32 array.
+// The degree of the visited vertex comes with the step (the augmented entry), so choosing costs no load.
+// A 16-bit half that wraps is detected exactly at the end of lt_run (the sum of all counts falls short of
+// the number of path entries) and the counts are then recomputed from the paths.
 template <int VIS>
-__device__ __forceinline__ void count_visit(const Walk& wk, uint32_t v, uint64_t pol_last) {
+__device__ __forceinline__ void count_visit(const Walk& wk, uint32_t v, uint32_t deg, uint64_t pol_last) {
+  if (VIS == 3) {
+    if (deg >= wk.hub_deg)
+      asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], 1, %1;" :: "l"(wk.visits32 + v), "l"(pol_last)
+                   : "memory");
+    else
+      asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], %1, %2;" :: "l"(wk.visits16 + (v >> 1)),
+                   "r"((v & 1u) ? 0x10000u : 1u), "l"(pol_last) : "memory");
+    return;
+  }
+  (void)deg;
 #if LT_VIS_HINT
   if (VIS == 1)
     asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u64 [%0], 1, %1;" :: "l"(wk.visits + v), "l"(pol_last)
@@ -508,10 +528,11 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
   const Walk& wk = p.wk;
   const Pool& pl = p.pool;
   const uint32_t* B = stage_bounds(wk, s_bounds);
-  const unsigned long long head = pl.head[k];
+  const unsigned long long head = pl.head[(uint64_t)k * pl.hs];
   // no appends to bucket k during its own launch; a spill-limited launch stops at tail_cap (the first
   // position of the bucket's first chunk still in host memory)
-  const unsigned long long tail = pl.cursor[k] < p.tail_cap ? pl.cursor[k] : p.tail_cap;
+  const unsigned long long cur_k = pl.cursor[(uint64_t)k * pl.hs];
+  const unsigned long long tail = cur_k < p.tail_cap ? cur_k : p.tail_cap;
   const uint32_t lo = wk.bounds[k];
   const uint32_t span = wk.bounds[k + 1] - lo;
   const uint32_t lane = threadIdx.x & 31u;
@@ -613,8 +634,8 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
                                    : (uint32_t)(m >> 32);
           if (restart) {
             nv[s] = idx;
-            kn[s] = LAY != 0 && idx - lo < span;
-            if (kn[s]) {  // staying: the next step needs its offset and degree
+            kn[s] = LAY != 0 && (idx - lo < span || VIS == 3);
+            if (kn[s]) {  // staying (or VIS 3: its degree picks the counter): its offset and degree
               off[s] = __ldg(wk.row_ptr + idx);
               d[s] = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off[s]);
             }
@@ -638,7 +659,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
         if (alive[s]) {
           rec[s].y = nv[s];
           rec[s].z += 1;
-          count_visit<VIS>(wk, nv[s], pol_last);
+          count_visit<VIS>(wk, nv[s], d[s], pol_last);
           const uint32_t t = rec[s].z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -718,14 +739,6 @@ template <int APP> struct RfMinBlocks {
 #endif
 };
 
-#ifndef LT_RF_RINGCACHE
-#define LT_RF_RINGCACHE 1
-#endif
-#ifndef LT_RF_PRECLAIM
-#define LT_RF_PRECLAIM 1
-#endif
-constexpr uint32_t kRfRingCache = 2048;  // chunk ids of the launched bucket staged in shared memory (8 KB)
-
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
   const uint32_t lane = threadIdx.x & 31u;
@@ -748,13 +761,14 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   const Walk& wk = p.wk;
   const Pool& pl = p.pool;
   const uint32_t* B = stage_bounds(wk, s_bounds);
-  const unsigned long long head = pl.head[k];
-  const unsigned long long tail = pl.cursor[k] < p.tail_cap ? pl.cursor[k] : p.tail_cap;
+  const unsigned long long head = pl.head[(uint64_t)k * pl.hs];
+  const unsigned long long cur_k = pl.cursor[(uint64_t)k * pl.hs];
+  const unsigned long long tail = cur_k < p.tail_cap ? cur_k : p.tail_cap;
   const uint32_t lo = wk.bounds[k];
   const uint32_t span = wk.bounds[k + 1] - lo;
   const uint32_t lane = threadIdx.x & 31u;
   const uint32_t* ring_k = pl.ring + (uint64_t)k * pl.ring_len;
-  unsigned long long* claim = pl.claim + k;
+  unsigned long long* claim = pl.claim + (uint64_t)k * pl.hs;
   const Policies pol = make_policies();
   const uint64_t pol_last = VIS ? make_evict_last() : 0;
   unsigned long long my_steps = 0, my_trunc = 0;
@@ -779,22 +793,6 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   uint32_t q_cnt = 0;
 #pragma unroll
   for (int q = 0; q < 8; ++q) pb[q] = 0;
-#if LT_RF_RINGCACHE
-  // the chunk ids of the launched bucket's positions [head, tail), staged once per CTA: a refill then
-  // finds its record's chunk in shared memory instead of an L2 read in front of the record load
-  __shared__ uint32_t s_ring[kRfRingCache];
-  const unsigned long long cb = head >> pl.c_shift;
-  const unsigned long long ncb = tail > head ? ((tail - 1) >> pl.c_shift) - cb + 1 : 0;
-  const bool ring_cached = p.direct.count == 0 && ncb <= kRfRingCache;
-  if (ring_cached)
-    for (uint32_t i = threadIdx.x; i < ncb; i += blockDim.x) s_ring[i] = ring_k[(cb + i) % pl.ring_len];
-  __syncthreads();
-#endif
-#if LT_RF_PRECLAIM
-  // the warp's next claim is issued one range ahead, so its atomic's latency overlaps the steps
-  unsigned long long q_next = 0;
-  if (lane == 0) q_next = atomicAdd(claim, (unsigned long long)kRefill);
-#endif
 
   for (;;) {
     // ---- refill idle lanes from the warp's claimed range (claim kRefill more when it runs out)
@@ -802,14 +800,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
     while (need && !drained) {
       if (q_cur >= q_end) {
         unsigned long long base = 0;
-#if LT_RF_PRECLAIM
-        if (lane == 0) {
-          base = q_next;
-          q_next = atomicAdd(claim, (unsigned long long)kRefill);  // used one range later
-        }
-#else
         if (lane == 0) base = atomicAdd(claim, (unsigned long long)kRefill);
-#endif
         base = __shfl_sync(kFull, base, 0);
         q_cur = base;
         q_end = (base + kRefill < tail) ? base + kRefill : tail;
@@ -819,16 +810,13 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
       const uint32_t r = __popc(need & lanemask_lt());
       if (!has && r < avail) {
         const unsigned long long pos = q_cur + r;
+        bool sv_count = false;
         if (pos < p.direct.count) {  // direct start: the new walk's record, built in registers (a2)
           rec = make_uint4((uint32_t)pos, __ldg(p.direct.starts + pos), 0u, 0u);
           if (wk.path_mode == 1) wk.paths[pos * wk.pitch] = rec.y;
-          count_visit<VIS>(wk, rec.y, pol_last);  // the start is the walk's first visit
+          sv_count = true;  // the start is the walk's first visit (counted below, once its degree is known)
         } else {
-#if LT_RF_RINGCACHE
-          const uint32_t c = ring_cached ? s_ring[(pos >> pl.c_shift) - cb] : ring_k[(pos >> pl.c_shift) % pl.ring_len];
-#else
           const uint32_t c = ring_k[(pos >> pl.c_shift) % pl.ring_len];
-#endif
           rec = __ldcs(pl.slots + (((uint64_t)c << pl.c_shift) | (pos & (pl.C - 1))));
         }
         has = true;
@@ -841,6 +829,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           off = __ldg(wk.row_ptr + rec.y);
           d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
         }
+        if (sv_count) count_visit<VIS>(wk, rec.y, d, pol_last);
         if (CONT) {  // a walk from the bucket starts in the launched partition's view
           c_rp = wk.row_ptr - wk.vbase;
           c_col = wk.col - wk.ebase;
@@ -887,7 +876,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           uint32_t nv;
           if (restart) {
             nv = idx;
-            kn = LAY != 0 && idx - lo < span;
+            kn = LAY != 0 && (idx - lo < span || VIS == 3);
             if (kn) {
               off = __ldg(wk.row_ptr + idx);
               d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
@@ -907,7 +896,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           }
           rec.y = nv;
           rec.z += 1;
-          count_visit<VIS>(wk, nv, pol_last);
+          count_visit<VIS>(wk, nv, d, pol_last);
           const uint32_t t = rec.z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -988,6 +977,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
   last_cta_retire(p, (int)k, head, tail);
 }
+
 
 // ------------------------------------------------------------------------- walk spill (f3, a8)
 // Eviction: block i copies chunk list[i] = (bucket, chunk index) into host slot
@@ -1087,10 +1077,11 @@ __global__ void k_gather_rows(Params p, const unsigned long long* rows, uint64_t
 // Scheduler snapshot: head/cursor of every bucket, the counters and the free-stack top, written
 // by the SMs straight into mapped pinned host memory. A cudaMemcpy would queue behind a large D2H
 // on the same copy engine (lt_run_to_host's path copy-out) and serialise the pipeline.
-__global__ void k_snapshot(const unsigned long long* __restrict__ hc, uint64_t n, const Counters* __restrict__ ctr,
-                           const int* __restrict__ free_top, volatile unsigned long long* out_hc,
-                           volatile Counters* out_ctr, volatile int* out_free) {
-  for (uint64_t i = threadIdx.x; i < n; i += blockDim.x) out_hc[i] = hc[i];
+// out_hc[b] = head of bucket b, out_hc[nb + b] = its cursor (compact, from the strided device blocks)
+__global__ void k_snapshot(const unsigned long long* __restrict__ hc, uint64_t nb, uint32_t hs,
+                           const Counters* __restrict__ ctr, const int* __restrict__ free_top,
+                           volatile unsigned long long* out_hc, volatile Counters* out_ctr, volatile int* out_free) {
+  for (uint64_t i = threadIdx.x; i < 2 * nb; i += blockDim.x) out_hc[i] = hc[(i % nb) * hs + i / nb];
   if (threadIdx.x == 0) {
     out_ctr->steps = ctr->steps;
     out_ctr->visits = ctr->visits;
@@ -1220,9 +1211,9 @@ __global__ void k_pool_reset(Params p) {
   const uint64_t nring = (uint64_t)pl.nbuckets * pl.ring_len;
   for (uint64_t i = tid; i < nring; i += stride) pl.ring[i] = kEmpty;
   for (uint64_t i = tid; i < pl.nbuckets; i += stride) {
-    pl.head[i] = 0;
-    pl.cursor[i] = (i == 0 && p.direct.starts) ? p.direct.count : 0;  // direct start: W virtual positions
-    pl.claim[i] = 0;
+    pl.head[i * pl.hs] = 0;
+    pl.cursor[i * pl.hs] = (i == 0 && p.direct.starts) ? p.direct.count : 0;  // direct start: W virtual positions
+    pl.claim[i * pl.hs] = 0;
   }
   if (tid == 0) {
     *pl.free_top = (int)pl.num_chunks;
@@ -1400,8 +1391,18 @@ void launch_update_vis(const Params& p, uint32_t k, uint32_t grid, uint32_t bloc
   else launch_update_app<2, VIS>(p, k, grid, block, s);
 }
 
+template <int APP>
+void launch_update_vis3(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
+  if (p.wk.adj) launch_update_ilp<APP, 3, 1, 3>(p, k, grid, block, s);
+  else launch_update_ilp<APP, 3, 2, 3>(p, k, grid, block, s);
+}
+
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  if (p.wk.visits32) launch_update_vis<2>(p, k, grid, block, s);
+  if (p.wk.visits16) {  // the host selects VIS 3 only with an augmented layout and gather_mode 3
+    if (p.wk.app == 0) launch_update_vis3<0>(p, k, grid, block, s);
+    else if (p.wk.app == 1) launch_update_vis3<1>(p, k, grid, block, s);
+    else launch_update_vis3<2>(p, k, grid, block, s);
+  } else if (p.wk.visits32) launch_update_vis<2>(p, k, grid, block, s);
   else if (p.wk.visits) launch_update_vis<1>(p, k, grid, block, s);
   else launch_update_vis<0>(p, k, grid, block, s);
   return cudaGetLastError();
@@ -1422,9 +1423,10 @@ cudaError_t launch_gather_rows(const Params& p, const unsigned long long* rows, 
   return cudaGetLastError();
 }
 
-cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t n, const Counters* ctr, const int* free_top,
-                            unsigned long long* out_hc, Counters* out_ctr, int* out_free, cudaStream_t s) {
-  k_snapshot<<<1, 256, 0, s>>>(hc, n, ctr, free_top, out_hc, out_ctr, out_free);
+cudaError_t launch_snapshot(const unsigned long long* hc, uint64_t nb, uint32_t hs, const Counters* ctr,
+                            const int* free_top, unsigned long long* out_hc, Counters* out_ctr, int* out_free,
+                            cudaStream_t s) {
+  k_snapshot<<<1, 256, 0, s>>>(hc, nb, hs, ctr, free_top, out_hc, out_ctr, out_free);
   return cudaGetLastError();
 }
 
@@ -1469,6 +1471,51 @@ cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_
     ts.val[i] = val[i];
   }
   k_table_set<<<1, 32, 0, s>>>(table, ts, count);
+  return cudaGetLastError();
+}
+
+// VIS 3: counts[v] = hub(v) ? visits32[v] : half v & 1 of visits16[v >> 1]; the sum of all counts goes to
+// *sum (compared on the host with the number of path entries: any 16-bit wrap makes it fall short).
+__global__ void k_widen16(const uint32_t* __restrict__ v16, const uint32_t* __restrict__ v32,
+                          const unsigned long long* __restrict__ row_ptr, uint32_t hub_deg,
+                          unsigned long long* __restrict__ dst, uint64_t n, unsigned long long* sum) {
+  unsigned long long acc = 0;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t dg = (uint32_t)(row_ptr[i + 1] - row_ptr[i]);
+    const uint32_t c = dg >= hub_deg ? v32[i] : ((v16[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu);
+    dst[i] = c;
+    acc += c;
+  }
+  using BR = cub::BlockReduce<unsigned long long, 256>;
+  __shared__ typename BR::TempStorage tmp;
+  acc = BR(tmp).Sum(acc);
+  if (threadIdx.x == 0 && acc) atomicAdd(sum, acc);
+}
+
+// Exact recount from the path matrix (the fallback after a detected 16-bit wrap): counts[paths[w][t]] += 1
+// for t < lengths[w], a warp per row.
+__global__ void k_recount(const uint32_t* __restrict__ paths, uint64_t pitch, const uint32_t* __restrict__ lengths,
+                          uint64_t W, unsigned long long* __restrict__ dst) {
+  const uint64_t lane = threadIdx.x & 31u;
+  for (uint64_t w = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < W;
+       w += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint32_t L = lengths[w];
+    for (uint64_t t = lane; t < L; t += 32) atomicAdd(dst + paths[w * pitch + t], 1ull);
+  }
+}
+
+cudaError_t launch_widen16(const uint32_t* v16, const uint32_t* v32, const unsigned long long* row_ptr,
+                           uint32_t hub_deg, unsigned long long* dst, uint64_t n, unsigned long long* sum,
+                           cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_widen16<<<num_sms() * 8, 256, 0, s>>>(v16, v32, row_ptr, hub_deg, dst, n, sum);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_recount(const uint32_t* paths, uint64_t pitch, const uint32_t* lengths, uint64_t W,
+                           unsigned long long* dst, cudaStream_t s) {
+  if (!W) return cudaSuccess;
+  k_recount<<<num_sms() * 8, 256, 0, s>>>(paths, pitch, lengths, W, dst);
   return cudaGetLastError();
 }
 

@@ -52,7 +52,7 @@ lt_status snapshot(lt_ctx* ctx) {
   CK(cudaHostGetDevicePointer((void**)&dh, ctx->h_hc, 0));
   CK(cudaHostGetDevicePointer((void**)&dc, ctx->h_ctr, 0));
   CK(cudaHostGetDevicePointer((void**)&df, ctx->h_free, 0));
-  CK(launch_snapshot(ctx->d_hc, 2 * (uint64_t)ctx->nb, ctx->d_ctr, (const int*)ctx->d_small, dh, dc, df, ctx->stream));
+  CK(launch_snapshot(ctx->d_hc, ctx->nb, ctx->hs, ctx->d_ctr, (const int*)ctx->d_small, dh, dc, df, ctx->stream));
   ctx->stats.kernel_launches++;
   CK(cudaStreamSynchronize(ctx->stream));
   ctx->snap_valid = true;

@@ -85,7 +85,7 @@ class Stats(ctypes.Structure):
             "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak",
             "spill_prefetched_chunks")] + [
         ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64),
-        ("arena_bytes_used", ctypes.c_uint64)]
+        ("arena_bytes_used", ctypes.c_uint64), ("hub_deg", ctypes.c_uint64), ("visit_recounts", ctypes.c_uint64)]
 
 
 class PoolState(ctypes.Structure):

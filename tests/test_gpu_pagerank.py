@@ -142,6 +142,68 @@ def test_visit_counts_errors(gpu, cfg1):
         assert ei.value.status == 1
 
 
+# ---- paired 16-bit visit counters with hub counters (VIS 3, DESIGN.md §7 "PageRank and visit counts")
+def _deg(g):
+    rp = g.row_ptr.astype(np.int64)
+    return rp[1:] - rp[:-1]
+
+
+@pytest.mark.parametrize("layout", [LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
+@pytest.mark.parametrize("P,refill", [(1, 2), (1, 1), (8, 2), (8, 1)])
+def test_visit_counts_16bit_halves_with_hubs(gpu, cfg1, layout, P, refill):
+    """65,536 PageRank walks of length 80 on configs[0]'s graph: 5.3M path entries over ~130K CSR entries
+    put the hub degree near 100, so both counter kinds (16-bit halves, u32 hubs) and both halves of a word
+    are exercised; counts equal the oracle's bincount vertex by vertex."""
+    starts = lt_inputs.deepwalk_starts(65_536, cfg1.n)
+    _, counts, st = assert_pagerank_parity(cfg1, starts, 80, 0.15, 21, P, layout=layout, refill=refill)
+    deg = _deg(cfg1)
+    assert 64 <= st["hub_deg"] < deg.max(), st["hub_deg"]
+    hub = deg >= st["hub_deg"]
+    assert hub.any() and (~hub).any()
+    assert counts[hub].sum() > 0 and counts[~hub].sum() > 0
+    assert st["visit_recounts"] == 0
+
+
+def test_visit_counts_csr_keeps_u32(gpu, cfg1):
+    starts = lt_inputs.deepwalk_starts(2048, cfg1.n)
+    _, _, st = assert_pagerank_parity(cfg1, starts, 10, 0.15, 2, 1, layout=LT.LAYOUT_CSR)
+    assert st["hub_deg"] == 0
+
+
+@pytest.mark.parametrize("P", [1, 4])
+def test_visit_counts_16bit_wrap_is_recounted(gpu, cfg1, P):
+    """70,000 DeepWalk walks of length 3 all from one low-degree vertex: its count (>= 70,000) wraps its
+    16-bit half (and carries into the neighbour's half); the end-of-run sum check sees the shortfall and
+    the counts are recomputed from the paths, exactly."""
+    deg = _deg(cfg1)
+    pos = np.flatnonzero(deg > 0)
+    v0 = int(pos[np.argmin(deg[pos])])
+    starts = np.full(70_000, v0, dtype=np.uint32)
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, LT.DEEPWALK, 3, 4)
+        e.run()
+        counts = e.visit_counts()
+        st = e.stats()
+    assert st["hub_deg"] > deg[v0] and st["visit_recounts"] == 1
+    op, ol, _, _ = O.walks(cfg1.row_ptr, cfg1.col, starts, app=O.DEEPWALK, length=3, seed=4)
+    np.testing.assert_array_equal(counts, O.visit_counts(op, ol, cfg1.n))
+    assert counts[v0] >= 70_000
+    # without paths there is nothing to recount from: a clear error, and u64 counters (visit_counts=2) work
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ, path_mode=2) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, LT.DEEPWALK, 3, 4)
+        with pytest.raises(LT.LTError) as ei:
+            e.run()
+        assert "wrapped" in str(ei.value)
+    with LT.Engine(visit_counts=2, layout=LT.LAYOUT_ADJ, path_mode=2) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, LT.DEEPWALK, 3, 4)
+        e.run()
+        np.testing.assert_array_equal(e.visit_counts(), O.visit_counts(op, ol, cfg1.n))
+        assert e.stats()["hub_deg"] == 0
+
+
 @pytest.mark.parametrize("blocks", [1, 3])
 @pytest.mark.parametrize("zero_copy", [False, True])
 def test_pagerank_out_of_core(gpu, blocks, zero_copy):
