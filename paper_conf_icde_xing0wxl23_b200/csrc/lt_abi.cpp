@@ -14,6 +14,7 @@
 
 namespace {
 thread_local std::string g_err;
+constexpr uint64_t kXcurStride = 32;  // u64 between the two exchange-epoch cursors (256 B)
 }  // namespace
 
 namespace lt {
@@ -1155,13 +1156,14 @@ lt_status lt_exchange_buffers(lt_ctx* ctx, uint64_t capacity, void** recv, void*
       ctx->d_xbuf[e] = nullptr;
       CK(cudaMalloc(&ctx->d_xbuf[e], capacity * sizeof(uint4)));
     }
-    if (!ctx->d_xcur) CK(cudaMalloc(&ctx->d_xcur, 2 * sizeof(unsigned long long)));
-    CK(cudaMemset(ctx->d_xcur, 0, 2 * sizeof(unsigned long long)));
+    // the two epochs' cursors (every sender's append atomic lands on one of them) in separate 256-B blocks
+    if (!ctx->d_xcur) CK(cudaMalloc(&ctx->d_xcur, 2 * kXcurStride * sizeof(unsigned long long)));
+    CK(cudaMemset(ctx->d_xcur, 0, 2 * kXcurStride * sizeof(unsigned long long)));
     ctx->xcap = capacity;
   }
   for (int e = 0; e < 2; ++e) {
     recv[e] = ctx->d_xbuf[e];
-    cursor[e] = ctx->d_xcur + e;
+    cursor[e] = ctx->d_xcur + e * kXcurStride;
   }
   return LT_OK;
 }
@@ -1222,7 +1224,7 @@ lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received) {
   CK(cudaSetDevice(ctx->cfg.device));
   const uint32_t e = ctx->peer_epoch;
   unsigned long long cnt = 0;
-  CK(cudaMemcpyAsync(&cnt, ctx->d_xcur + e, sizeof(cnt), cudaMemcpyDeviceToHost, ctx->stream));
+  CK(cudaMemcpyAsync(&cnt, ctx->d_xcur + e * kXcurStride, sizeof(cnt), cudaMemcpyDeviceToHost, ctx->stream));
   CK(cudaStreamSynchronize(ctx->stream));
   if (cnt > ctx->xcap) return fail(LT_ERR_INVALID, "a peer receive buffer overflowed; raise its capacity");
   if (cnt) {
@@ -1232,7 +1234,7 @@ lt_status lt_exchange_take(lt_ctx* ctx, uint64_t* received) {
   }
   // stream-ordered after the insert: the buffer of epoch e is written again only in superstep s + 2,
   // whose senders start after this rank's next lt_run (hence this reset) has completed
-  CK(cudaMemsetAsync(ctx->d_xcur + e, 0, sizeof(unsigned long long), ctx->stream));
+  CK(cudaMemsetAsync(ctx->d_xcur + e * kXcurStride, 0, sizeof(unsigned long long), ctx->stream));
   CK(cudaMemsetAsync(&ctx->d_ctr->sent, 0, sizeof(unsigned long long), ctx->stream));
   ctx->snap_valid = false;
   ctx->peer_epoch ^= 1u;
@@ -1252,8 +1254,8 @@ lt_status lt_superstep_p2p(lt_ctx* ctx, unsigned long long* d_sent) {
   cudaStream_t s = ctx->stream;
   // (1) the walks peers appended in the previous superstep (parity epoch ^ 1) into the owned bucket
   const uint32_t prev = ctx->peer_epoch ^ 1u;
-  CK(lt::launch_insert_records_dev(ctx->params, ctx->d_xbuf[prev], ctx->d_xcur + prev, s));
-  CK(cudaMemsetAsync(ctx->d_xcur + prev, 0, sizeof(unsigned long long), s));
+  CK(lt::launch_insert_records_dev(ctx->params, ctx->d_xbuf[prev], ctx->d_xcur + prev * kXcurStride, s));
+  CK(cudaMemsetAsync(ctx->d_xcur + prev * kXcurStride, 0, sizeof(unsigned long long), s));
   CK(cudaMemsetAsync(&ctx->d_ctr->sent, 0, sizeof(unsigned long long), s));
   // (2) every owned walk steps until it ends or leaves for a peer (parity epoch), in one launch: the
   // owned bucket is the only one this rank consumes and walks stay in the kernel while inside it

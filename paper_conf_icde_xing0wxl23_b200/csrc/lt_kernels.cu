@@ -108,7 +108,11 @@ __device__ uint32_t wait_chunk(const Params& p, uint32_t dest, unsigned long lon
 }
 
 // a5: warp-collective append of the lanes with `active` set to bucket `dest`.
-__device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32_t dest, uint4 rec) {
+// Records for another rank are counted into *sent_acc (a shared-memory counter of the CTA that the update
+// kernels add to ctr->sent once at their end: one global atomic per group on one counter would serialise
+// the peer path the way one shared cursor line did); without it straight into ctr->sent.
+__device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32_t dest, uint4 rec,
+                                            unsigned long long* sent_acc = nullptr) {
   const uint32_t act = __ballot_sync(kFull, active);
   if (act == 0 || !active) return;
   const Pool& pl = p.pool;
@@ -131,7 +135,8 @@ __device__ __forceinline__ void insert_warp(const Params& p, bool active, uint32
       const uint32_t cnt = __popc(grp);
       base = atomicAdd(p.peer.cursor[slot], (unsigned long long)cnt);
       if (base + cnt > p.peer.cap) atomicOr(&p.ctr->err, kErrPeer);
-      atomicAdd(&p.ctr->sent, (unsigned long long)cnt);
+      if (sent_acc) atomicAdd(sent_acc, (unsigned long long)cnt);
+      else atomicAdd(&p.ctr->sent, (unsigned long long)cnt);
     }
     base = __shfl_sync(grp, base, leader);
     if (base + rank < p.peer.cap) p.peer.recv[slot][base + rank] = rec;
@@ -541,6 +546,9 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
   const Policies pol = make_policies();
   const uint64_t pol_last = VIS ? make_evict_last() : 0;
   unsigned long long my_steps = 0, my_trunc = 0;
+  __shared__ unsigned long long s_sent;
+  if (threadIdx.x == 0) s_sent = 0;
+  __syncthreads();
 
   for (unsigned long long base = head + ((uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * (32 * ILP);
        base < tail; base += nwarps * (32 * ILP)) {
@@ -710,13 +718,15 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
           my_trunc += trunc[s] ? 1 : 0;
         }
       }
-      insert_warp(p, had && left[s], dest, rec[s]);
+      insert_warp(p, had && left[s], dest, rec[s], &s_sent);
     }
   }
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
   if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
   if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
+  __syncthreads();
+  if (threadIdx.x == 0 && s_sent) atomicAdd(&p.ctr->sent, s_sent);
   last_cta_retire(p, (int)k, head, tail);
 }
 
@@ -740,11 +750,12 @@ template <int APP> struct RfMinBlocks {
 };
 
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
-__device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt) {
+__device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt,
+                                             unsigned long long* sent_acc) {
   const uint32_t lane = threadIdx.x & 31u;
   for (uint32_t r = 0; r < cnt; r += 32) {
     const bool act = r + lane < cnt;
-    insert_warp(p, act, act ? qd[r + lane] : 0u, act ? qr[r + lane] : make_uint4(0, 0, 0, 0));
+    insert_warp(p, act, act ? qd[r + lane] : 0u, act ? qr[r + lane] : make_uint4(0, 0, 0, 0), sent_acc);
   }
   __syncwarp();
 }
@@ -772,6 +783,9 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   const Policies pol = make_policies();
   const uint64_t pol_last = VIS ? make_evict_last() : 0;
   unsigned long long my_steps = 0, my_trunc = 0;
+  __shared__ unsigned long long s_sent;
+  if (threadIdx.x == 0) s_sent = 0;
+  __syncthreads();
 
   bool has = false;
   uint4 rec = make_uint4(0, 0, 0, 0);  // .x = row, .y = v, .z = t
@@ -964,17 +978,19 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
     q_cnt += __popc(lm);
     if (q_cnt >= 32) {
       __syncwarp();
-      flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
+      flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
       q_cnt = 0;
     }
     if (ended) has = false;
   }
   __syncwarp();
-  flush_staged(p, s_qr[wib], s_qd[wib], q_cnt);
+  flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
   if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
   if (lane == 0 && my_trunc) atomicAdd(&p.ctr->truncated, my_trunc);
+  __syncthreads();
+  if (threadIdx.x == 0 && s_sent) atomicAdd(&p.ctr->sent, s_sent);
   last_cta_retire(p, (int)k, head, tail);
 }
 
