@@ -89,6 +89,7 @@ def parse():
                     help="> 0: out-of-core mode, CSR in pinned host memory, device graph pool of this size")
     ap.add_argument("--zero-copy", type=int, default=1, help="out-of-core: adaptive zero copy (PAPER.md:265)")
     ap.add_argument("--ooc-prefetch", type=int, default=1, help="out-of-core: load the next partition during a compute")
+    ap.add_argument("--ooc-compress", type=int, default=1, help="out-of-core: partitions travel as compressed column blocks")
     ap.add_argument("--continue-resident", type=int, default=1,
                     help="out-of-core: walks keep stepping into partitions resident in the graph pool (f4)")
     ap.add_argument("--app", default="config", choices=["config", "deepwalk", "ppr", "pagerank"],
@@ -390,7 +391,8 @@ def main():
                     graph_pool_bytes=int(args.graph_pool_gb * 2 ** 30), zero_copy=bool(args.zero_copy),
                     rank=rank if own else 0, world=world if own else 1, refill=args.refill,
                     continue_resident=bool(args.continue_resident), direct_start=bool(args.direct_start),
-                    l2_persist=args.l2_persist, ooc_prefetch=bool(args.ooc_prefetch))
+                    l2_persist=args.l2_persist, ooc_prefetch=bool(args.ooc_prefetch),
+                    ooc_compress=bool(args.ooc_compress))
     torch.cuda.empty_cache()  # generator scratch back to the device before the library reserves its graph
     t0 = time.time()
     eng.graph_load(g.row_ptr, g.col, P)
@@ -605,7 +607,12 @@ def main():
                      "preemptive_launches": last["preemptive_launches"], "prefetches": last["prefetches"],
                      "hit_rate": last["pool_hits"] / max(1, last["iterations"]),
                      "continue_resident": bool(args.continue_resident),
-                     "visits_per_step": last["visits"] / max(1, last["steps"])}
+                     "visits_per_step": last["visits"] / max(1, last["steps"]),
+                     # compressed partition transfers: raw CSR bytes delivered per byte over the link
+                     "ooc_compress": bool(args.ooc_compress),
+                     "graph_h2d_raw_bytes_per_step": sum(s["graph_h2d_raw_bytes"] for s in stats) / len(stats),
+                     "compression_ratio": (sum(s["graph_h2d_raw_bytes"] for s in stats) / gb) if gb else None,
+                     "ooc_compressed_host_bytes": last["ooc_compressed_bytes"]}
 
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0 and not own and vis:

@@ -167,6 +167,13 @@ typedef struct lt_config {
                                  buffers shared through CUDA IPC (lt_exchange_buffers; lt_paths_buffers is
                                  refused) nor for the temporaries of lt_get_paths_rows. */
   uint64_t arena_bytes;
+  uint32_t ooc_compress;      /* out-of-core: 0 auto -> a partition copied into the graph pool travels as
+                                 compressed column blocks (32 entries: first value + zigzag deltas
+                                 bit-packed at the block's width), expanded by a decode kernel on the
+                                 load stream; partitions that would not shrink travel raw. Built once by
+                                 lt_graph_load* (host threads). 1 -> off (raw CSR slices). The graph the
+                                 steps read is identical either way (DESIGN.md §7 "Compressed partition
+                                 transfers"). */
 } lt_config;
 
 typedef struct lt_stats {
@@ -224,6 +231,9 @@ typedef struct lt_stats {
                                   < hub_deg, u32 for the rest (chosen at lt_walks_init) */
   uint64_t visit_recounts;     /* 1 if a 16-bit counter wrapped and the counts were recomputed from the
                                   paths at the end of lt_run (exact either way) */
+  uint64_t graph_h2d_raw_bytes;/* out-of-core: CSR bytes of the partitions copied (graph_h2d_bytes is what
+                                  crossed the link: smaller with lt_config.ooc_compress) */
+  uint64_t ooc_compressed_bytes;/* out-of-core: host bytes of the compressed column blocks (0: off) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,
@@ -363,7 +373,7 @@ lt_status lt_exchange_insert(lt_ctx* ctx, const void* d_recv, uint64_t count);
  * the loop) -> lt_exchange_take (insert what arrived, reset that cursor, flip the parity).
  * Every rank must take in every superstep so that the parities stay aligned. */
 /* This rank's buffers: recv[e] (capacity records) and cursor[e] for e = 0, 1; cursor[1] is
- * cursor[0] + 8 bytes (one allocation). Reallocated only when the capacity changes (not once attached).
+ * cursor[0] + 256 bytes (one allocation; each cursor in its own 256-B block). Reallocated only when the capacity changes (not once attached).
  * Zeroed cursors. LT_ERR_INVALID if world < 2. */
 lt_status lt_exchange_buffers(lt_ctx* ctx, uint64_t capacity, void** recv, void** cursor);
 /* Install the tables recv[e * world + q], cursor[e * world + q] (host arrays of device pointers,

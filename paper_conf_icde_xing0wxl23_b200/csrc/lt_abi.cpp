@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <atomic>
 #include <thread>
 #include <cstdio>
 #include <cstring>
@@ -107,6 +108,7 @@ lt_status lt_create(const lt_config* cfg, lt_ctx** out) {
   if (c.refill > 2) return fail(LT_ERR_INVALID, "bad refill");
   if (c.visit_counts > 2) return fail(LT_ERR_INVALID, "visit_counts must be 0, 1 or 2");
   if (c.direct_start > 1) return fail(LT_ERR_INVALID, "direct_start must be 0 (auto) or 1 (off)");
+  if (c.ooc_compress > 1) return fail(LT_ERR_INVALID, "ooc_compress must be 0 (auto) or 1 (off)");
   if (c.walk_spill > 1) return fail(LT_ERR_INVALID, "walk_spill must be 0 or 1");
   if (c.ilp != 0 && c.ilp != 1 && c.ilp != 2 && c.ilp != 4) return fail(LT_ERR_INVALID, "ilp must be 0, 1, 2 or 4");
   int ndev = 0;
@@ -176,6 +178,9 @@ static void free_ooc(lt_ctx* ctx) {
   if (o.d_table) dfree(ctx, o.d_table);
   if (o.h_row_ptr) cudaFreeHost(o.h_row_ptr);
   if (o.h_col) cudaFreeHost(o.h_col);
+  if (o.h_chdr) cudaFreeHost(o.h_chdr);
+  if (o.h_cpay) cudaFreeHost(o.h_cpay);
+  if (o.d_cstage) dfree(ctx, o.d_cstage);
   ctx->ooc = lt::OutOfCore();
 }
 
@@ -394,6 +399,99 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   return LT_OK;
 }
 
+// Compressed partition transfers (lt_config.ooc_compress): each partition's column slice is
+// cut into blocks of 32 entries; block j stores its first value and the zigzag-coded differences of
+// consecutive entries (mod 2^32, so any values round-trip), bit-packed at the block's width w (the bits of
+// the largest code) in exactly w payload words. Sorted adjacency lists give small differences, so the
+// link carries fewer bytes; a partition whose blocks would not be smaller than its raw slice travels raw.
+// Host threads build it once per lt_graph_load* (two passes: widths, then packing).
+static inline uint32_t zz(uint32_t d) { return (d << 1) ^ (uint32_t)((int32_t)d >> 31); }
+
+static lt_status compress_columns(lt_ctx* ctx, const std::vector<uint32_t>& b, uint32_t P) {
+  lt::OutOfCore& o = ctx->ooc;
+  std::vector<uint64_t> nblk(P), words(P, 0);
+  std::vector<std::vector<uint8_t>> width(P);
+  std::atomic<uint32_t> next{0};
+  auto pass1 = [&]() {
+    for (uint32_t k; (k = next.fetch_add(1)) < P;) {
+      const uint64_t e0 = o.h_row_ptr[b[k]], e1 = o.h_row_ptr[b[k + 1]], len = e1 - e0;
+      nblk[k] = (len + 31) / 32;
+      width[k].resize(nblk[k]);
+      uint64_t wsum = 0;
+      for (uint64_t j = 0; j < nblk[k]; ++j) {
+        const uint32_t* c = o.h_col + e0 + 32 * j;
+        const uint64_t L = std::min<uint64_t>(32, len - 32 * j);
+        uint32_t mx = 0;
+        for (uint64_t i = 1; i < L; ++i) mx = std::max(mx, zz(c[i] - c[i - 1]));
+        const uint8_t w = mx ? (uint8_t)(32 - __builtin_clz(mx)) : 0;
+        width[k][j] = w;
+        wsum += w;
+      }
+      words[k] = wsum;
+    }
+  };
+  const unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+  {
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < nt; ++t) th.emplace_back(pass1);
+    for (auto& x : th) x.join();
+  }
+  o.craw.assign(P, 0);
+  o.chdr_at.assign(P + 1, 0);
+  o.cpay_at.assign(P + 1, 0);
+  uint64_t stage = 0;
+  for (uint32_t k = 0; k < P; ++k) {
+    const uint64_t raw = 4ull * (o.h_row_ptr[b[k + 1]] - o.h_row_ptr[b[k]]);
+    const uint64_t comp = 8ull * (nblk[k] + 1) + 4ull * words[k];
+    if (words[k] >= 0xFFFFFFFFull || comp >= raw) {
+      o.craw[k] = 1;
+      nblk[k] = 0;
+      words[k] = 0;
+    } else {
+      stage = std::max<uint64_t>(stage, comp);
+    }
+    o.chdr_at[k + 1] = o.chdr_at[k] + (o.craw[k] ? 0 : nblk[k] + 1);
+    o.cpay_at[k + 1] = o.cpay_at[k] + words[k];
+  }
+  if (!stage) return LT_OK;  // nothing shrinks: raw copies only
+  CK(cudaHostAlloc((void**)&o.h_chdr, o.chdr_at[P] * sizeof(uint2), cudaHostAllocPortable));
+  CK(cudaHostAlloc((void**)&o.h_cpay, std::max<uint64_t>(o.cpay_at[P], 1) * 4, cudaHostAllocPortable));
+  next = 0;
+  auto pass2 = [&]() {
+    for (uint32_t k; (k = next.fetch_add(1)) < P;) {
+      if (o.craw[k]) continue;
+      const uint64_t e0 = o.h_row_ptr[b[k]], len = o.h_row_ptr[b[k + 1]] - e0;
+      uint2* hdr = o.h_chdr + o.chdr_at[k];
+      uint32_t* pay = o.h_cpay + o.cpay_at[k];
+      uint64_t off = 0;
+      for (uint64_t j = 0; j < nblk[k]; ++j) {
+        const uint32_t* c = o.h_col + e0 + 32 * j;
+        const uint64_t L = std::min<uint64_t>(32, len - 32 * j);
+        const uint32_t w = width[k][j];
+        hdr[j] = make_uint2(c[0], (uint32_t)off);
+        for (uint32_t q = 0; q < w; ++q) pay[off + q] = 0;
+        for (uint64_t i = 1; i < L && w; ++i) {
+          const uint64_t z = zz(c[i] - c[i - 1]), bit = i * w;
+          pay[off + (bit >> 5)] |= (uint32_t)(z << (bit & 31));
+          if ((bit & 31) + w > 32) pay[off + (bit >> 5) + 1] |= (uint32_t)(z >> (32 - (bit & 31)));
+        }
+        off += w;
+      }
+      hdr[nblk[k]] = make_uint2(0, (uint32_t)off);  // sentinel: the last block's width
+    }
+  };
+  {
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < nt; ++t) th.emplace_back(pass2);
+    for (auto& x : th) x.join();
+  }
+  o.cstage_bytes = (stage + 255) & ~255ull;
+  CK(dmalloc(ctx, (void**)&o.d_cstage, o.cstage_bytes));
+  o.comp = true;
+  o.comp_bytes = 8ull * o.chdr_at[P] + 4ull * o.cpay_at[P];
+  return LT_OK;
+}
+
 // Out-of-core graph (a7/a8): G_cpu is a pinned, mapped host copy of the CSR;
 // the device graph pool holds m_g blocks, each big enough for the largest partition's row_ptr slice
 // (at offset 0) plus col slice (at rp_bytes).
@@ -429,6 +527,10 @@ static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   }
   o.rp_bytes = (rp_max + 255) & ~255ull;
   o.block_bytes = (o.rp_bytes + col_max + 255) & ~255ull;
+  if (ctx->cfg.ooc_compress == 0 && m) {
+    lt_status cs = compress_columns(ctx, b, P);
+    if (cs != LT_OK) return cs;
+  }
   uint64_t mg = ctx->cfg.graph_pool_bytes / o.block_bytes;
   if (mg == 0)
     return fail(LT_ERR_INVALID, "graph pool smaller than one partition (" + std::to_string(o.block_bytes) +
@@ -451,6 +553,7 @@ static lt_status setup_out_of_core(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   o.on = true;
   ctx->stats.pool_blocks = o.m_g;
   ctx->stats.pool_block_bytes = o.block_bytes;
+  ctx->stats.ooc_compressed_bytes = o.comp_bytes;
   return LT_OK;
 }
 
@@ -764,6 +867,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   ctx->stats.preemptive_launches = 0;
   ctx->stats.prefetches = 0;
   ctx->stats.graph_h2d_bytes = 0;
+  ctx->stats.graph_h2d_raw_bytes = 0;
   ctx->stats.run_ms = 0;
   ctx->stats.chunks_free_min = num_chunks;
   ctx->stats.spilled_chunks = 0;

@@ -57,6 +57,17 @@ struct OutOfCore {
   // its host mirror
   uint32_t* d_table = nullptr;
   std::vector<uint32_t> table;
+  // compressed column slices (lt_config.ooc_compress): partition k's slice in blocks of 32 entries, header
+  // j = {first value, payload word offset from the partition's first payload word} (nblk + 1 headers, the
+  // last a sentinel), payload = the block's zigzag deltas bit-packed at width w = next offset - offset
+  bool comp = false;
+  uint2* h_chdr = nullptr;                 // pinned: every partition's headers
+  uint32_t* h_cpay = nullptr;              // pinned: every partition's payload words
+  std::vector<uint64_t> chdr_at, cpay_at;  // per partition: first header / first payload word
+  std::vector<uint8_t> craw;               // per partition: 1 = copied raw (compression saves nothing)
+  char* d_cstage = nullptr;                // device staging of one partition's compressed slice
+  size_t cstage_bytes = 0;
+  uint64_t comp_bytes = 0;
 };
 
 // Walk spill (lt_config.walk_spill): the walk pool keeps at most its

@@ -174,6 +174,7 @@ cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_
                              cudaStream_t s);  // table[idx[i]] = val[i], count <= kTableSetMax
 constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
+cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t len, uint32_t* out, cudaStream_t s);
 cudaError_t launch_widen16(const uint32_t* v16, const uint32_t* v32, const unsigned long long* row_ptr,
                            uint32_t hub_deg, unsigned long long* dst, uint64_t n, unsigned long long* sum,
                            cudaStream_t s);

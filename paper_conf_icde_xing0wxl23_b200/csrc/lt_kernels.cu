@@ -1535,6 +1535,43 @@ cudaError_t launch_recount(const uint32_t* paths, uint64_t pitch, const uint32_t
   return cudaGetLastError();
 }
 
+// Compressed partition transfer (lt_config.ooc_compress): a warp per block of 32 column entries. Lane i
+// extracts its w-bit zigzag delta (bits [i w, (i+1) w) of the block's payload; lane 0's delta is 0), the
+// warp's inclusive prefix sum (mod 2^32) plus the block's first value gives entry i.
+__global__ void k_decode_cols(const uint2* __restrict__ hdr, const uint32_t* __restrict__ pay, uint64_t len,
+                              uint32_t* __restrict__ out) {
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint64_t nblk = (len + 31) >> 5;
+  for (uint64_t j = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; j < nblk;
+       j += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    const uint2 h = hdr[j];
+    const uint32_t w = hdr[j + 1].y - h.y;
+    uint32_t z = 0;
+    if (w) {
+      const uint32_t bit = lane * w, wi = bit >> 5, sh = bit & 31u;
+      uint64_t x = pay[h.y + wi];
+      if (sh + w > 32) x |= (uint64_t)pay[h.y + wi + 1] << 32;
+      z = (uint32_t)(x >> sh) & (w == 32 ? 0xFFFFFFFFu : ((1u << w) - 1u));
+    }
+    uint32_t v = (z >> 1) ^ (0u - (z & 1u));  // unzigzag: the delta mod 2^32
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(kFull, v, o);
+      if (lane >= (uint32_t)o) v += y;
+    }
+    const uint64_t i = (j << 5) + lane;
+    if (i < len) out[i] = h.x + v;
+  }
+}
+
+cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t len, uint32_t* out, cudaStream_t s) {
+  if (!len) return cudaSuccess;
+  const uint64_t warps = (len + 31) >> 5;
+  const uint32_t grid = (uint32_t)std::min<uint64_t>((warps + 7) / 8, (uint64_t)num_sms() * 16);
+  k_decode_cols<<<grid, 256, 0, s>>>(hdr, pay, len, out);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s) {
   if (!n) return cudaSuccess;
   k_widen<<<num_sms() * 8, 256, 0, s>>>(src, dst, n);

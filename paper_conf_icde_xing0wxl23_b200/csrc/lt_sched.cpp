@@ -399,6 +399,14 @@ uint64_t partition_bytes(const lt_ctx* ctx, uint32_t k) {
   return 8ull * (v1 - v0 + 1) + 4ull * (ctx->ooc.h_row_ptr[v1] - ctx->ooc.h_row_ptr[v0]);
 }
 
+// bytes an explicit copy of partition k moves over the link (its compressed blocks when they are smaller)
+uint64_t transfer_bytes(const lt_ctx* ctx, uint32_t k) {
+  const OutOfCore& o = ctx->ooc;
+  if (!o.comp || o.craw[k]) return partition_bytes(ctx, k);
+  const uint32_t v0 = ctx->h_bounds[k], v1 = ctx->h_bounds[k + 1];
+  return 8ull * (v1 - v0 + 1) + 8ull * (o.chdr_at[k + 1] - o.chdr_at[k]) + 4ull * (o.cpay_at[k + 1] - o.cpay_at[k]);
+}
+
 // Params whose graph view is partition k's slice in block b, or the whole mapped host CSR.
 Params view_block(const lt_ctx* ctx, uint32_t k, int b) {
   Params p = ctx->params;
@@ -468,8 +476,19 @@ lt_status load_partition(lt_ctx* ctx, uint32_t k, int b, uint64_t seq) {
   Range rg("lt load partition (H2D)");
   if (ctx->cfg.timing) CK(ctx->load_ev.begin(o.load_stream));
   CK(cudaMemcpyAsync(base, o.h_row_ptr + v0, 8ull * (v1 - v0 + 1), cudaMemcpyHostToDevice, o.load_stream));
-  if (e1 > e0)
+  if (e1 > e0 && o.comp && !o.craw[k]) {  // compressed blocks into the staging buffer, expanded into the block
+    const uint64_t nh = o.chdr_at[k + 1] - o.chdr_at[k], nw = o.cpay_at[k + 1] - o.cpay_at[k];
+    CK(cudaMemcpyAsync(o.d_cstage, o.h_chdr + o.chdr_at[k], nh * sizeof(uint2), cudaMemcpyHostToDevice, o.load_stream));
+    if (nw)
+      CK(cudaMemcpyAsync(o.d_cstage + nh * sizeof(uint2), o.h_cpay + o.cpay_at[k], nw * 4, cudaMemcpyHostToDevice,
+                         o.load_stream));
+    CK(launch_decode_cols(reinterpret_cast<const uint2*>(o.d_cstage),
+                          reinterpret_cast<const uint32_t*>(o.d_cstage + nh * sizeof(uint2)), e1 - e0,
+                          reinterpret_cast<uint32_t*>(base + o.rp_bytes), o.load_stream));
+    ctx->stats.kernel_launches++;
+  } else if (e1 > e0) {
     CK(cudaMemcpyAsync(base + o.rp_bytes, o.h_col + e0, 4ull * (e1 - e0), cudaMemcpyHostToDevice, o.load_stream));
+  }
   if (ctx->cfg.timing) CK(ctx->load_ev.end(o.load_stream));
   CK(cudaEventRecord(o.ev_ready[b], o.load_stream));
   if (o.part_in[b] >= 0) o.block_of[o.part_in[b]] = -1;
@@ -477,8 +496,9 @@ lt_status load_partition(lt_ctx* ctx, uint32_t k, int b, uint64_t seq) {
   o.block_of[k] = b;
   o.loaded_at[b] = seq;
   ctx->stats.explicit_copies++;
-  ctx->stats.graph_h2d_bytes += partition_bytes(ctx, k);
-  ctx->stats.h2d_bytes += partition_bytes(ctx, k);
+  ctx->stats.graph_h2d_bytes += transfer_bytes(ctx, k);
+  ctx->stats.graph_h2d_raw_bytes += partition_bytes(ctx, k);
+  ctx->stats.h2d_bytes += transfer_bytes(ctx, k);
   return LT_OK;
 }
 
@@ -511,7 +531,7 @@ lt_status prefetch(lt_ctx* ctx, uint32_t i, bool selective, uint64_t alpha, uint
   int j = -1;
   for (uint32_t k = ctx->own_lo; k < ctx->own_hi; ++k) {
     if (k == i || o.block_of[k] >= 0 || !pending(ctx, k)) continue;
-    if (ctx->cfg.zero_copy && alpha * pending(ctx, k) < partition_bytes(ctx, k)) continue;
+    if (ctx->cfg.zero_copy && alpha * pending(ctx, k) < transfer_bytes(ctx, k)) continue;
     if (j < 0 || pending(ctx, k) > pending(ctx, (uint32_t)j)) j = (int)k;
   }
   if (j < 0) return LT_OK;
@@ -582,7 +602,7 @@ lt_status run_out_of_core(lt_ctx* ctx) {
       continue;
     }
     // adaptive scheduling: zero copy when alpha * w < S_p (Alg. 2 l.3-4)
-    if (ctx->cfg.zero_copy && alpha * pending(ctx, i) < partition_bytes(ctx, i)) {
+    if (ctx->cfg.zero_copy && alpha * pending(ctx, i) < transfer_bytes(ctx, i)) {
       ctx->stats.zero_copy_launches++;
       st = table_publish(ctx, -1);
       if (st != LT_OK) return st;

@@ -70,6 +70,7 @@ class Config(ctypes.Structure):
         ("l2_persist", ctypes.c_uint32),
         ("arena", ctypes.c_void_p),
         ("arena_bytes", ctypes.c_uint64),
+        ("ooc_compress", ctypes.c_uint32),
     ]
 
 
@@ -85,7 +86,8 @@ class Stats(ctypes.Structure):
             "spilled_chunks", "reloaded_chunks", "spill_d2h_bytes", "spill_h2d_bytes", "host_chunks_peak",
             "spill_prefetched_chunks")] + [
         ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64),
-        ("arena_bytes_used", ctypes.c_uint64), ("hub_deg", ctypes.c_uint64), ("visit_recounts", ctypes.c_uint64)]
+        ("arena_bytes_used", ctypes.c_uint64), ("hub_deg", ctypes.c_uint64), ("visit_recounts", ctypes.c_uint64),
+        ("graph_h2d_raw_bytes", ctypes.c_uint64), ("ooc_compressed_bytes", ctypes.c_uint64)]
 
 
 class PoolState(ctypes.Structure):
@@ -207,7 +209,7 @@ class Engine:
                  zc_alpha_bytes: int = 0, rank: int = 0, world: int = 1, refill: int = 0,
                  visit_counts: bool = False, continue_resident: bool = False, walk_pool_walks: int = 0,
                  direct_start: bool = True, l2_persist: int = 0, ooc_prefetch: bool = False,
-                 walk_spill: bool = False, arena=None):
+                 walk_spill: bool = False, arena=None, ooc_compress: bool = True):
         cfg = Config()
         _check(_lib.lt_config_default(ctypes.byref(cfg)))
         cfg.device = device
@@ -240,6 +242,7 @@ class Engine:
         self._arena_keep = arena
         cfg.direct_start = 0 if direct_start else 1  # 0 auto (on where it applies), 1 off
         cfg.l2_persist = int(l2_persist)
+        cfg.ooc_compress = 0 if ooc_compress else 1  # 0 auto (compressed partition copies), 1 off
         cfg.ooc_prefetch = int(bool(ooc_prefetch))
         cfg.visit_counts = int(visit_counts)  # False/0 off, True/1 on (auto counter width), 2 u64 counters
         self._lmax = ppr_max_len
@@ -489,7 +492,7 @@ class Engine:
     def import_buffers(self, handles):
         """Open another rank's export_buffers() handles: ([recv0, recv1], [cursor0, cursor1])."""
         r0, r1, c0 = (self.ipc_open(h) for h in handles)
-        return [r0, r1], [c0, c0 + 8]  # cursor[1] = cursor[0] + 8 bytes (one allocation)
+        return [r0, r1], [c0, c0 + 256]  # cursor[1] = cursor[0] + 256 bytes (one allocation, lt.h)
 
     def ipc_open(self, handle: bytes) -> int:
         """Open another process's CUDA IPC handle (64 bytes) on this engine's device."""

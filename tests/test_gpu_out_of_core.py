@@ -189,3 +189,75 @@ def test_out_of_core_lane_refill_without_continuation(gpu, g14, zero_copy):
     op, ol, _, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
     np.testing.assert_array_equal(paths, op)
     np.testing.assert_array_equal(lengths, ol)
+
+
+# ---- compressed partition transfers (lt_config.ooc_compress)
+@pytest.mark.parametrize("blocks", [1, 3])
+@pytest.mark.parametrize("zero_copy", [False, True])
+def test_compressed_transfers_exact_and_smaller(gpu, g14, blocks, zero_copy):
+    """The same out-of-core run with raw and with compressed partition copies: identical paths (both
+    equal to the oracle), and on the sorted R-MAT adjacency the link carries fewer bytes than the raw
+    CSR slices it delivers."""
+    P = 16
+    starts = lt_inputs.deepwalk_starts(2 * g14.n, g14.n)
+    op, ol, _, _ = oracle_of(g14, starts, LT.DEEPWALK, 20, 1)
+    res = {}
+    for comp in (False, True):
+        paths, lengths, st = run(g14, starts, LT.DEEPWALK, 20, 1, P, blocks, zero_copy=zero_copy, ooc_compress=comp)
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+        res[comp] = st
+    off, on = res[False], res[True]
+    assert off["ooc_compressed_bytes"] == 0 and off["graph_h2d_bytes"] == off["graph_h2d_raw_bytes"]
+    assert on["ooc_compressed_bytes"] > 0
+    if on["explicit_copies"]:
+        assert on["graph_h2d_bytes"] < on["graph_h2d_raw_bytes"]
+
+
+def _csr(n, rows):
+    row_ptr = np.zeros(n + 1, dtype=np.uint64)
+    for u, nb in rows.items():
+        row_ptr[u + 1] = len(nb)
+    row_ptr = np.cumsum(row_ptr).astype(np.uint64)
+    col = np.zeros(int(row_ptr[-1]), dtype=np.uint32)
+    for u, nb in rows.items():
+        col[int(row_ptr[u]):int(row_ptr[u + 1])] = nb
+    deg = np.diff(row_ptr.astype(np.int64))
+    return lt_inputs.Graph(n, int(row_ptr[-1]), row_ptr, col, int(deg.max()), int(np.argmax(deg)))
+
+
+@pytest.mark.parametrize("P", [3, 16])
+def test_compressed_transfers_adversarial_columns(gpu, P):
+    """Unsorted neighbour lists whose consecutive entries jump across the whole ID range (n = 2^24: codes
+    of 25 bits, deltas of both signs), alternating extremes (0, n - 1), runs of equal entries (width 0),
+    degree-1 rows and rows that are not a multiple of 32 long: every block width and the partial last
+    block of a slice go through the decode kernel; paths equal the oracle."""
+    n = 1 << 24
+    rng = np.random.default_rng(5)
+    rows = {}
+    for u in range(0, 3000):
+        k = int(rng.integers(1, 70))
+        kind = u % 4
+        if kind == 0:
+            nb = rng.integers(0, n, k)
+        elif kind == 1:
+            nb = np.where(np.arange(k) % 2 == 0, 0, n - 1)
+        elif kind == 2:
+            nb = np.full(k, int(rng.integers(0, n)))
+        else:
+            nb = np.sort(rng.integers(0, n, k))
+        rows[u] = nb.astype(np.uint32)
+    # every neighbour has edges of its own (walks keep going): point the targets into [0, 3000)
+    for u in rows:
+        rows[u] = (rows[u] % 3000).astype(np.uint32) if u % 8 == 7 else rows[u]
+    for v in set(int(x) for nb in rows.values() for x in nb):
+        if v not in rows:
+            rows[v] = np.array([int(rng.integers(0, 3000))], dtype=np.uint32)
+    g = _csr(n, rows)
+    starts = np.arange(0, 3000, dtype=np.uint32)
+    op, ol, _, _ = oracle_of(g, starts, LT.DEEPWALK, 9, 3)
+    for comp in (True, False):
+        paths, lengths, st = run(g, starts, LT.DEEPWALK, 9, 3, P, 1, ooc_compress=comp)
+        np.testing.assert_array_equal(lengths, ol)
+        np.testing.assert_array_equal(paths, op)
+        assert (st["ooc_compressed_bytes"] > 0) == comp
