@@ -128,7 +128,10 @@ typedef struct lt_config {
                                  reserved at lt_walks_init* and zeroed there: every path entry (start
                                  included) adds 1 to its vertex. Read with lt_get_visit_counts*. The
                                  kernels count in u32 while no count can reach 2^32 (W * stride <
-                                 2^32) and widen at the end of lt_run — with an augmented layout in
+                                 2^32) and widen at the end of lt_run — with the ADJ layout the 2^24 - 1
+                                 highest-degree vertices count in slots packed by degree rank (the ADJ
+                                 entry carries the slot; lt_stats.visit_hot_slots), otherwise with an
+                                 augmented layout in
                                  16-bit halves for the vertices below a hub degree (lt_stats.hub_deg),
                                  a wrap detected exactly and recounted from the paths (an error under
                                  path_mode 2); 2 -> always count in u64. */
@@ -234,6 +237,8 @@ typedef struct lt_stats {
   uint64_t graph_h2d_raw_bytes;/* out-of-core: CSR bytes of the partitions copied (graph_h2d_bytes is what
                                   crossed the link: smaller with lt_config.ooc_compress) */
   uint64_t ooc_compressed_bytes;/* out-of-core: host bytes of the compressed column blocks (0: off) */
+  uint64_t visit_hot_slots;    /* visit counting with the ADJ layout: vertices whose counters are packed by
+                                  degree rank (0: not used; then hub_deg tells the mode) */
 } lt_stats;
 
 /* Fill *cfg with defaults (device 0, legacy stream, C=8192, L_max=127, selective, aggregated,

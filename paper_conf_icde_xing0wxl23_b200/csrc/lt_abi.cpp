@@ -220,6 +220,8 @@ void lt_destroy(lt_ctx* ctx) {
   dfree(ctx, ctx->d_visits);
   dfree(ctx, ctx->d_visits32);
   dfree(ctx, ctx->d_visits16);
+  dfree(ctx, ctx->d_slot);
+  dfree(ctx, ctx->d_vhot);
   dfree(ctx, ctx->d_vsum);
   dfree(ctx, ctx->d_slots);
   dfree(ctx, ctx->d_ring);
@@ -305,7 +307,10 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
   const bool fits12 = m < (1ull << 40) && dmax < (1ull << 24);
   int lay = LT_LAYOUT_CSR;
   if (!ctx->ooc.on && ml) {
-    if (ctx->cfg.layout == LT_LAYOUT_ADJ) lay = LT_LAYOUT_ADJ;
+    if (ctx->cfg.layout == LT_LAYOUT_ADJ) {
+      if (m >= (1ull << 40)) return fail(LT_ERR_INVALID, "LT_LAYOUT_ADJ needs m < 2^40 (40-bit offsets)");
+      lay = LT_LAYOUT_ADJ;
+    }
     if (ctx->cfg.layout == LT_LAYOUT_ADJ12) {
       if (!fits12) return fail(LT_ERR_INVALID, "LT_LAYOUT_ADJ12 needs m < 2^40 and every degree < 2^24");
       lay = LT_LAYOUT_ADJ12;
@@ -319,13 +324,37 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
       size_t fr = 0, tot = 0;
       CK(cudaMemGetInfo(&fr, &tot));
       const double a16 = (double)ml * 16.0, a12 = (double)ml * 12.0;
-      if (a16 <= 0.5 * (double)fr && a16 <= kGatherReach) lay = LT_LAYOUT_ADJ;
+      if (a16 <= 0.5 * (double)fr && a16 <= kGatherReach && m < (1ull << 40)) lay = LT_LAYOUT_ADJ;
       else if (fits12 && a12 <= 0.5 * (double)fr && a12 <= kGatherReach) lay = LT_LAYOUT_ADJ12;
     }
   }
+  // VIS 4 slots (visit counting on, one rank, ADJ): the kHotSlots - 1 highest-degree vertices get slots 1..,
+  // in descending degree order (a counting sort of the degrees), embedded in the ADJ entries below
+  ctx->hot_slots = 0;
+  if (lay == LT_LAYOUT_ADJ && ctx->cfg.visit_counts == 1 && ctx->world == 1 && ctx->cfg.gather_mode == 3 && n) {
+    std::vector<uint64_t> cnt(dmax + 2, 0);
+    for (uint32_t v = 0; v < n; ++v) cnt[h_row_ptr[v + 1] - h_row_ptr[v]]++;
+    // start of each degree's ranks in descending order
+    std::vector<uint64_t> at(dmax + 2, 0);
+    uint64_t acc = 0;
+    for (uint64_t dg = dmax + 1; dg-- > 0;) {
+      at[dg] = acc;
+      acc += cnt[dg];
+    }
+    std::vector<uint32_t> slot(n);
+    for (uint32_t v = 0; v < n; ++v) {
+      const uint64_t r = at[h_row_ptr[v + 1] - h_row_ptr[v]]++;
+      slot[v] = r + 1 < lt::kHotSlots ? (uint32_t)(r + 1) : 0u;
+    }
+    ctx->hot_slots = std::min<uint64_t>(n, lt::kHotSlots - 1);
+    CK(ensure(ctx, ctx->d_slot, ctx->slot_cap, n));
+    CK(cudaMemcpyAsync(ctx->d_slot, slot.data(), (size_t)n * 4, cudaMemcpyHostToDevice, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+  }
   if (lay == LT_LAYOUT_ADJ) {
     CK(ensure(ctx, ctx->d_adj, ctx->adj_cap, ml));
-    CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj, ctx->stream));
+    CK(lt::launch_build_adj(ctx->d_row_ptr, ctx->d_col, ml, ctx->d_adj, ctx->hot_slots ? ctx->d_slot : nullptr,
+                            ctx->stream));
   } else if (ctx->d_adj) {
     dfree(ctx, ctx->d_adj);
     ctx->d_adj = nullptr;
@@ -754,7 +783,12 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // still possible (e.g. all starts on one low-degree vertex); it is detected exactly and recounted.
   uint32_t hub_deg = 0;
   bool half = false;
-  if (narrow && ctx->world == 1 && !ctx->ooc.on && (ctx->d_adj || ctx->d_adj12) && ctx->cfg.gather_mode == 3 &&
+  // VIS 4 (counters by degree slot) when the ADJ entries carry slots; else VIS 3 below
+  const bool slots = narrow && ctx->hot_slots && ctx->d_adj && ctx->world == 1 && !ctx->ooc.on;
+  if (slots) {
+    CK(ensure(ctx, ctx->d_vhot, ctx->vhot_cap, lt::hot_index((uint32_t)ctx->hot_slots) + 1));
+  }
+  if (!slots && narrow && ctx->world == 1 && !ctx->ooc.on && (ctx->d_adj || ctx->d_adj12) && ctx->cfg.gather_mode == 3 &&
       ctx->m && W) {
     const double Nt = (double)W * stride;
     const double rest = (app == LT_APP_PAGERANK ? Nt * alpha : 0.0) / ctx->n + (double)W / ctx->n;
@@ -802,6 +836,8 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.wk.visits = ctx->cfg.visit_counts ? ctx->d_visits : nullptr;
   p.wk.visits32 = narrow ? ctx->d_visits32 : nullptr;
   p.wk.visits16 = half ? ctx->d_visits16 : nullptr;
+  p.wk.vhot = slots ? ctx->d_vhot : nullptr;
+  ctx->stats.visit_hot_slots = slots ? ctx->hot_slots : 0;
   p.wk.hub_deg = hub_deg;
   ctx->stats.hub_deg = hub_deg;
   ctx->stats.visit_recounts = 0;
@@ -916,6 +952,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   if (W && !home && !ctx->is_home) CK(cudaMemsetAsync(ctx->d_lengths, 0, W * sizeof(uint32_t), s));
   if (narrow) CK(cudaMemsetAsync(ctx->d_visits32, 0, (size_t)ctx->n * sizeof(uint32_t), s));
   if (half) CK(cudaMemsetAsync(ctx->d_visits16, 0, (size_t)((ctx->n + 1) / 2) * sizeof(uint32_t), s));
+  if (slots) CK(cudaMemsetAsync(ctx->d_vhot, 0, (size_t)(lt::hot_index((uint32_t)ctx->hot_slots) + 1) * sizeof(uint32_t), s));
   else if (ctx->cfg.visit_counts) CK(cudaMemsetAsync(ctx->d_visits, 0, (size_t)ctx->n * sizeof(unsigned long long), s));
   // with range ownership each rank writes only its share of every row: unwritten entries must
   // read 0xFFFFFFFF so that the cross-rank merge is an element-wise min
@@ -968,7 +1005,11 @@ lt_status lt_run(lt_ctx* ctx) {
   // Path rows hold entries 0..length-1; the 0xFFFFFFFF padding of the rest is output formatting and is
   // written lazily by the first copy-out (ensure_padded). With ownership the rows were pre-filled.
   ctx->padded = ctx->world > 1 && !ctx->is_home;
-  if (ctx->params.wk.visits16) {  // the result is u64[n]; the sum of all counts checks for a 16-bit wrap
+  if (ctx->params.wk.vhot) {  // the result is u64[n]: per-vertex counts plus the slotted ones
+    CK(lt::launch_widen_slots(ctx->params.wk.visits32, ctx->params.wk.vhot, ctx->d_slot, ctx->params.wk.visits,
+                              ctx->n, s));
+    ctx->stats.kernel_launches++;
+  } else if (ctx->params.wk.visits16) {  // the result is u64[n]; the sum of all counts checks for a 16-bit wrap
     CK(cudaMemsetAsync(ctx->d_vsum, 0, sizeof(unsigned long long), s));
     CK(lt::launch_widen16(ctx->params.wk.visits16, ctx->params.wk.visits32, ctx->d_row_ptr, ctx->params.wk.hub_deg,
                           ctx->params.wk.visits, ctx->n, ctx->d_vsum, s));

@@ -65,7 +65,17 @@ struct Walk {
                                   // with visits16: the hub counters (degree >= hub_deg)
   uint32_t* visits16;             // [ceil(n/2)] paired 16-bit counters of the non-hub vertices, or nullptr
   uint32_t hub_deg;               // degree from which a vertex counts in visits32 (visits16 on)
+  uint32_t* vhot;                 // VIS 4: [2^24] counters by degree slot (the ADJ entry's .w >> 8), or nullptr
 };
+
+constexpr uint32_t kHotSlots = 1u << 24;  // VIS 4: slots 1 .. kHotSlots - 1 (24 bits of the ADJ entry's .w)
+// VIS 4 counter index of slot s: the kHotSpread hottest slots one per 128-B line (their REDs would
+// otherwise serialise on a few L2 lines), the rest packed densely after them
+constexpr uint32_t kHotSpread = 1u << 15;
+__host__ __device__ inline uint64_t hot_index(uint32_t s) {
+  return s < kHotSpread ? (uint64_t)s * 32 : (uint64_t)kHotSpread * 32 + (s - kHotSpread);
+}
+constexpr uint64_t kHotWords = (uint64_t)kHotSpread * 32 + kHotSlots;
 
 struct Counters {
   unsigned long long steps, visits, truncated;
@@ -174,6 +184,8 @@ cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_
                              cudaStream_t s);  // table[idx[i]] = val[i], count <= kTableSetMax
 constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
+cudaError_t launch_widen_slots(const uint32_t* cold, const uint32_t* hot, const uint32_t* slot, unsigned long long* dst,
+                               uint64_t n, cudaStream_t s);
 cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t len, uint32_t* out, cudaStream_t s);
 cudaError_t launch_widen16(const uint32_t* v16, const uint32_t* v32, const unsigned long long* row_ptr,
                            uint32_t hub_deg, unsigned long long* dst, uint64_t n, unsigned long long* sum,
@@ -181,7 +193,7 @@ cudaError_t launch_widen16(const uint32_t* v16, const uint32_t* v32, const unsig
 cudaError_t launch_recount(const uint32_t* paths, uint64_t pitch, const uint32_t* lengths, uint64_t W,
                            unsigned long long* dst, cudaStream_t s);
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
-                             cudaStream_t s);
+                             const uint32_t* slot, cudaStream_t s);
 cudaError_t launch_build_adj12(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint32_t* a12,
                                cudaStream_t s);
 // resident blocks per SM of the update kernel the launch uses (refill: 0 batch, 1 lane refill)

@@ -496,8 +496,24 @@ template <> struct MinBlocks<4> { static constexpr int v = 2; };
 // The degree of the visited vertex comes with the step (the augmented entry), so choosing costs no load.
 // A 16-bit half that wraps is detected exactly at the end of lt_run (the sum of all counts falls short of
 // the number of path entries) and the counts are then recomputed from the paths.
+// VIS 4 (round 2, the ADJ layout): the hottest vertices' counters packed densely by degree rank. The ADJ
+// entry of a step carries the visited vertex's *slot* (its rank by degree + 1, for the 2^24 - 1 highest
+// degrees; 0 for the rest) in the spare bits of its offset word, so a visit through an edge counts in
+// vhot[slot] — a 64-MB array whose hot prefix (the vertices most visits go to) stays in L2 — and every
+// other visit (starts, restarts, unslotted vertices) in the per-vertex u32 array visits32. The result is
+// their sum per vertex (k_widen_slots); every count is < 2^32 (W * stride < 2^32), so nothing can wrap.
 template <int VIS>
-__device__ __forceinline__ void count_visit(const Walk& wk, uint32_t v, uint32_t deg, uint64_t pol_last) {
+__device__ __forceinline__ void count_visit(const Walk& wk, uint32_t v, uint32_t deg, uint64_t pol_last,
+                                            uint32_t slot = 0) {
+  if (VIS == 4) {
+    if (slot)
+      asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], 1, %1;" :: "l"(wk.vhot + hot_index(slot)), "l"(pol_last)
+                   : "memory");
+    else
+      asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" :: "l"(wk.visits32 + v) : "memory");
+    return;
+  }
+  (void)slot;
   if (VIS == 3) {
     if (deg >= wk.hub_deg)
       asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u32 [%0], 1, %1;" :: "l"(wk.visits32 + v), "l"(pol_last)
@@ -625,10 +641,11 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
         const uint64_t wid = wk.first_walk_id + rec[s].x;
         b[s] = philox10(make_uint4(rec[s].z, 0u, (uint32_t)wid, (uint32_t)(wid >> 32)), wk.seed_lo, wk.seed_hi);
       }
-      uint32_t nv[ILP];
+      uint32_t nv[ILP], sl[ILP];
 #pragma unroll
       for (int s = 0; s < ILP; ++s) {
         nv[s] = 0;
+        sl[s] = 0;
         if (APP == 1 && alive[s] && b[s].x < wk.T) alive[s] = false;  // terminate before moving
         const bool restart = APP == 2 && alive[s] && b[s].x < wk.T;    // PageRank: jump to a uniform vertex
         if (alive[s] && !restart && d[s] == 0) alive[s] = false;        // dead end
@@ -653,7 +670,8 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
             const uint4 e = ld_adj<GM>(wk.adj + (off[s] - wk.ebase) + idx, pol);
             nv[s] = e.x;
             d[s] = e.y;
-            off[s] = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+            off[s] = (unsigned long long)e.z | ((unsigned long long)(e.w & 0xFFu) << 32);
+            sl[s] = e.w >> 8;
           } else {
             const Adj e = ld_adj12<GM>(wk.adj12, off[s] - wk.ebase + idx, pol);
             nv[s] = e.u;
@@ -667,7 +685,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
         if (alive[s]) {
           rec[s].y = nv[s];
           rec[s].z += 1;
-          count_visit<VIS>(wk, nv[s], d[s], pol_last);
+          count_visit<VIS>(wk, nv[s], d[s], pol_last, sl[s]);
           const uint32_t t = rec[s].z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -887,7 +905,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           const uint32_t idx = ((uint32_t)m < dd) ? lemire_slow(dd, b, rec.z, (uint32_t)wid, (uint32_t)(wid >> 32),
                                                                wk.seed_lo, wk.seed_hi)
                                                   : (uint32_t)(m >> 32);
-          uint32_t nv;
+          uint32_t nv, sl = 0;
           if (restart) {
             nv = idx;
             kn = LAY != 0 && (idx - lo < span || VIS == 3);
@@ -901,7 +919,8 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
             const uint4 e = ld_adj<GM>(wk.adj + (off - wk.ebase) + idx, pol);
             nv = e.x;
             d = e.y;
-            off = (unsigned long long)e.z | ((unsigned long long)e.w << 32);
+            off = (unsigned long long)e.z | ((unsigned long long)(e.w & 0xFFu) << 32);
+            sl = e.w >> 8;
           } else {
             const Adj e = ld_adj12<GM>(wk.adj12, off - wk.ebase + idx, pol);
             nv = e.u;
@@ -910,7 +929,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           }
           rec.y = nv;
           rec.z += 1;
-          count_visit<VIS>(wk, nv, d, pol_last);
+          count_visit<VIS>(wk, nv, d, pol_last, sl);
           const uint32_t t = rec.z;
           if (wk.path_mode == 0) {
 #pragma unroll
@@ -1269,21 +1288,23 @@ int update_kernel_occupancy(uint32_t block, uint32_t ilp, uint32_t refill, uint3
   return nb > 0 ? nb : 1;
 }
 
-// Augmented adjacency (LAY 1): adj[i] = {u, deg(u), row_ptr[u] lo, row_ptr[u] hi} for u = col[i].
+// Augmented adjacency (LAY 1): adj[i] = {u, deg(u), row_ptr[u] lo, row_ptr[u] hi8 | slot(u) << 8} for u = col[i].
+// .w = row_ptr[u] bits 32..39 | slot(u) << 8 (the visit-count slot of VIS 4, 0 without; offsets < 2^40).
 __global__ void k_build_adj(const unsigned long long* __restrict__ row_ptr, const uint32_t* __restrict__ col,
-                            uint64_t m, uint4* __restrict__ adj) {
+                            uint64_t m, uint4* __restrict__ adj, const uint32_t* __restrict__ slot) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint32_t u = col[i];
     const unsigned long long o = __ldg(row_ptr + u);
     const uint32_t dg = (uint32_t)(__ldg(row_ptr + u + 1) - o);
-    adj[i] = make_uint4(u, dg, (uint32_t)o, (uint32_t)(o >> 32));
+    const uint32_t sl = slot ? __ldg(slot + u) : 0u;
+    adj[i] = make_uint4(u, dg, (uint32_t)o, (uint32_t)(o >> 32) | (sl << 8));
   }
 }
 
 cudaError_t launch_build_adj(const unsigned long long* row_ptr, const uint32_t* col, uint64_t m, uint4* adj,
-                             cudaStream_t s) {
+                             const uint32_t* slot, cudaStream_t s) {
   if (!m) return cudaSuccess;
-  k_build_adj<<<num_sms() * 8, 256, 0, s>>>(row_ptr, col, m, adj);
+  k_build_adj<<<num_sms() * 8, 256, 0, s>>>(row_ptr, col, m, adj, slot);
   return cudaGetLastError();
 }
 
@@ -1414,7 +1435,11 @@ void launch_update_vis3(const Params& p, uint32_t k, uint32_t grid, uint32_t blo
 }
 
 cudaError_t launch_update(const Params& p, uint32_t k, uint32_t grid, uint32_t block, cudaStream_t s) {
-  if (p.wk.visits16) {  // the host selects VIS 3 only with an augmented layout and gather_mode 3
+  if (p.wk.vhot) {  // the host selects VIS 4 only with the ADJ layout built with slots and gather_mode 3
+    if (p.wk.app == 0) launch_update_ilp<0, 3, 1, 4>(p, k, grid, block, s);
+    else if (p.wk.app == 1) launch_update_ilp<1, 3, 1, 4>(p, k, grid, block, s);
+    else launch_update_ilp<2, 3, 1, 4>(p, k, grid, block, s);
+  } else if (p.wk.visits16) {  // the host selects VIS 3 only with an augmented layout and gather_mode 3
     if (p.wk.app == 0) launch_update_vis3<0>(p, k, grid, block, s);
     else if (p.wk.app == 1) launch_update_vis3<1>(p, k, grid, block, s);
     else launch_update_vis3<2>(p, k, grid, block, s);
@@ -1569,6 +1594,22 @@ cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t l
   const uint64_t warps = (len + 31) >> 5;
   const uint32_t grid = (uint32_t)std::min<uint64_t>((warps + 7) / 8, (uint64_t)num_sms() * 16);
   k_decode_cols<<<grid, 256, 0, s>>>(hdr, pay, len, out);
+  return cudaGetLastError();
+}
+
+// VIS 4: counts[v] = visits32[v] + (slot[v] ? vhot[slot[v]] : 0)
+__global__ void k_widen_slots(const uint32_t* __restrict__ cold, const uint32_t* __restrict__ hot,
+                              const uint32_t* __restrict__ slot, unsigned long long* __restrict__ dst, uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t sl = slot[i];
+    dst[i] = (unsigned long long)cold[i] + (sl ? hot[hot_index(sl)] : 0u);
+  }
+}
+
+cudaError_t launch_widen_slots(const uint32_t* cold, const uint32_t* hot, const uint32_t* slot, unsigned long long* dst,
+                               uint64_t n, cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_widen_slots<<<num_sms() * 8, 256, 0, s>>>(cold, hot, slot, dst, n);
   return cudaGetLastError();
 }
 

@@ -87,7 +87,8 @@ class Stats(ctypes.Structure):
             "spill_prefetched_chunks")] + [
         ("load_ms", ctypes.c_double), ("spill_xfer_ms", ctypes.c_double), ("host_syncs", ctypes.c_uint64),
         ("arena_bytes_used", ctypes.c_uint64), ("hub_deg", ctypes.c_uint64), ("visit_recounts", ctypes.c_uint64),
-        ("graph_h2d_raw_bytes", ctypes.c_uint64), ("ooc_compressed_bytes", ctypes.c_uint64)]
+        ("graph_h2d_raw_bytes", ctypes.c_uint64), ("ooc_compressed_bytes", ctypes.c_uint64),
+        ("visit_hot_slots", ctypes.c_uint64)]
 
 
 class PoolState(ctypes.Structure):

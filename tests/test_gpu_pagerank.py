@@ -148,15 +148,15 @@ def _deg(g):
     return rp[1:] - rp[:-1]
 
 
-@pytest.mark.parametrize("layout", [LT.LAYOUT_ADJ, LT.LAYOUT_ADJ12])
 @pytest.mark.parametrize("P,refill", [(1, 2), (1, 1), (8, 2), (8, 1)])
-def test_visit_counts_16bit_halves_with_hubs(gpu, cfg1, layout, P, refill):
-    """65,536 PageRank walks of length 80 on configs[0]'s graph: 5.3M path entries over ~130K CSR entries
-    put the hub degree near 100, so both counter kinds (16-bit halves, u32 hubs) and both halves of a word
-    are exercised; counts equal the oracle's bincount vertex by vertex."""
+def test_visit_counts_16bit_halves_with_hubs(gpu, cfg1, P, refill):
+    """VIS 3 (ADJ12): 65,536 PageRank walks of length 80 on configs[0]'s graph: 5.3M path entries over ~130K
+    CSR entries put the hub degree near 100, so both counter kinds (16-bit halves, u32 hubs) and both halves
+    of a word are exercised; counts equal the oracle's bincount vertex by vertex."""
     starts = lt_inputs.deepwalk_starts(65_536, cfg1.n)
-    _, counts, st = assert_pagerank_parity(cfg1, starts, 80, 0.15, 21, P, layout=layout, refill=refill)
+    _, counts, st = assert_pagerank_parity(cfg1, starts, 80, 0.15, 21, P, layout=LT.LAYOUT_ADJ12, refill=refill)
     deg = _deg(cfg1)
+    assert st["visit_hot_slots"] == 0
     assert 64 <= st["hub_deg"] < deg.max(), st["hub_deg"]
     hub = deg >= st["hub_deg"]
     assert hub.any() and (~hub).any()
@@ -164,43 +164,100 @@ def test_visit_counts_16bit_halves_with_hubs(gpu, cfg1, layout, P, refill):
     assert st["visit_recounts"] == 0
 
 
+@pytest.mark.parametrize("P,refill", [(1, 2), (1, 1), (8, 2), (8, 1)])
+@pytest.mark.parametrize("app", ["pagerank", "deepwalk", "ppr"])
+def test_visit_counts_degree_slots(gpu, cfg1, P, refill, app):
+    """VIS 4 (ADJ): counters of the highest-degree vertices packed by degree rank, the slot carried by the
+    ADJ entry; starts, restarts and unslotted vertices count per vertex. Exact against the oracle for
+    every app, kernel and partition count."""
+    if app == "pagerank":
+        starts = lt_inputs.deepwalk_starts(20_000, cfg1.n)
+        _, counts, st = assert_pagerank_parity(cfg1, starts, 30, 0.15, 5, P, layout=LT.LAYOUT_ADJ, refill=refill)
+    else:
+        starts = (lt_inputs.deepwalk_starts(20_000, cfg1.n) if app == "deepwalk"
+                  else lt_inputs.ppr_starts(20_000, cfg1.argmax_deg))
+        with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ, refill=refill) as e:
+            e.graph_load(cfg1.row_ptr, cfg1.col, P)
+            if app == "deepwalk":
+                e.walks_init(starts, LT.DEEPWALK, 30, 5)
+            else:
+                e.walks_init(starts, LT.PPR, 0.15, 5)
+            e.run()
+            counts, st = e.visit_counts(), e.stats()
+        kw = dict(app=O.DEEPWALK, length=30) if app == "deepwalk" else dict(app=O.PPR, alpha=0.15)
+        op, ol, _, _ = O.walks(cfg1.row_ptr, cfg1.col, starts, seed=5, **kw)
+        np.testing.assert_array_equal(counts, O.visit_counts(op, ol, cfg1.n))
+    assert st["visit_hot_slots"] == cfg1.n and st["hub_deg"] == 0
+
+
+def test_visit_counts_degree_slots_beyond_2_24(gpu):
+    """More vertices than slots (n > 2^24 - 1): the lowest-degree vertices have no slot and count per
+    vertex through the same kernel. R-MAT scale 26 with 400M tuples, 1M PageRank walks of length 20;
+    exact against the oracle."""
+    import torch
+    g = lt_inputs.rmat_gpu(26, 400_000_000, seed=4)
+    assert g.n > (1 << 24)
+    rp, col = g.row_ptr.cpu().numpy().view(np.uint64), g.col.cpu().numpy().view(np.uint32)
+    starts = lt_inputs.deepwalk_starts(1_000_000, g.n)
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ) as e:
+        e.graph_load(g.row_ptr, g.col, 1)
+        e.walks_init_pagerank(torch.from_numpy(starts.view(np.int32)).cuda(), 20, 0.15, 9)
+        e.run()
+        counts, st = e.visit_counts(), e.stats()
+    op, ol, _, _ = O.walks(rp, col, starts, app=O.PAGERANK, length=20, alpha=0.15, seed=9)
+    ref = O.visit_counts(op, ol, g.n)
+    np.testing.assert_array_equal(counts, ref)
+    assert st["visit_hot_slots"] == (1 << 24) - 1
+    deg = np.diff(rp.astype(np.int64))
+    unslotted = np.argsort(-deg, kind="stable")[(1 << 24) - 1:]
+    assert ref[unslotted].sum() > 0
+
+
 def test_visit_counts_csr_keeps_u32(gpu, cfg1):
     starts = lt_inputs.deepwalk_starts(2048, cfg1.n)
     _, _, st = assert_pagerank_parity(cfg1, starts, 10, 0.15, 2, 1, layout=LT.LAYOUT_CSR)
-    assert st["hub_deg"] == 0
+    assert st["hub_deg"] == 0 and st["visit_hot_slots"] == 0
 
 
 @pytest.mark.parametrize("P", [1, 4])
 def test_visit_counts_16bit_wrap_is_recounted(gpu, cfg1, P):
-    """70,000 DeepWalk walks of length 3 all from one low-degree vertex: its count (>= 70,000) wraps its
-    16-bit half (and carries into the neighbour's half); the end-of-run sum check sees the shortfall and
-    the counts are recomputed from the paths, exactly."""
+    """VIS 3 (ADJ12): 70,000 DeepWalk walks of length 3 all from one low-degree vertex: its count
+    (>= 70,000) wraps its 16-bit half (and carries into the neighbour's half); the end-of-run sum check
+    sees the shortfall and the counts are recomputed from the paths, exactly. VIS 4 (ADJ) counts the
+    same run exactly with nothing to recount."""
     deg = _deg(cfg1)
     pos = np.flatnonzero(deg > 0)
     v0 = int(pos[np.argmin(deg[pos])])
     starts = np.full(70_000, v0, dtype=np.uint32)
-    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ) as e:
+    op, ol, _, _ = O.walks(cfg1.row_ptr, cfg1.col, starts, app=O.DEEPWALK, length=3, seed=4)
+    ref = O.visit_counts(op, ol, cfg1.n)
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ12) as e:
         e.graph_load(cfg1.row_ptr, cfg1.col, P)
         e.walks_init(starts, LT.DEEPWALK, 3, 4)
         e.run()
         counts = e.visit_counts()
         st = e.stats()
     assert st["hub_deg"] > deg[v0] and st["visit_recounts"] == 1
-    op, ol, _, _ = O.walks(cfg1.row_ptr, cfg1.col, starts, app=O.DEEPWALK, length=3, seed=4)
-    np.testing.assert_array_equal(counts, O.visit_counts(op, ol, cfg1.n))
+    np.testing.assert_array_equal(counts, ref)
     assert counts[v0] >= 70_000
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ) as e:
+        e.graph_load(cfg1.row_ptr, cfg1.col, P)
+        e.walks_init(starts, LT.DEEPWALK, 3, 4)
+        e.run()
+        np.testing.assert_array_equal(e.visit_counts(), ref)
+        assert e.stats()["visit_hot_slots"] > 0 and e.stats()["visit_recounts"] == 0
     # without paths there is nothing to recount from: a clear error, and u64 counters (visit_counts=2) work
-    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ, path_mode=2) as e:
+    with LT.Engine(visit_counts=True, layout=LT.LAYOUT_ADJ12, path_mode=2) as e:
         e.graph_load(cfg1.row_ptr, cfg1.col, P)
         e.walks_init(starts, LT.DEEPWALK, 3, 4)
         with pytest.raises(LT.LTError) as ei:
             e.run()
         assert "wrapped" in str(ei.value)
-    with LT.Engine(visit_counts=2, layout=LT.LAYOUT_ADJ, path_mode=2) as e:
+    with LT.Engine(visit_counts=2, layout=LT.LAYOUT_ADJ12, path_mode=2) as e:
         e.graph_load(cfg1.row_ptr, cfg1.col, P)
         e.walks_init(starts, LT.DEEPWALK, 3, 4)
         e.run()
-        np.testing.assert_array_equal(e.visit_counts(), O.visit_counts(op, ol, cfg1.n))
+        np.testing.assert_array_equal(e.visit_counts(), ref)
         assert e.stats()["hub_deg"] == 0
 
 
