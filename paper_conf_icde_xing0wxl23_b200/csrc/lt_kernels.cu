@@ -404,6 +404,24 @@ __device__ __forceinline__ uint4 ld_adj(const uint4* p, const Policies& pol) {
   return v;
 }
 
+// The first step of a walk (t = 0) gathers from its start vertex's adjacency with an L2 evict_last policy:
+// when many walks share a start (PPR: every walk starts at the source) those lines are re-read by every
+// walk, unlike the entries of later steps (evict_first, never reused). LT_FIRST_KEEP=0 turns it off.
+#ifndef LT_FIRST_KEEP
+#define LT_FIRST_KEEP 1
+#endif
+template <int GM>
+__device__ __forceinline__ uint4 ld_adj_step(const uint4* p, const Policies& pol, bool first) {
+  if (GM != 0 && LT_FIRST_KEEP && first) {
+    uint4 v;
+    asm volatile("{\n\t.reg .b64 pk;\n\tcreatepolicy.fractional.L2::evict_last.b64 pk, 1.0;\n\t"
+                 "ld.global.nc.L2::cache_hint.L2::64B.v4.u32 {%0, %1, %2, %3}, [%4], pk;\n\t}"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+  }
+  return ld_adj<GM>(p, pol);
+}
+
 // Compact augmented adjacency (LAY 2): entry j is 12 bytes = 3 words {u, off lo32, off hi8 | deg << 8}
 // (row_ptr[u] < 2^40, deg(u) < 2^24). Two aligned 8-B loads cover the entry wherever it starts (byte
 // 12j is 8-aligned for even j, 4 past an 8-B boundary for odd j); they fall in one 64-B block unless the
@@ -667,7 +685,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
           } else if (LAY == 0) {
             nv[s] = ld_col<GM>(wk.col + off[s] + idx, pol);
           } else if (LAY == 1) {
-            const uint4 e = ld_adj<GM>(wk.adj + (off[s] - wk.ebase) + idx, pol);
+            const uint4 e = ld_adj_step<GM>(wk.adj + (off[s] - wk.ebase) + idx, pol, rec[s].z == 0);
             nv[s] = e.x;
             d[s] = e.y;
             off[s] = (unsigned long long)e.z | ((unsigned long long)(e.w & 0xFFu) << 32);
@@ -916,7 +934,7 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           } else if (LAY == 0) {
             nv = ld_col<GM>((CONT ? c_col : wk.col) + off + idx, pol);
           } else if (LAY == 1) {
-            const uint4 e = ld_adj<GM>(wk.adj + (off - wk.ebase) + idx, pol);
+            const uint4 e = ld_adj_step<GM>(wk.adj + (off - wk.ebase) + idx, pol, rec.z == 0);
             nv = e.x;
             d = e.y;
             off = (unsigned long long)e.z | ((unsigned long long)(e.w & 0xFFu) << 32);
