@@ -483,8 +483,16 @@ static lt_status compress_columns(lt_ctx* ctx, const std::vector<uint32_t>& b, u
     o.cpay_at[k + 1] = o.cpay_at[k] + words[k];
   }
   if (!stage) return LT_OK;  // nothing shrinks: raw copies only
-  CK(cudaHostAlloc((void**)&o.h_chdr, o.chdr_at[P] * sizeof(uint2), cudaHostAllocPortable));
-  CK(cudaHostAlloc((void**)&o.h_cpay, std::max<uint64_t>(o.cpay_at[P], 1) * 4, cudaHostAllocPortable));
+  // the blocks are an optimisation: without the pinned host memory for them, partitions travel raw
+  if (cudaHostAlloc((void**)&o.h_chdr, o.chdr_at[P] * sizeof(uint2), cudaHostAllocPortable) != cudaSuccess ||
+      cudaHostAlloc((void**)&o.h_cpay, std::max<uint64_t>(o.cpay_at[P], 1) * 4, cudaHostAllocPortable) != cudaSuccess) {
+    (void)cudaGetLastError();
+    if (o.h_chdr) cudaFreeHost(o.h_chdr);
+    o.h_chdr = nullptr;
+    o.h_cpay = nullptr;
+    o.craw.assign(P, 1);
+    return LT_OK;
+  }
   next = 0;
   auto pass2 = [&]() {
     for (uint32_t k; (k = next.fetch_add(1)) < P;) {
