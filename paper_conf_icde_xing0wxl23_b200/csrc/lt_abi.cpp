@@ -221,6 +221,7 @@ void lt_destroy(lt_ctx* ctx) {
   dfree(ctx, ctx->d_visits32);
   dfree(ctx, ctx->d_visits16);
   dfree(ctx, ctx->d_slot);
+  dfree(ctx, ctx->d_vinfo);
   dfree(ctx, ctx->d_vhot);
   dfree(ctx, ctx->d_vsum);
   dfree(ctx, ctx->d_slots);
@@ -349,6 +350,8 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
     ctx->hot_slots = std::min<uint64_t>(n, lt::kHotSlots - 1);
     CK(ensure(ctx, ctx->d_slot, ctx->slot_cap, n));
     CK(cudaMemcpyAsync(ctx->d_slot, slot.data(), (size_t)n * 4, cudaMemcpyHostToDevice, ctx->stream));
+    CK(ensure(ctx, ctx->d_vinfo, ctx->vinfo_cap, n));
+    CK(lt::launch_build_vinfo(ctx->d_row_ptr, ctx->d_slot, n, ctx->d_vinfo, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
   }
   if (lay == LT_LAYOUT_ADJ) {
@@ -845,6 +848,7 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   p.wk.visits32 = narrow ? ctx->d_visits32 : nullptr;
   p.wk.visits16 = half ? ctx->d_visits16 : nullptr;
   p.wk.vhot = slots ? ctx->d_vhot : nullptr;
+  p.wk.vinfo = slots ? ctx->d_vinfo : nullptr;
   ctx->stats.visit_hot_slots = slots ? ctx->hot_slots : 0;
   p.wk.hub_deg = hub_deg;
   ctx->stats.hub_deg = hub_deg;

@@ -192,12 +192,13 @@ struct lt_ctx {
   size_t visits16_cap = 0;
   unsigned long long* d_vsum = nullptr;    // [1] sum of the widened counts (VIS 3 wrap check)
   size_t vsum_cap = 0;
-  uint64_t vis_entries = 0;                // path entries of the current walks (W + steps), for the check
   uint32_t* d_slot = nullptr;              // [n] VIS 4 visit-count slot of each vertex (0: none), or nullptr
   size_t slot_cap = 0;
   uint32_t* d_vhot = nullptr;              // [kHotSlots] VIS 4 counters by slot
   size_t vhot_cap = 0;
   uint64_t hot_slots = 0;                  // slotted vertices (the highest degrees)
+  uint4* d_vinfo = nullptr;                // [n] VIS 4 per-vertex {offset, slot, degree}
+  size_t vinfo_cap = 0;
   bool visits_ready = false;
   uint32_t* d_starts = nullptr;
   size_t starts_cap = 0;

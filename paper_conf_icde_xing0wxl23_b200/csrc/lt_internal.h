@@ -66,6 +66,7 @@ struct Walk {
   uint32_t* visits16;             // [ceil(n/2)] paired 16-bit counters of the non-hub vertices, or nullptr
   uint32_t hub_deg;               // degree from which a vertex counts in visits32 (visits16 on)
   uint32_t* vhot;                 // VIS 4: [2^24] counters by degree slot (the ADJ entry's .w >> 8), or nullptr
+  const uint4* vinfo;             // VIS 4: [n] {off lo32, off hi8 | slot << 8, deg, 0} per vertex
 };
 
 constexpr uint32_t kHotSlots = 1u << 24;  // VIS 4: slots 1 .. kHotSlots - 1 (24 bits of the ADJ entry's .w)
@@ -184,6 +185,8 @@ cudaError_t launch_table_set(uint32_t* table, const uint32_t* idx, const uint32_
                              cudaStream_t s);  // table[idx[i]] = val[i], count <= kTableSetMax
 constexpr uint32_t kTableSetMax = 32;
 cudaError_t launch_widen(const uint32_t* src, unsigned long long* dst, uint64_t n, cudaStream_t s);
+cudaError_t launch_build_vinfo(const unsigned long long* row_ptr, const uint32_t* slot, uint64_t n, uint4* vinfo,
+                               cudaStream_t s);
 cudaError_t launch_widen_slots(const uint32_t* cold, const uint32_t* hot, const uint32_t* slot, unsigned long long* dst,
                                uint64_t n, cudaStream_t s);
 cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t len, uint32_t* out, cudaStream_t s);

@@ -387,6 +387,48 @@ __device__ __forceinline__ unsigned long long ld_rp(const unsigned long long* p)
 #endif
 }
 
+// A visit's (or a restart's) offset and degree from row_ptr with augmented layouts: a random vertex, so
+// with GM != 0 each read fills a 64-B DRAM block (L2::64B) instead of a 128-B line (PageRank restarts are
+// 15 % of its steps).
+#ifndef LT_RP64
+#define LT_RP64 1
+#endif
+template <int GM>
+__device__ __forceinline__ void rp_pair(const unsigned long long* p, unsigned long long& off, uint32_t& d) {
+  if (GM == 0 || !LT_RP64) {
+    off = __ldg(p);
+    d = (uint32_t)(__ldg(p + 1) - off);
+    return;
+  }
+  unsigned long long a, b;
+  asm volatile("ld.global.nc.L2::64B.u64 %0, [%1];" : "=l"(a) : "l"(p));
+  asm volatile("ld.global.nc.L2::64B.u64 %0, [%1];" : "=l"(b) : "l"(p + 1));
+  off = a;
+  d = (uint32_t)(b - a);
+}
+
+// VIS 4: a vertex's offset, degree and counter slot from the per-vertex table vinfo = {off lo32, off hi8 |
+// slot << 8, deg, 0} (one 16-B read where rp_pair would read row_ptr twice, and the slot lets a restart or a
+// start count in the slot counters instead of a random per-vertex counter).
+#ifndef LT_VINFO
+#define LT_VINFO 1
+#endif
+template <int VIS, int GM>
+__device__ __forceinline__ void vert_info(const Walk& wk, uint32_t v, unsigned long long& off, uint32_t& d,
+                                          uint32_t& slot) {
+  if (VIS == 4 && LT_VINFO) {
+    uint4 q;
+    asm volatile("ld.global.nc.L2::64B.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(q.x), "=r"(q.y), "=r"(q.z), "=r"(q.w) : "l"(wk.vinfo + v));
+    off = (unsigned long long)q.x | ((unsigned long long)(q.y & 0xFFu) << 32);
+    d = q.z;
+    slot = q.y >> 8;
+    return;
+  }
+  rp_pair<GM>(wk.row_ptr + v, off, d);
+  slot = 0;
+}
+
 template <int GM>
 __device__ __forceinline__ uint32_t ld_col(const uint32_t* p, const Policies& pol) {
   if (GM == 0) return __ldg(p);
@@ -621,8 +663,7 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
       // written from t0 + 1 on, a partial sector)
       nb[s] = (alive[s] && !o && (rec[s].z & 7u) == 0) ? 1u : 0u;
       if (LAY != 0 && alive[s] && !o) {  // the visit's first vertex: its offset and degree from row_ptr
-        off[s] = __ldg(wk.row_ptr + rec[s].y);
-        d[s] = (uint32_t)(__ldg(wk.row_ptr + rec[s].y + 1) - off[s]);
+        rp_pair<GM>(wk.row_ptr + rec[s].y, off[s], d[s]);
       }
     }
     for (;;) {
@@ -677,10 +718,9 @@ __global__ void __launch_bounds__(256, MinBlocks<ILP>::v) k_update(Params p, uin
                                    : (uint32_t)(m >> 32);
           if (restart) {
             nv[s] = idx;
-            kn[s] = LAY != 0 && (idx - lo < span || VIS == 3);
-            if (kn[s]) {  // staying (or VIS 3: its degree picks the counter): its offset and degree
-              off[s] = __ldg(wk.row_ptr + idx);
-              d[s] = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off[s]);
+            kn[s] = LAY != 0 && (idx - lo < span || VIS >= 3);
+            if (kn[s]) {  // staying (or VIS 3 / 4: its degree / slot picks the counter): its offset and degree
+              vert_info<VIS, GM>(wk, idx, off[s], d[s], sl[s]);
             }
           } else if (LAY == 0) {
             nv[s] = ld_col<GM>(wk.col + off[s] + idx, pol);
@@ -875,11 +915,9 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
         prow = wk.paths + (uint64_t)rec.x * wk.pitch;
         pb[7] = rec.y;
         nb = (!o && (rec.z & 7u) == 0) ? 1u : 0u;
-        if (LAY != 0 && !o) {
-          off = __ldg(wk.row_ptr + rec.y);
-          d = (uint32_t)(__ldg(wk.row_ptr + rec.y + 1) - off);
-        }
-        if (sv_count) count_visit<VIS>(wk, rec.y, d, pol_last);
+        uint32_t s0 = 0;
+        if (LAY != 0 && !o) vert_info<VIS, GM>(wk, rec.y, off, d, s0);
+        if (sv_count) count_visit<VIS>(wk, rec.y, d, pol_last, s0);
         if (CONT) {  // a walk from the bucket starts in the launched partition's view
           c_rp = wk.row_ptr - wk.vbase;
           c_col = wk.col - wk.ebase;
@@ -926,11 +964,8 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
           uint32_t nv, sl = 0;
           if (restart) {
             nv = idx;
-            kn = LAY != 0 && (idx - lo < span || VIS == 3);
-            if (kn) {
-              off = __ldg(wk.row_ptr + idx);
-              d = (uint32_t)(__ldg(wk.row_ptr + idx + 1) - off);
-            }
+            kn = LAY != 0 && (idx - lo < span || VIS >= 3);
+            if (kn) vert_info<VIS, GM>(wk, idx, off, d, sl);
           } else if (LAY == 0) {
             nv = ld_col<GM>((CONT ? c_col : wk.col) + off + idx, pol);
           } else if (LAY == 1) {
@@ -1612,6 +1647,22 @@ cudaError_t launch_decode_cols(const uint2* hdr, const uint32_t* pay, uint64_t l
   const uint64_t warps = (len + 31) >> 5;
   const uint32_t grid = (uint32_t)std::min<uint64_t>((warps + 7) / 8, (uint64_t)num_sms() * 16);
   k_decode_cols<<<grid, 256, 0, s>>>(hdr, pay, len, out);
+  return cudaGetLastError();
+}
+
+// VIS 4 per-vertex table: vinfo[v] = {row_ptr[v] lo32, row_ptr[v] hi8 | slot[v] << 8, deg(v), 0}
+__global__ void k_build_vinfo(const unsigned long long* __restrict__ row_ptr, const uint32_t* __restrict__ slot,
+                              uint64_t n, uint4* __restrict__ vinfo) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long o = row_ptr[i];
+    vinfo[i] = make_uint4((uint32_t)o, (uint32_t)(o >> 32) | (slot[i] << 8), (uint32_t)(row_ptr[i + 1] - o), 0u);
+  }
+}
+
+cudaError_t launch_build_vinfo(const unsigned long long* row_ptr, const uint32_t* slot, uint64_t n, uint4* vinfo,
+                               cudaStream_t s) {
+  if (!n) return cudaSuccess;
+  k_build_vinfo<<<num_sms() * 8, 256, 0, s>>>(row_ptr, slot, n, vinfo);
   return cudaGetLastError();
 }
 

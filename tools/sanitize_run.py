@@ -6,7 +6,8 @@ visit counters, out-of-core continuation, walk admission, paths off, the direct 
 path modes, device starts), the compact ADJ12 layout, slice-only ownership (CSR / ADJ / ADJ12, host and
 borrowed device graphs), the peer exchange (CSR / ADJ); round 2: O records through the lane-refill kernel at
 P > 1 and the walk spill
-(evict / reload kernels, tail-capped launches)."""
+(evict / reload kernels, tail-capped launches); second session: visit counters by degree slot and paired
+16-bit counters with a forced wrap recount, compressed partition transfers (decode kernel)."""
 import os
 import sys
 import threading
@@ -62,7 +63,9 @@ with LT.Engine() as e:
     e.run()
     e.get_paths_compact()
 # PageRank with fused visit counters (u32 and u64), the CSR and ADJ layouts, P = 1 and P = 4
-for kw in [dict(P=1, visit_counts=1), dict(P=4, visit_counts=2, layout=LT.LAYOUT_CSR), dict(P=4, visit_counts=1)]:
+# (round 2, second session: ADJ -> counters by degree slot, ADJ12 -> paired 16-bit counters)
+for kw in [dict(P=1, visit_counts=1), dict(P=4, visit_counts=2, layout=LT.LAYOUT_CSR), dict(P=4, visit_counts=1),
+           dict(P=1, visit_counts=1, layout=LT.LAYOUT_ADJ12), dict(P=4, visit_counts=1, layout=LT.LAYOUT_ADJ12)]:
     P = kw.pop("P")
     with LT.Engine(chunk_walks=256, **kw) as e:
         e.graph_load(g.row_ptr, g.col, P)
@@ -70,6 +73,20 @@ for kw in [dict(P=1, visit_counts=1), dict(P=4, visit_counts=2, layout=LT.LAYOUT
         e.run()
         e.get_paths()
         e.visit_counts()
+# a forced 16-bit wrap recounted from the paths (k_widen16 + k_recount)
+with LT.Engine(visit_counts=1, layout=LT.LAYOUT_ADJ12) as e:
+    e.graph_load(g.row_ptr, g.col, 1)
+    e.walks_init(np.full(70_000, int(np.flatnonzero(np.diff(g.row_ptr.astype(np.int64)) > 0)[-1]), dtype=np.uint32),
+                 LT.DEEPWALK, 3, 4)
+    e.run()
+    e.visit_counts()
+# compressed partition transfers (k_decode_cols) with and without zero copy, P = 16
+for zc in (False, True):
+    with LT.Engine(graph_pool_bytes=1 << 20, zero_copy=zc, chunk_walks=256, ooc_compress=True) as e:
+        e.graph_load(g14.row_ptr, g14.col, 16)
+        e.walks_init(s14[:4096], LT.DEEPWALK, 10, 1)
+        e.run()
+        e.get_paths()
 # out of core with continuation into resident partitions, and walk admission under a pool cap
 with LT.Engine(graph_pool_bytes=1 << 20, zero_copy=True, continue_resident=True, chunk_walks=256,
                walk_pool_walks=1000) as e:
