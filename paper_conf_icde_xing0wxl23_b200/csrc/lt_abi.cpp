@@ -324,6 +324,8 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
       constexpr double kGatherReach = 64.0 * (1ull << 30);
       size_t fr = 0, tot = 0;
       CK(cudaMemGetInfo(&fr, &tot));
+      // an augmented array this context already holds is replaced (or reused) by this load: count it as free
+      if (!ctx->cfg.arena) fr += ctx->adj_cap * sizeof(uint4) + ctx->adj12_cap * 4;
       const double a16 = (double)ml * 16.0, a12 = (double)ml * 12.0;
       if (a16 <= 0.5 * (double)fr && a16 <= kGatherReach && m < (1ull << 40)) lay = LT_LAYOUT_ADJ;
       else if (fits12 && a12 <= 0.5 * (double)fr && a12 <= kGatherReach) lay = LT_LAYOUT_ADJ12;
