@@ -28,12 +28,13 @@ def main():
     ap.add_argument("--chunk-walks", type=int, default=8192)
     ap.add_argument("--insert-mode", default="0")
     ap.add_argument("--parity", type=int, default=20000, help="sampled walks checked against the oracle (0: off)")
+    ap.add_argument("--walks-mult", type=float, default=1.0, help="W = mult x |V| (launch-size sensitivity)")
     a = ap.parse_args()
     import torch
     c = lt_inputs.CONFIGS[a.config]
     g = lt_inputs.rmat_gpu(c["scale"], c["tuples"], seed=1, permute=c["permute"])
     app = c["app"] if a.app == "config" else a.app
-    W = g.n
+    W = int(g.n * a.walks_mult)
     starts = (lt_inputs.deepwalk_starts(W, g.n) if app in ("deepwalk", "pagerank") else lt_inputs.ppr_starts(W, g.argmax_deg))
     sd = torch.from_numpy(starts.view(np.int32)).cuda()
     host = None
@@ -64,7 +65,7 @@ def main():
                     torch.cuda.synchronize()
                     ms = ev0.elapsed_time(ev1)
                     steps = sum(s["steps"] for s in sts)
-                    line = {"config": a.config, "app": app, "P": P, "refill": rf, "insert_mode": im,
+                    line = {"config": a.config, "app": app, "P": P, "refill": rf, "insert_mode": im, "walks": W,
                             "kernel": {0: "k_update", 1: "k_update", 2: "k_update_rf"}[rf],
                             "layout": sts[-1]["layout"], "steps_per_s": steps / (ms / 1e3), "ms_per_step": ms / a.steps,
                             "update_ms_per_step": sum(s["update_ms"] for s in sts) / a.steps,
