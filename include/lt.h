@@ -121,8 +121,9 @@ typedef struct lt_config {
                                  partitions. Every partition must fit one block
                                  (block = the largest partition's CSR slice). */
   uint32_t rank, world;       /* range ownership across ranks (see lt_exchange_pack); world 0/1 -> off */
-  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P <= 16, the measured
-                                 best), 1 off (the batch kernel), 2 on */
+  uint32_t refill;            /* lane refill in the update kernel: 0 auto (on when P <= 16, or with at most
+                                 64 buckets where its sorted flush applies: the measured best), 1 off (the
+                                 batch kernel), 2 on */
   uint32_t visit_counts;      /* 1 -> count per-vertex visit frequency ("the visit
                                  frequency of each vertex is recorded") into a u64[n] device array
                                  reserved at lt_walks_init* and zeroed there: every path entry (start

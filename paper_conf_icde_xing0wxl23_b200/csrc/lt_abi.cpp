@@ -884,7 +884,10 @@ static lt_status walks_init_impl(lt_ctx* ctx, uint64_t W, const uint32_t* starts
   // vs 7.7 ms on cfg 4 / cfg 3); with O records (round 2) also at P = 4 (15.7 vs 14.2-14.4·10^9 steps/s
   // on cfg 4, four runs), P = 16 (8.7-8.8 vs 8.4-8.6, three runs), P = 8 in one of two runs (12.7 vs 12.2;
   // 11.1 vs 11.8), tied at P = 64 and behind at P = 256 (3.8 vs 4.0), DESIGN.md §8
-  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && ctx->P <= 16) ? 1u : 0u;
+  // (second session: with the sorted flush — at most 64 buckets, C >= 128, aggregated insertion — lane refill
+  // also wins at P = 32 (11.8 vs 10.8) and P = 64 (9.8 vs 9.3), profiles/r02b_sorted_flush.txt)
+  const bool sorted_flush = ctx->nb <= 64 && ctx->cfg.chunk_walks >= 128 && ctx->cfg.insert_mode == 0;
+  p.refill = ctx->cfg.refill == 2 || (ctx->cfg.refill == 0 && (ctx->P <= 16 || sorted_flush)) ? 1u : 0u;
   if (p.cont.table) p.refill = 1;  // continuation lives in the lane-refill kernel
   if (p.refill) p.ilp = 1;
   ctx->occ = ctx->cfg.blocks_per_sm ? (int)ctx->cfg.blocks_per_sm

@@ -825,6 +825,71 @@ template <int APP> struct RfMinBlocks {
 #endif
 };
 
+// Sorted flush (LT_SORTED_FLUSH; lane refill with at most kSortBuckets buckets and C >= kStage): the warp's
+// staged departures (up to kStage) are counted per destination in shared memory, ONE cursor atomic per
+// destination reserves a contiguous run for all of them, and every record is stored at run base + its rank.
+// Against 32-lane rounds (one atomic per (round, destination) group, runs of ~2 records at P = 16) this
+// writes longer contiguous runs — whole 32-B sectors instead of partial ones the memory controller has to
+// read-modify-write — and issues fewer cursor atomics.
+#ifndef LT_SORTED_FLUSH
+#define LT_SORTED_FLUSH 1
+#endif
+constexpr uint32_t kSortBuckets = 64;
+#ifndef LT_STAGE_N
+#define LT_STAGE_N 128
+#endif
+constexpr uint32_t kStage = LT_STAGE_N;  // staged departures per warp with the sorted flush (flushed at >= kStage - 32)
+struct SortScratch {
+  uint32_t hist[kSortBuckets];
+  uint32_t c0[kSortBuckets], c1[kSortBuckets];
+  unsigned long long base[kSortBuckets];
+  uint32_t rank[kStage];
+};
+
+__device__ __forceinline__ void flush_sorted(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt,
+                                             unsigned long long* sent_acc, SortScratch& ss) {
+  const uint32_t lane = threadIdx.x & 31u;
+  const Pool& pl = p.pool;
+  const unsigned long long cmask = pl.C - 1;
+  for (uint32_t d = lane; d < kSortBuckets; d += 32) ss.hist[d] = 0;
+  __syncwarp();
+  for (uint32_t i = lane; i < cnt; i += 32) ss.rank[i] = atomicAdd(&ss.hist[qd[i]], 1u);
+  __syncwarp();
+  for (uint32_t d = lane; d < kSortBuckets; d += 32) {  // one reservation per destination with departures
+    const uint32_t n = ss.hist[d];
+    if (!n) continue;
+    if (p.peer.recv && d >= p.wk.P) {  // walks for rank q: a run in q's receive buffer (peer memory)
+      const uint32_t slot = p.peer.epoch * (pl.nbuckets - p.wk.P) + (d - p.wk.P);
+      const unsigned long long b = atomicAdd(p.peer.cursor[slot], (unsigned long long)n);
+      if (b + n > p.peer.cap) atomicOr(&p.ctr->err, kErrPeer);
+      atomicAdd(sent_acc, (unsigned long long)n);
+      ss.base[d] = b;
+      continue;
+    }
+    const unsigned long long b = atomicAdd(pl.cursor + (uint64_t)d * pl.hs, (unsigned long long)n);
+    const unsigned long long ci0 = b >> pl.c_shift, ci1 = (b + n - 1) >> pl.c_shift;  // n <= C: two chunks
+    uint32_t c1 = 0;
+    if (ci1 != ci0) c1 = install_chunk(p, d, ci1);
+    const uint32_t c0 = (b & cmask) == 0 ? install_chunk(p, d, ci0) : wait_chunk(p, d, ci0);
+    ss.base[d] = b;
+    ss.c0[d] = c0;
+    ss.c1[d] = ci1 == ci0 ? c0 : c1;
+  }
+  __syncwarp();
+  for (uint32_t i = lane; i < cnt; i += 32) {
+    const uint32_t d = qd[i];
+    const unsigned long long pos = ss.base[d] + ss.rank[i];
+    if (p.peer.recv && d >= p.wk.P) {
+      const uint32_t slot = p.peer.epoch * (pl.nbuckets - p.wk.P) + (d - p.wk.P);
+      if (pos < p.peer.cap) p.peer.recv[slot][pos] = qr[i];
+      continue;
+    }
+    const uint32_t c = ((pos >> pl.c_shift) == (ss.base[d] >> pl.c_shift)) ? ss.c0[d] : ss.c1[d];
+    pl.slots[((uint64_t)c << pl.c_shift) | (pos & cmask)] = qr[i];
+  }
+  __syncwarp();
+}
+
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt,
                                              unsigned long long* sent_acc) {
@@ -877,8 +942,12 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
   bool kn = false;  // off / d belong to the current vertex (augmented layouts; false after a restart that left)
   unsigned long long q_cur = 0, q_end = 0;  // this warp's claimed, not yet handed out positions
   bool drained = false;
-  __shared__ uint4 s_qr[8][2 * 32];     // per-warp staging of departing walks (records)
-  __shared__ uint32_t s_qd[8][2 * 32];  // and their destination buckets
+  __shared__ uint4 s_qr[8][kStage];     // per-warp staging of departing walks (records)
+  __shared__ uint32_t s_qd[8][kStage];  // and their destination buckets
+  __shared__ SortScratch s_ss[LT_SORTED_FLUSH ? 8 : 1];
+  // the sorted flush when every bucket fits its histogram and a run of kStage records spans <= 2 chunks
+  const bool sorted = LT_SORTED_FLUSH && pl.nbuckets <= kSortBuckets && pl.C >= kStage && p.insert_mode == 0;
+  const uint32_t q_lim = sorted ? kStage - 32 : 32;
   const uint32_t wib = threadIdx.x >> 5;
   uint32_t q_cnt = 0;
 #pragma unroll
@@ -1048,15 +1117,17 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
       s_qd[wib][slot] = dest;
     }
     q_cnt += __popc(lm);
-    if (q_cnt >= 32) {
+    if (q_cnt >= q_lim) {
       __syncwarp();
-      flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
+      if (sorted) flush_sorted(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent, s_ss[LT_SORTED_FLUSH ? wib : 0]);
+      else flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
       q_cnt = 0;
     }
     if (ended) has = false;
   }
   __syncwarp();
-  flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
+  if (sorted) flush_sorted(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent, s_ss[LT_SORTED_FLUSH ? wib : 0]);
+  else flush_staged(p, s_qr[wib], s_qd[wib], q_cnt, &s_sent);
   my_steps = warp_sum(my_steps);
   my_trunc = warp_sum(my_trunc);
   if (lane == 0 && my_steps) atomicAdd(&p.ctr->steps, my_steps);
