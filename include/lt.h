@@ -427,6 +427,14 @@ lt_status lt_ipc_open(lt_ctx* ctx, const void* handle, void** dptr);
  * Lets tests compare the device RNG with cuRAND's curand_Philox4x32_10. Synchronous. */
 lt_status lt_philox_device(int device, uint64_t n, const uint32_t* ctr, const uint32_t* key, uint32_t* out);
 
+/* The compressed-partition format of lt_config.ooc_compress (host encoder, for tests and tools; no GPU):
+ * col[0, len) is cut into blocks of 32 entries; block j is hdr[2j] = its first value, hdr[2j+1] = the offset
+ * of its payload in words; its width w = hdr[2(j+1)+1] - hdr[2j+1] (hdr holds ceil(len/32) + 1 entries, the
+ * last a sentinel); bits [i w, (i+1) w) of its payload (little-endian within words) hold entry i's zigzag-
+ * coded difference (col[i] - col[i-1]) mod 2^32 for i = 1..31 (entry 0 codes 0). *words receives the payload
+ * length; with pay == NULL only that is computed. Caller-owned host buffers. */
+lt_status lt_compress_columns(const uint32_t* col, uint64_t len, uint32_t* hdr, uint32_t* pay, uint64_t* words);
+
 /* Walk-pool invariants (a6), for tests and debugging; synchronizes the stream. Conservation:
  * pending + finished == num_walks; free_chunks + ring_chunks == total_chunks. */
 typedef struct lt_pool_state {

@@ -441,6 +441,33 @@ static lt_status finish_graph_load(lt_ctx* ctx, uint32_t n, uint64_t m, const ui
 // Host threads build it once per lt_graph_load* (two passes: widths, then packing).
 static inline uint32_t zz(uint32_t d) { return (d << 1) ^ (uint32_t)((int32_t)d >> 31); }
 
+// width of block j of a slice (bits of its largest zigzag code; 0 when all entries are equal)
+static inline uint32_t block_width(const uint32_t* c, uint64_t L) {
+  uint32_t mx = 0;
+  for (uint64_t i = 1; i < L; ++i) mx = std::max(mx, zz(c[i] - c[i - 1]));
+  return mx ? (uint32_t)(32 - __builtin_clz(mx)) : 0u;
+}
+
+// encode blocks [0, nblk) of a slice of len entries into hdr[nblk + 1] / pay (payload words zeroed here)
+static void encode_slice(const uint32_t* col, uint64_t len, const uint8_t* width, uint2* hdr, uint32_t* pay) {
+  const uint64_t nblk = (len + 31) / 32;
+  uint64_t off = 0;
+  for (uint64_t j = 0; j < nblk; ++j) {
+    const uint32_t* c = col + 32 * j;
+    const uint64_t L = std::min<uint64_t>(32, len - 32 * j);
+    const uint32_t w = width[j];
+    hdr[j] = make_uint2(c[0], (uint32_t)off);
+    for (uint32_t q = 0; q < w; ++q) pay[off + q] = 0;
+    for (uint64_t i = 1; i < L && w; ++i) {
+      const uint64_t z = zz(c[i] - c[i - 1]), bit = i * w;
+      pay[off + (bit >> 5)] |= (uint32_t)(z << (bit & 31));
+      if ((bit & 31) + w > 32) pay[off + (bit >> 5) + 1] |= (uint32_t)(z >> (32 - (bit & 31)));
+    }
+    off += w;
+  }
+  hdr[nblk] = make_uint2(0, (uint32_t)off);  // sentinel: the last block's width
+}
+
 static lt_status compress_columns(lt_ctx* ctx, const std::vector<uint32_t>& b, uint32_t P) {
   lt::OutOfCore& o = ctx->ooc;
   std::vector<uint64_t> nblk(P), words(P, 0);
@@ -453,13 +480,8 @@ static lt_status compress_columns(lt_ctx* ctx, const std::vector<uint32_t>& b, u
       width[k].resize(nblk[k]);
       uint64_t wsum = 0;
       for (uint64_t j = 0; j < nblk[k]; ++j) {
-        const uint32_t* c = o.h_col + e0 + 32 * j;
-        const uint64_t L = std::min<uint64_t>(32, len - 32 * j);
-        uint32_t mx = 0;
-        for (uint64_t i = 1; i < L; ++i) mx = std::max(mx, zz(c[i] - c[i - 1]));
-        const uint8_t w = mx ? (uint8_t)(32 - __builtin_clz(mx)) : 0;
-        width[k][j] = w;
-        wsum += w;
+        width[k][j] = (uint8_t)block_width(o.h_col + e0 + 32 * j, std::min<uint64_t>(32, len - 32 * j));
+        wsum += width[k][j];
       }
       words[k] = wsum;
     }
@@ -503,23 +525,7 @@ static lt_status compress_columns(lt_ctx* ctx, const std::vector<uint32_t>& b, u
     for (uint32_t k; (k = next.fetch_add(1)) < P;) {
       if (o.craw[k]) continue;
       const uint64_t e0 = o.h_row_ptr[b[k]], len = o.h_row_ptr[b[k + 1]] - e0;
-      uint2* hdr = o.h_chdr + o.chdr_at[k];
-      uint32_t* pay = o.h_cpay + o.cpay_at[k];
-      uint64_t off = 0;
-      for (uint64_t j = 0; j < nblk[k]; ++j) {
-        const uint32_t* c = o.h_col + e0 + 32 * j;
-        const uint64_t L = std::min<uint64_t>(32, len - 32 * j);
-        const uint32_t w = width[k][j];
-        hdr[j] = make_uint2(c[0], (uint32_t)off);
-        for (uint32_t q = 0; q < w; ++q) pay[off + q] = 0;
-        for (uint64_t i = 1; i < L && w; ++i) {
-          const uint64_t z = zz(c[i] - c[i - 1]), bit = i * w;
-          pay[off + (bit >> 5)] |= (uint32_t)(z << (bit & 31));
-          if ((bit & 31) + w > 32) pay[off + (bit >> 5) + 1] |= (uint32_t)(z >> (32 - (bit & 31)));
-        }
-        off += w;
-      }
-      hdr[nblk[k]] = make_uint2(0, (uint32_t)off);  // sentinel: the last block's width
+      encode_slice(o.h_col + e0, len, width[k].data(), o.h_chdr + o.chdr_at[k], o.h_cpay + o.cpay_at[k]);
     }
   };
   {
@@ -1696,3 +1702,23 @@ lt_status lt_get_stats(lt_ctx* ctx, lt_stats* out) {
 }
 
 }  // extern "C"
+
+// The compressed-partition encoder on one column slice (host only; tests and tools): *words receives the
+// payload length; hdr must hold ceil(len / 32) + 1 entries (2 u32 each: first value, payload word offset),
+// pay (may be NULL to query *words) at least *words u32.
+lt_status lt_compress_columns(const uint32_t* col, uint64_t len, uint32_t* hdr, uint32_t* pay, uint64_t* words) {
+  if ((len && !col) || !words) return fail(LT_ERR_INVALID, "NULL argument");
+  const uint64_t nblk = (len + 31) / 32;
+  std::vector<uint8_t> w(nblk);
+  uint64_t tot = 0;
+  for (uint64_t j = 0; j < nblk; ++j) {
+    w[j] = (uint8_t)block_width(col + 32 * j, std::min<uint64_t>(32, len - 32 * j));
+    tot += w[j];
+  }
+  *words = tot;
+  if (!pay) return LT_OK;
+  if (!hdr) return fail(LT_ERR_INVALID, "NULL hdr");
+  if (tot >= 0xFFFFFFFFull) return fail(LT_ERR_INVALID, "slice too large for 32-bit payload offsets");
+  encode_slice(col, len, w.data(), reinterpret_cast<uint2*>(hdr), pay);
+  return LT_OK;
+}

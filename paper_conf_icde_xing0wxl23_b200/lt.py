@@ -35,7 +35,7 @@ EXPORTED = [
     "lt_pending", "lt_exchange_pack", "lt_exchange_insert", "lt_run_to_host", "lt_walks_init_pagerank",
     "lt_get_visit_counts", "lt_get_visit_counts_device", "lt_get_paths_compact", "lt_run_to_host_compact",
     "lt_exchange_buffers", "lt_exchange_attach", "lt_exchange_sent", "lt_exchange_take", "lt_ipc_handle",
-    "lt_ipc_open", "lt_superstep_p2p", "lt_paths_buffers", "lt_paths_attach", "lt_philox_device",
+    "lt_ipc_open", "lt_superstep_p2p", "lt_paths_buffers", "lt_paths_attach", "lt_philox_device", "lt_compress_columns",
 ]
 
 
@@ -133,6 +133,18 @@ _lib.lt_superstep_p2p.argtypes = [_vp, _vp]
 _lib.lt_paths_buffers.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_vp), ctypes.POINTER(_u64)]
 _lib.lt_paths_attach.argtypes = [_vp, _vp, _vp, _u64]
 _lib.lt_philox_device.argtypes = [ctypes.c_int, _u64, _vp, _vp, _vp]
+_lib.lt_compress_columns.argtypes = [_vp, _u64, _vp, _vp, ctypes.POINTER(_u64)]
+
+
+def compress_columns(col):
+    """lt_compress_columns (host): (hdr u32[nblk + 1, 2], payload u32[words]) of a u32 column slice."""
+    col = np.ascontiguousarray(col, dtype=np.uint32)
+    words = _u64()
+    _check(_lib.lt_compress_columns(col.ctypes.data, len(col), None, None, ctypes.byref(words)))
+    hdr = np.zeros(((len(col) + 31) // 32 + 1, 2), dtype=np.uint32)
+    pay = np.zeros(max(1, words.value), dtype=np.uint32)
+    _check(_lib.lt_compress_columns(col.ctypes.data, len(col), hdr.ctypes.data, pay.ctypes.data, ctypes.byref(words)))
+    return hdr, pay[:words.value]
 
 
 def philox_device(ctr, key, device: int = 0) -> np.ndarray:

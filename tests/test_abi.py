@@ -107,3 +107,51 @@ def test_struct_layout_matches_header(tmp_path):
     sizes = [int(x) for x in subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()]
     assert sizes == [ctypes.sizeof(ltmod.Config), ctypes.sizeof(ltmod.Stats), ctypes.sizeof(ltmod.PoolState),
                      ltmod.Config.graph_pool_bytes.offset, ltmod.Stats.iterations.offset]
+
+
+# ---- compressed partition format (lt_config.ooc_compress): the host encoder against an independent decoder
+def _decode_blocks(hdr, pay, n):
+    """Decode the documented format (include/lt.h, lt_compress_columns) with plain integer arithmetic."""
+    out = np.zeros(n, dtype=np.uint64)
+    pay = [int(x) for x in pay]
+    for j in range((n + 31) // 32):
+        base, off = int(hdr[j, 0]), int(hdr[j, 1])
+        w = int(hdr[j + 1, 1]) - off
+        acc = base
+        for i in range(min(32, n - 32 * j)):
+            z = 0
+            if i and w:
+                bit = i * w
+                word = pay[off + (bit >> 5)] | ((pay[off + (bit >> 5) + 1] << 32) if (bit & 31) + w > 32 else 0)
+                z = (word >> (bit & 31)) & ((1 << w) - 1)
+            delta = (z >> 1) ^ (-(z & 1) & 0xFFFFFFFF)  # unzigzag, mod 2^32
+            acc = (acc + delta) & 0xFFFFFFFF if i else base
+            out[32 * j + i] = acc
+    return out
+
+
+@pytest.mark.parametrize("kind", ["sorted_rmat", "random_u32", "extremes", "constant", "short"])
+def test_compress_columns_roundtrip(kind):
+    rng = np.random.default_rng(11)
+    if kind == "sorted_rmat":
+        g = lt_inputs.rmat_cpu(12, 65_536, seed=1)
+        col = g.col.astype(np.uint32)
+    elif kind == "random_u32":
+        col = rng.integers(0, 1 << 32, 1000, dtype=np.uint64).astype(np.uint32)  # differences >= 2^31: w = 32
+    elif kind == "extremes":
+        col = np.where(np.arange(777) % 3 == 0, 0, 0xFFFFFFFF).astype(np.uint32)
+    elif kind == "constant":
+        col = np.full(100, 12345, dtype=np.uint32)  # width 0: no payload
+    else:
+        col = np.array([7, 3], dtype=np.uint32)
+    hdr, pay = LT.compress_columns(col)
+    assert hdr.shape == ((len(col) + 31) // 32 + 1, 2)
+    np.testing.assert_array_equal(_decode_blocks(hdr, pay, len(col)), col.astype(np.uint64))
+    widths = np.diff(hdr[:, 1].astype(np.int64))
+    assert widths.min() >= 0 and widths.max() <= 32
+    if kind == "sorted_rmat":  # sorted adjacency compresses: fewer bytes than 4 per entry
+        assert 8 * len(hdr) + 4 * len(pay) < 4 * len(col)
+    if kind == "random_u32":
+        assert widths.max() == 32
+    if kind == "constant":
+        assert len(pay) == 0
