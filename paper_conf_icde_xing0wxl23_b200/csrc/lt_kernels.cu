@@ -890,6 +890,10 @@ __device__ __forceinline__ void flush_sorted(const Params& p, const uint4* qr, c
   __syncwarp();
 }
 
+#ifndef LT_PAD_SECTOR
+#define LT_PAD_SECTOR 1
+#endif
+
 // Insert `cnt` (<= 64) staged walks, 32 lanes per round (warp-collective).
 __device__ __forceinline__ void flush_staged(const Params& p, const uint4* qr, const uint32_t* qd, uint32_t cnt,
                                              unsigned long long* sent_acc) {
@@ -1096,9 +1100,26 @@ __global__ void __launch_bounds__(256, RfMinBlocks<APP>::v) k_update_rf(Params p
     const bool ended = done || left;
     if (ended && wk.path_mode == 0) {
       const uint32_t t = rec.z;
+      const uint32_t lo8 = t & 7u;  // the open sector holds entries [t - lo8, t]
+      if (LT_PAD_SECTOR && done && nb > lo8) {
+        // the walk ended and its open sector is wholly buffered: write the sector whole, the entries past
+        // the end as the row padding (0xFFFFFFFF), instead of a partial sector the memory controller would
+        // complete by read-modify-write (PPR: one per walk)
+        uint32_t sec[8];
 #pragma unroll
-      for (int q = 0; q < 8; ++q)
-        if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
+        for (int q = 0; q < 8; ++q) {  // sec[q] = pb[7 - lo8 + q] by selects (no dynamic register indexing)
+          uint32_t v = kEmpty;
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            if ((uint32_t)j + lo8 == (uint32_t)q + 7u) v = pb[j];
+          sec[q] = v;
+        }
+        st_sector(prow + (t - lo8), sec, pol);
+      } else {
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+          if ((uint32_t)q < nb) prow[t - q] = pb[7 - q];
+      }
       nb = 0;
     }
     if (done) {
